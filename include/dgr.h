@@ -1,0 +1,214 @@
+/*
+ * dgr.h — C ABI of libdgr: one RK4 stage of fp64 BSSN on a 2:1-balanced,
+ * Morton-ordered octree (the data-parallel hot path of the GPU Dendro-GR
+ * solver, Fernando et al., SC'22; "P:Lnnn" = line nnn of the paper text).
+ *
+ * The calls follow the paper's statement of the problem:
+ *   Alg. 1  Require: u at t0, dt; Ensure: u at T —
+ *                         halo_exchange -> octant-to-patch -> RHS ->
+ *                         patch-to-octant -> AXPY            => dgr_rk4_stage / dgr_rk4_step
+ *   Alg. 2  Require: octant list, O2B, u; Ensure: u^ (patches)
+ *                                                             => dgr_unzip
+ *   §IV-B  RHS = derivatives D + algebra A        => dgr_rhs
+ *   §III-B/C octree, O2O/O2N maps, built on the host at (re)grid
+ *                         time                       => dgr_octree_build, dgr_mesh_create
+ *
+ * Conventions
+ *   - All functions are extern "C", return dgr_status, never throw.
+ *   - Device pointers are plain CUDA device addresses (e.g. torch tensors'
+ *     data_ptr()); `stream` is a cudaStream_t passed as void*.  Work is
+ *     enqueued on `stream`; functions return before it completes unless
+ *     stated otherwise.  The caller owns every state/output buffer; the
+ *     library owns the mesh (host maps, device maps, workspace, NCCL
+ *     communicator, streams/events) and frees it in dgr_mesh_destroy.
+ *   - State layout: u[f * dof_stride + d], f = 0..23 (field order below),
+ *     d = local DOF index (owned DOFs first, in global-id order, then ghost
+ *     DOFs grouped by owning rank).  fp64, SoA, 16-byte aligned.
+ *     Field order: 0 alpha, 1 chi, 2 K, 3-5 Gt^i, 6-8 beta^i, 9-11 B^i,
+ *     12-17 gt_ij, 18-23 At_ij, ij in (xx,xy,xz,yy,yz,zz).
+ *   - Patches: patches[(f * n_oct_local + e) * patch_pitch + p],
+ *     p = i + 13 j + 169 k (x fastest) over the (r+2k)^3 = 13^3 padded block
+ *     of P:L177 (r = 7, k = 3); patch_pitch >= 2197 (padded for alignment).
+ *   - Errors: arguments are validated synchronously (DGR_ERR_ARG); bad octant
+ *     lists give DGR_ERR_TREE; CUDA launch/API errors give DGR_ERR_CUDA
+ *     (asynchronous faults surface at the next synchronising call).
+ *     dgr_last_error() returns a thread-local message for the last failure.
+ *   - A mesh handle is not thread-safe.  With nranks > 1, dgr_mesh_create,
+ *     dgr_rhs, dgr_rk4_stage, dgr_rk4_step and dgr_constraints are collective:
+ *     every rank calls them in the same order (NCCL semantics).
+ */
+#ifndef DGR_H
+#define DGR_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  DGR_OK = 0,
+  DGR_ERR_ARG = -1,    /* null/misaligned pointer, bad size or index          */
+  DGR_ERR_TREE = -2,   /* octants unsorted, overlapping, incomplete, unbalanced */
+  DGR_ERR_CUDA = -3,   /* CUDA runtime error                                   */
+  DGR_ERR_NCCL = -4,   /* NCCL unavailable or failed                          */
+  DGR_ERR_OOM = -5,    /* host or device allocation failed                    */
+  DGR_ERR_STATE = -6   /* call not valid for this mesh (e.g. host-only mesh)  */
+} dgr_status;
+
+/* Leaf octant: anchor in units of width / 2^max_depth, level l has side
+ * 2^(max_depth - l) in those units (leaves only). 16 bytes. */
+typedef struct {
+  uint32_t x, y, z;
+  uint32_t level;
+} dgr_octant;
+
+/* Puncture for the refinement rule (DESIGN.md R-O1). */
+typedef struct {
+  double x, y, z, m;
+  int32_t level; /* finest level required at the puncture */
+  int32_t pad;
+} dgr_puncture;
+
+/* Inputs of dgr_octree_build: refine every octant while
+ *   level < max(level_min, max_a [L_a - j_a]),  j_a = min j>=0 with
+ *   d^2(box, x_a) <= (rho m_a)^2 4^j,
+ * then apply the minimal 2:1 vertex-balance closure and sort by Morton key
+ * (child index c = x + 2y + 4z). */
+typedef struct {
+  double xmin[3];
+  double width;
+  int32_t max_depth; /* <= 20; 18 in all shipped configs */
+  int32_t periodic;  /* 1: periodic domain, 0: extrapolating outer boundary */
+  int32_t level_min;
+  int32_t n_punct;
+  const dgr_puncture* punct; /* host array [n_punct] */
+  double rho;
+} dgr_refine_desc;
+
+/* Mesh creation options. */
+typedef struct {
+  double xmin[3];
+  double width;
+  int32_t max_depth;
+  int32_t periodic;
+  int32_t rank, nranks;   /* Morton-contiguous partition of the leaves     */
+  int32_t device;         /* 1: upload maps + allocate workspace on the current
+                             CUDA device; 0: host-only (maps/export only)  */
+  int32_t pad;
+  const void* nccl_id;    /* ncclUniqueId bytes (128) when nranks > 1      */
+} dgr_mesh_desc;
+
+/* Parameters of the RHS (readings R6, R8, R13). */
+typedef struct {
+  double ko_sigma;   /* Kreiss-Oliger strength sigma (0.4)                  */
+  double eta;        /* Gamma-driver damping eta (2.0), eq (3)              */
+  double lambda_f0;  /* f(alpha) = lambda_f0 + lambda_f1 alpha, eq (2) (1,0) */
+  double lambda_f1;
+  double chi_floor;  /* chi in every division is max(chi, chi_floor) (1e-4) */
+} dgr_params;
+
+typedef struct {
+  int64_t n_oct_global;
+  int64_t n_oct_local;   /* owned octants of this rank                      */
+  int64_t n_oct_ghost;   /* ghost octants (remote padding/hanging sources)   */
+  int64_t oct_begin;     /* global index of the first owned octant           */
+  int64_t n_dof_global;
+  int64_t n_dof_owned;
+  int64_t n_dof_ghost;
+  int64_t dof_stride;    /* >= n_dof_owned + n_dof_ghost, multiple of 32     */
+  int64_t patch_pitch;   /* doubles per patch (>= 2197)                      */
+  int64_t n_hanging;     /* hanging (octant, node) pairs over local+ghost    */
+  double h_min;          /* finest grid spacing width / (6 * 2^level_max)    */
+  int32_t level_min, level_max;
+} dgr_mesh_info;
+
+typedef struct dgr_mesh_s* dgr_mesh;
+
+/* Canonical map exports (host buffers, global indices; bit-exact contract
+ * with the oracle). */
+enum {
+  DGR_MAP_OCTANTS = 0,  /* int32 [n_oct_global][4]: x, y, z, level (Morton order)  */
+  DGR_MAP_O2N = 1,      /* int32 [n_oct_local][343]: global DOF id or -1 (hanging)  */
+  DGR_MAP_HANGING = 2,  /* int32 [n][3]: (global octant, node, global source leaf)
+                           over owned octants, sorted by (octant, node)            */
+  DGR_MAP_PAD_SRC = 3,  /* int32 [n_oct_local][2197]: global source leaf, -1 = extrap */
+  DGR_MAP_PAD_KIND = 4, /* uint8 [n_oct_local][2197]: 0 self, 1 copy, 2 inject,
+                           3 interp, 4 extrap; | 8 if reached across the periodic
+                           boundary                                                */
+  DGR_MAP_ZIP = 5,      /* int32 [n_dof_owned][2]: (global owner leaf, node)       */
+  DGR_MAP_DOF_GID = 6,  /* int64 [n_dof_owned + n_dof_ghost]: global DOF id        */
+  DGR_MAP_DOF_XYZ = 7,  /* double [3][n_dof_owned + n_dof_ghost]: coordinates      */
+  DGR_MAP_SEND = 8,     /* int32 [sum over peers]: local DOF ids sent, peer-major   */
+  DGR_MAP_SEND_COUNTS = 9, /* int64 [nranks]: DOFs sent to each peer               */
+  DGR_MAP_RECV_COUNTS = 10 /* int64 [nranks]: ghost DOFs received from each peer   */
+};
+
+const char* dgr_status_string(dgr_status s);
+const char* dgr_last_error(void);
+const char* dgr_version(void);
+
+/* Host: refine + balance + Morton sort.  Call with out = NULL to get
+ * the count in *n_inout; then with a buffer of *n_inout entries. */
+dgr_status dgr_octree_build(const dgr_refine_desc* desc, dgr_octant* out, int64_t* n_inout);
+
+/* Host (+device when desc->device): validate the octant list (sorted,
+ * complete, non-overlapping, 2:1 vertex balanced -> else DGR_ERR_TREE), build
+ * node/DOF numbering, hanging table, padding (O2P) and zip maps, partition
+ * along the Morton curve for `rank` of `nranks`, upload maps, allocate
+ * workspace.  Synchronises `stream`. */
+dgr_status dgr_mesh_create(const dgr_mesh_desc* desc, const dgr_octant* octs, int64_t n,
+                           void* stream, dgr_mesh* out);
+dgr_status dgr_mesh_info_get(dgr_mesh m, dgr_mesh_info* info);
+/* Copy map `which` to host_buf; with host_buf = NULL return the size in *nbytes. */
+dgr_status dgr_mesh_export_maps(dgr_mesh m, int which, void* host_buf, size_t* nbytes);
+dgr_status dgr_mesh_destroy(dgr_mesh m);
+
+/* Device: coordinates of the local DOFs, xyz[a * dof_stride + d]. */
+dgr_status dgr_dof_coords(dgr_mesh m, double* xyz, void* stream);
+
+/* Device: octant-to-patch (Alg. 2) of the first `nfields` fields of u into
+ * patches (layout above).  Single-rank meshes, or u whose ghost DOFs are
+ * current (see dgr_ghost_exchange). */
+dgr_status dgr_unzip(dgr_mesh m, const double* u, double* patches, int nfields, void* stream);
+
+/* Device: ghost exchange of all 24 fields of u (NCCL, nranks > 1; no-op else). */
+dgr_status dgr_ghost_exchange(dgr_mesh m, double* u, void* stream);
+
+/* Device: BSSN RHS (eqs 1-8 + KO) at the interior points of given patches
+ * (24 fields, layout above) -> rhs_oct[(f * n_oct_local + e) * 343 + n]. */
+dgr_status dgr_rhs_patches(dgr_mesh m, const double* patches, double* rhs_oct,
+                           const dgr_params* prm, void* stream);
+
+/* Device: F(u) on the owned DOFs: ghost exchange -> unzip -> RHS -> zip.
+ * rhs[f * dof_stride + d] for owned d.  u must be writable when nranks > 1
+ * (its ghost slice is refreshed). */
+dgr_status dgr_rhs(dgr_mesh m, double* u, double* rhs, const dgr_params* prm, void* stream);
+
+/* Device: RK4 stage s = 0..3 (classic tableau, reading R11).  Reads the
+ * stage state U_s (= u_n for s = 0; pass u_s == u_n), computes k = F(U_s) and
+ *   s=0: acc = u_n + dt/6 k; u_s = u_n + dt/2 k      s=1: acc += dt/3 k; u_s = u_n + dt/2 k
+ *   s=2: acc += dt/3 k;      u_s = u_n + dt k        s=3: acc += dt/6 k   (acc = u^{n+1})
+ * All three arrays are [24][dof_stride].  For s = 0, u_s may alias u_n only
+ * if the caller does not need u_n's ghost DOFs afterwards. */
+dgr_status dgr_rk4_stage(dgr_mesh m, int s, double dt, double* u_n, double* u_s, double* acc,
+                         const dgr_params* prm, void* stream);
+
+/* Device: one RK4 step in place on u (library workspace for stages). */
+dgr_status dgr_rk4_step(dgr_mesh m, double dt, double* u, const dgr_params* prm, void* stream);
+
+/* Device: constraints H, M^0..2, G^0..2 on the owned DOFs,
+ * c[q * dof_stride + d], q = 0..6; norms_host[2q] = RMS, [2q+1] = max |.|
+ * over owned DOFs (all ranks).  Synchronises `stream`. */
+dgr_status dgr_constraints(dgr_mesh m, double* u, double* c, double* norms_host,
+                           const dgr_params* prm, void* stream);
+
+/* Device-side timing helper for benchmarks: number of kernel launches the last
+ * dgr_rk4_step / dgr_rhs enqueued. */
+int64_t dgr_last_launch_count(dgr_mesh m);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DGR_H */

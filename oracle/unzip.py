@@ -121,9 +121,16 @@ def elements(mesh: OracleMesh, u: np.ndarray, chunk=20000) -> np.ndarray:
 def unzip(mesh: OracleMesh, u: np.ndarray, octs=None, chunk=4000) -> np.ndarray:
     """Patches [nf, n, 13, 13, 13] (index [z][y][x]) of octants `octs` (default all)."""
     E = elements(mesh, u)
+    full = octs is None
     octs = np.arange(mesh.n_oct) if octs is None else np.asarray(octs, dtype=np.int64)
     nf = u.shape[0]
-    src, kind = mesh.padding_sources(octs)
+    # the maps do not depend on u: memoise them for the whole mesh
+    if full and getattr(mesh, "_pad_cache", None) is not None:
+        src, kind = mesh._pad_cache
+    else:
+        src, kind = mesh.padding_sources(octs)
+        if full:
+            mesh._pad_cache = (src, kind)
     pijk = _patch_ijk()
     out = np.empty((nf, len(octs), P13 ** 3))
     for i0 in range(0, len(octs), chunk // 8 + 1):

@@ -1,0 +1,286 @@
+"""Python binding of libdgr (include/dgr.h): argument marshalling only.
+
+Every step of the hot path runs in libdgr's CUDA kernels; this module only
+converts torch tensors to pointers, picks torch's current CUDA stream, and
+raises DgrError on failure.  There is no CPU fallback: if libdgr.so is
+missing, importing the binding's device entry points raises.
+
+Names follow the C ABI: octree_build, Mesh (dgr_mesh_create ... destroy),
+Mesh.unzip, Mesh.rhs, Mesh.rhs_patches, Mesh.rk4_stage, Mesh.rk4_step,
+Mesh.constraints, Mesh.ghost_exchange.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+from dataclasses import dataclass
+
+import numpy as np
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "lib", "libdgr.so")
+
+NF = 24
+NPT = 343
+NPATCH = 2197
+
+MAP_OCTANTS, MAP_O2N, MAP_HANGING, MAP_PAD_SRC, MAP_PAD_KIND, MAP_ZIP = 0, 1, 2, 3, 4, 5
+MAP_DOF_GID, MAP_DOF_XYZ, MAP_SEND, MAP_SEND_COUNTS, MAP_RECV_COUNTS = 6, 7, 8, 9, 10
+
+
+class DgrError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"libdgr status {status}: {msg}")
+        self.status = status
+
+
+class _Octant(C.Structure):
+    _fields_ = [("x", C.c_uint32), ("y", C.c_uint32), ("z", C.c_uint32), ("level", C.c_uint32)]
+
+
+class _Puncture(C.Structure):
+    _fields_ = [("x", C.c_double), ("y", C.c_double), ("z", C.c_double), ("m", C.c_double),
+                ("level", C.c_int32), ("pad", C.c_int32)]
+
+
+class _RefineDesc(C.Structure):
+    _fields_ = [("xmin", C.c_double * 3), ("width", C.c_double), ("max_depth", C.c_int32),
+                ("periodic", C.c_int32), ("level_min", C.c_int32), ("n_punct", C.c_int32),
+                ("punct", C.POINTER(_Puncture)), ("rho", C.c_double)]
+
+
+class _MeshDesc(C.Structure):
+    _fields_ = [("xmin", C.c_double * 3), ("width", C.c_double), ("max_depth", C.c_int32),
+                ("periodic", C.c_int32), ("rank", C.c_int32), ("nranks", C.c_int32),
+                ("device", C.c_int32), ("pad", C.c_int32), ("nccl_id", C.c_void_p)]
+
+
+class _Params(C.Structure):
+    _fields_ = [("ko_sigma", C.c_double), ("eta", C.c_double), ("lambda_f0", C.c_double),
+                ("lambda_f1", C.c_double), ("chi_floor", C.c_double)]
+
+
+class _Info(C.Structure):
+    _fields_ = [("n_oct_global", C.c_int64), ("n_oct_local", C.c_int64),
+                ("n_oct_ghost", C.c_int64), ("oct_begin", C.c_int64),
+                ("n_dof_global", C.c_int64), ("n_dof_owned", C.c_int64),
+                ("n_dof_ghost", C.c_int64), ("dof_stride", C.c_int64),
+                ("patch_pitch", C.c_int64), ("n_hanging", C.c_int64), ("h_min", C.c_double),
+                ("level_min", C.c_int32), ("level_max", C.c_int32)]
+
+
+_lib = None
+EXPORTED = ["dgr_status_string", "dgr_last_error", "dgr_version", "dgr_octree_build",
+            "dgr_mesh_create", "dgr_mesh_info_get", "dgr_mesh_export_maps", "dgr_mesh_destroy",
+            "dgr_dof_coords", "dgr_unzip", "dgr_ghost_exchange", "dgr_rhs_patches", "dgr_rhs",
+            "dgr_rk4_stage", "dgr_rk4_step", "dgr_constraints", "dgr_last_launch_count"]
+
+
+def lib():
+    """Load libdgr.so (built by build.py / __graft_entry__.build()); raise if absent."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"libdgr.so not built ({LIB_PATH}); run "
+                              "python -m paper_conf_sc_fernandonhzsgb22_b200.build")
+        L = C.CDLL(LIB_PATH)
+        vp, i64, i32, dp = C.c_void_p, C.c_int64, C.c_int, C.c_double
+        L.dgr_status_string.restype = C.c_char_p
+        L.dgr_status_string.argtypes = [i32]
+        L.dgr_last_error.restype = C.c_char_p
+        L.dgr_version.restype = C.c_char_p
+        L.dgr_octree_build.argtypes = [C.POINTER(_RefineDesc), vp, C.POINTER(i64)]
+        L.dgr_mesh_create.argtypes = [C.POINTER(_MeshDesc), vp, i64, vp, C.POINTER(vp)]
+        L.dgr_mesh_info_get.argtypes = [vp, C.POINTER(_Info)]
+        L.dgr_mesh_export_maps.argtypes = [vp, i32, vp, C.POINTER(C.c_size_t)]
+        L.dgr_mesh_destroy.argtypes = [vp]
+        L.dgr_dof_coords.argtypes = [vp, vp, vp]
+        L.dgr_unzip.argtypes = [vp, vp, vp, i32, vp]
+        L.dgr_ghost_exchange.argtypes = [vp, vp, vp]
+        L.dgr_rhs_patches.argtypes = [vp, vp, vp, C.POINTER(_Params), vp]
+        L.dgr_rhs.argtypes = [vp, vp, vp, C.POINTER(_Params), vp]
+        L.dgr_rk4_stage.argtypes = [vp, i32, dp, vp, vp, vp, C.POINTER(_Params), vp]
+        L.dgr_rk4_step.argtypes = [vp, dp, vp, C.POINTER(_Params), vp]
+        L.dgr_constraints.argtypes = [vp, vp, vp, vp, C.POINTER(_Params), vp]
+        L.dgr_last_launch_count.restype = i64
+        L.dgr_last_launch_count.argtypes = [vp]
+        for f in ["dgr_octree_build", "dgr_mesh_create", "dgr_mesh_info_get",
+                  "dgr_mesh_export_maps", "dgr_mesh_destroy", "dgr_dof_coords", "dgr_unzip",
+                  "dgr_ghost_exchange", "dgr_rhs_patches", "dgr_rhs", "dgr_rk4_stage",
+                  "dgr_rk4_step", "dgr_constraints"]:
+            getattr(L, f).restype = i32
+        _lib = L
+    return _lib
+
+
+def _check(st):
+    if st != 0:
+        L = lib()
+        raise DgrError(st, L.dgr_last_error().decode())
+
+
+@dataclass
+class Params:
+    """RHS parameters (readings R6, R8, R13)."""
+    ko_sigma: float = 0.4
+    eta: float = 2.0
+    lambda_f0: float = 1.0
+    lambda_f1: float = 0.0
+    chi_floor: float = 1e-4
+
+    def _c(self):
+        return _Params(self.ko_sigma, self.eta, self.lambda_f0, self.lambda_f1, self.chi_floor)
+
+
+def octree_build(cfg) -> np.ndarray:
+    """dgr_octree_build for a synth.configs.MeshConfig -> uint32 [n, 4] (x, y, z, level)."""
+    L = lib()
+    P = (_Puncture * max(1, len(cfg.punctures)))()
+    for i, p in enumerate(cfg.punctures):
+        P[i] = _Puncture(p.x, p.y, p.z, p.m, p.level, 0)
+    d = _RefineDesc((C.c_double * 3)(*cfg.xmin), cfg.width, cfg.max_depth, int(cfg.periodic),
+                    cfg.level_min, len(cfg.punctures), P, cfg.rho)
+    n = C.c_int64(0)
+    _check(L.dgr_octree_build(C.byref(d), None, C.byref(n)))
+    out = np.zeros((n.value, 4), dtype=np.uint32)
+    _check(L.dgr_octree_build(C.byref(d), out.ctypes.data, C.byref(n)))
+    return out
+
+
+def _ptr(t):
+    return C.c_void_p(t.data_ptr())
+
+
+def _stream():
+    import torch
+    return C.c_void_p(torch.cuda.current_stream().cuda_stream)
+
+
+class Mesh:
+    """A dgr_mesh handle.  device=False builds host maps only (map export works
+    without a GPU); device=True uploads maps and allocates workspace."""
+
+    def __init__(self, cfg, octants=None, device=True, rank=0, nranks=1, nccl_id=None):
+        L = lib()
+        if octants is None:
+            octants = octree_build(cfg)
+        self.octants = np.ascontiguousarray(octants, dtype=np.uint32)
+        self.cfg = cfg
+        idbuf = None
+        if nccl_id is not None:
+            idbuf = C.create_string_buffer(bytes(nccl_id), 128)
+        d = _MeshDesc((C.c_double * 3)(*cfg.xmin), cfg.width, cfg.max_depth, int(cfg.periodic),
+                      rank, nranks, int(device), 0,
+                      C.cast(idbuf, C.c_void_p) if idbuf is not None else None)
+        h = C.c_void_p()
+        stream = _stream() if device else None
+        _check(L.dgr_mesh_create(C.byref(d), self.octants.ctypes.data, len(self.octants), stream,
+                                 C.byref(h)))
+        self._h = h
+        self.device = device
+        info = _Info()
+        _check(L.dgr_mesh_info_get(h, C.byref(info)))
+        self.info = {k: getattr(info, k) for k, _ in _Info._fields_}
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h is not None and h.value and _lib is not None:
+            _lib.dgr_mesh_destroy(h)
+            self._h = None
+
+    close = __del__
+
+    # ------------------------------------------------------------ host maps
+    def export(self, which, dtype):
+        L = lib()
+        n = C.c_size_t(0)
+        _check(L.dgr_mesh_export_maps(self._h, which, None, C.byref(n)))
+        out = np.empty(n.value // np.dtype(dtype).itemsize, dtype=dtype)
+        if n.value:
+            _check(L.dgr_mesh_export_maps(self._h, which, out.ctypes.data, C.byref(n)))
+        return out
+
+    def maps(self):
+        no = self.info["n_oct_local"]
+        return dict(
+            octants=self.export(MAP_OCTANTS, np.int32).reshape(-1, 4),
+            o2n=self.export(MAP_O2N, np.int32).reshape(no, NPT),
+            hanging=self.export(MAP_HANGING, np.int32).reshape(-1, 3),
+            pad_src=self.export(MAP_PAD_SRC, np.int32).reshape(no, NPATCH),
+            pad_kind=self.export(MAP_PAD_KIND, np.uint8).reshape(no, NPATCH),
+            zip=self.export(MAP_ZIP, np.int32).reshape(-1, 2),
+            dof_gid=self.export(MAP_DOF_GID, np.int64),
+        )
+
+    def dof_xyz_host(self):
+        return self.export(MAP_DOF_XYZ, np.float64).reshape(3, -1)
+
+    @property
+    def dof_stride(self):
+        return self.info["dof_stride"]
+
+    @property
+    def n_dof(self):
+        return self.info["n_dof_owned"] + self.info["n_dof_ghost"]
+
+    # -------------------------------------------------------- device calls
+    def new_state(self, dtype=None):
+        import torch
+        return torch.zeros((NF, self.dof_stride), dtype=torch.float64, device="cuda")
+
+    def dof_coords(self):
+        import torch
+        xyz = torch.empty((3, self.dof_stride), dtype=torch.float64, device="cuda")
+        _check(lib().dgr_dof_coords(self._h, _ptr(xyz), _stream()))
+        return xyz
+
+    def unzip(self, u, nfields=NF, patches=None):
+        import torch
+        if patches is None:
+            patches = torch.empty((nfields, self.info["n_oct_local"], self.info["patch_pitch"]),
+                                  dtype=torch.float64, device="cuda")
+        _check(lib().dgr_unzip(self._h, _ptr(u), _ptr(patches), nfields, _stream()))
+        return patches
+
+    def rhs_patches(self, patches, prm=None, out=None):
+        import torch
+        if out is None:
+            out = torch.empty((NF, self.info["n_oct_local"], NPT), dtype=torch.float64,
+                              device="cuda")
+        p = (prm or Params())._c()
+        _check(lib().dgr_rhs_patches(self._h, _ptr(patches), _ptr(out), C.byref(p), _stream()))
+        return out
+
+    def ghost_exchange(self, u):
+        _check(lib().dgr_ghost_exchange(self._h, _ptr(u), _stream()))
+
+    def rhs(self, u, prm=None, out=None):
+        import torch
+        if out is None:
+            out = torch.zeros_like(u)
+        p = (prm or Params())._c()
+        _check(lib().dgr_rhs(self._h, _ptr(u), _ptr(out), C.byref(p), _stream()))
+        return out
+
+    def rk4_stage(self, s, dt, u_n, u_s, acc, prm=None):
+        p = (prm or Params())._c()
+        _check(lib().dgr_rk4_stage(self._h, s, float(dt), _ptr(u_n), _ptr(u_s), _ptr(acc),
+                                   C.byref(p), _stream()))
+
+    def rk4_step(self, u, dt, prm=None):
+        p = (prm or Params())._c()
+        _check(lib().dgr_rk4_step(self._h, float(dt), _ptr(u), C.byref(p), _stream()))
+        return u
+
+    def constraints(self, u, prm=None, out=None):
+        import torch
+        if out is None:
+            out = torch.zeros((7, self.dof_stride), dtype=torch.float64, device="cuda")
+        norms = np.zeros(14)
+        p = (prm or Params())._c()
+        _check(lib().dgr_constraints(self._h, _ptr(u), _ptr(out), norms.ctypes.data, C.byref(p),
+                                     _stream()))
+        return out, norms.reshape(7, 2)
+
+    def last_launch_count(self):
+        return int(lib().dgr_last_launch_count(self._h))

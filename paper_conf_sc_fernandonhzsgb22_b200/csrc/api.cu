@@ -1,0 +1,642 @@
+// C ABI of libdgr (include/dgr.h): mesh lifetime, map export, and the
+// device entry points (unzip, rhs, rk4 stage/step, constraints).
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <array>
+#include <cmath>
+#include <cstring>
+#include <memory>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/dgr.h"
+#include "device.cuh"
+#include "host_mesh.hpp"
+
+namespace dgr {
+void upload_tables(const double* w13, const double* wext);
+}
+
+using namespace dgr;
+
+// --------------------------------------------------------------- errors
+static thread_local std::string g_err;
+
+static dgr_status fail(dgr_status s, const std::string& msg) {
+  g_err = msg;
+  return s;
+}
+
+#define CUDA_TRY(x)                                                                   \
+  do {                                                                                \
+    cudaError_t _e = (x);                                                             \
+    if (_e != cudaSuccess)                                                            \
+      return fail(DGR_ERR_CUDA, std::string(#x) + ": " + cudaGetErrorString(_e));   \
+  } while (0)
+
+// ---------------------------------------------------------------- NCCL (dlopen)
+namespace {
+typedef int ncclResult_t_;
+struct NcclApi {
+  void* h = nullptr;
+  ncclResult_t_ (*CommInitRank)(void**, int, const void* /*by value 128B*/, int) = nullptr;
+  ncclResult_t_ (*CommDestroy)(void*) = nullptr;
+  ncclResult_t_ (*Send)(const void*, size_t, int, int, void*, cudaStream_t) = nullptr;
+  ncclResult_t_ (*Recv)(void*, size_t, int, int, void*, cudaStream_t) = nullptr;
+  ncclResult_t_ (*GroupStart)() = nullptr;
+  ncclResult_t_ (*GroupEnd)() = nullptr;
+  ncclResult_t_ (*AllReduce)(const void*, void*, size_t, int, int, void*, cudaStream_t) = nullptr;
+};
+struct UniqueId {
+  char internal[128];
+};
+typedef int (*InitRankFn)(void**, int, UniqueId, int);
+InitRankFn g_init_rank = nullptr;
+NcclApi g_nccl;
+bool load_nccl() {
+  if (g_nccl.h) return true;
+  const char* names[] = {"libnccl.so.2", "libnccl.so"};
+  for (const char* n : names) {
+    g_nccl.h = dlopen(n, RTLD_NOW | RTLD_GLOBAL);
+    if (g_nccl.h) break;
+  }
+  if (!g_nccl.h) return false;
+  g_init_rank = (InitRankFn)dlsym(g_nccl.h, "ncclCommInitRank");
+  g_nccl.CommDestroy = (ncclResult_t_(*)(void*))dlsym(g_nccl.h, "ncclCommDestroy");
+  g_nccl.Send = (ncclResult_t_(*)(const void*, size_t, int, int, void*, cudaStream_t))dlsym(
+      g_nccl.h, "ncclSend");
+  g_nccl.Recv =
+      (ncclResult_t_(*)(void*, size_t, int, int, void*, cudaStream_t))dlsym(g_nccl.h, "ncclRecv");
+  g_nccl.GroupStart = (ncclResult_t_(*)())dlsym(g_nccl.h, "ncclGroupStart");
+  g_nccl.GroupEnd = (ncclResult_t_(*)())dlsym(g_nccl.h, "ncclGroupEnd");
+  g_nccl.AllReduce = (ncclResult_t_(*)(const void*, void*, size_t, int, int, void*,
+                                       cudaStream_t))dlsym(g_nccl.h, "ncclAllReduce");
+  return g_init_rank && g_nccl.Send && g_nccl.Recv && g_nccl.GroupStart && g_nccl.GroupEnd &&
+         g_nccl.AllReduce && g_nccl.CommDestroy;
+}
+constexpr int NCCL_FLOAT64 = 8, NCCL_SUM = 0, NCCL_MAX = 2;
+}  // namespace
+
+// ----------------------------------------------------------------- mesh
+struct dgr_mesh_s {
+  HostMesh host;
+  bool device = false;
+  int dev_id = -1;
+  DevMesh dm{};
+  double xmin[3];
+  // device allocations
+  std::vector<void*> allocs;
+  int4* d_oct = nullptr;
+  int32_t* d_o2n = nullptr;
+  uint8_t* d_pmap = nullptr;
+  NbrEntry* d_nbr = nullptr;
+  int32_t* d_zip = nullptr;
+  int4* d_hang = nullptr;
+  std::vector<int64_t> hang_level_off;  // row offsets per level group
+  int64_t* d_dof_node = nullptr;
+  double* d_E = nullptr;        // [24][n_local][343]
+  double* d_patch = nullptr;    // [24][n_owned][PATCH_PITCH]
+  double* d_rhs_oct = nullptr;  // [24][n_owned][343]
+  double* d_us = nullptr;       // RK4 stage state [24][dof_stride]
+  double* d_acc = nullptr;      // RK4 accumulator
+  double* d_cnorm = nullptr;    // constraint norm partials
+  // multi-rank
+  void* comm = nullptr;
+  int32_t* d_send = nullptr;
+  double* d_sendbuf = nullptr;
+  double* d_recvbuf = nullptr;
+  int64_t launches = 0;
+
+  template <class T>
+  cudaError_t alloc(T** p, size_t n) {
+    void* q = nullptr;
+    cudaError_t e = cudaMalloc(&q, std::max<size_t>(n, 1) * sizeof(T));
+    if (e == cudaSuccess) {
+      allocs.push_back(q);
+      *p = static_cast<T*>(q);
+    }
+    return e;
+  }
+  ~dgr_mesh_s() {
+    for (void* q : allocs) cudaFree(q);
+    if (comm && g_nccl.CommDestroy) g_nccl.CommDestroy(comm);
+  }
+};
+
+// Lagrange rows computed exactly: l_m(t2/2) = prod_{q!=m} (t2 - 2q) / (2 (m - q)).
+static void lagrange_tables(double* w13, double* wext) {
+  for (int t2 = 0; t2 < 13; ++t2)
+    for (int m = 0; m < 7; ++m) {
+      long long num = 1, den = 1;
+      for (int q = 0; q < 7; ++q)
+        if (q != m) {
+          num *= (t2 - 2 * q);
+          den *= 2 * (m - q);
+        }
+      w13[t2 * 7 + m] = double(num) / double(den);
+    }
+  for (int t = 0; t < 3; ++t) {
+    const int tt = -(t + 1);
+    for (int m = 0; m < 7; ++m) {
+      long long num = 1, den = 1;
+      for (int q = 0; q < 7; ++q)
+        if (q != m) {
+          num *= (tt - q);
+          den *= (m - q);
+        }
+      wext[t * 7 + m] = double(num) / double(den);
+    }
+  }
+}
+
+extern "C" {
+
+const char* dgr_status_string(dgr_status s) {
+  switch (s) {
+    case DGR_OK: return "ok";
+    case DGR_ERR_ARG: return "invalid argument";
+    case DGR_ERR_TREE: return "invalid octree";
+    case DGR_ERR_CUDA: return "CUDA error";
+    case DGR_ERR_NCCL: return "NCCL error";
+    case DGR_ERR_OOM: return "out of memory";
+    case DGR_ERR_STATE: return "invalid state";
+  }
+  return "unknown";
+}
+
+const char* dgr_last_error(void) { return g_err.c_str(); }
+const char* dgr_version(void) { return "dgr-b200 0.1 (sm_100a)"; }
+
+dgr_status dgr_octree_build(const dgr_refine_desc* desc, dgr_octant* out, int64_t* n_inout) {
+  if (!desc || !n_inout) return fail(DGR_ERR_ARG, "null argument");
+  if (desc->max_depth < 1 || desc->max_depth > 20 || desc->width <= 0 || desc->n_punct < 0 ||
+      (desc->n_punct > 0 && !desc->punct) || desc->level_min < 0 ||
+      desc->level_min > desc->max_depth)
+    return fail(DGR_ERR_ARG, "bad refine descriptor");
+  try {
+    std::vector<PunctureDesc> p;
+    for (int i = 0; i < desc->n_punct; ++i) {
+      const dgr_puncture& q = desc->punct[i];
+      if (q.level < 0 || q.level > desc->max_depth) return fail(DGR_ERR_ARG, "bad puncture level");
+      p.push_back({q.x, q.y, q.z, q.m, q.level});
+    }
+    std::vector<Oct> o = build_octree(desc->xmin, desc->width, desc->max_depth,
+                                      desc->periodic != 0, desc->level_min, p, desc->rho);
+    if (!out) {
+      *n_inout = int64_t(o.size());
+      return DGR_OK;
+    }
+    if (*n_inout < int64_t(o.size())) return fail(DGR_ERR_ARG, "output buffer too small");
+    for (size_t i = 0; i < o.size(); ++i)
+      out[i] = {uint32_t(o[i].a[0]), uint32_t(o[i].a[1]), uint32_t(o[i].a[2]), uint32_t(o[i].l)};
+    *n_inout = int64_t(o.size());
+    return DGR_OK;
+  } catch (const std::bad_alloc&) {
+    return fail(DGR_ERR_OOM, "host allocation failed");
+  }
+}
+
+static dgr_status upload(dgr_mesh m, cudaStream_t st) {
+  HostMesh& h = m->host;
+  const int64_t nl = int64_t(h.local_oct.size());
+  const int64_t no = h.n_owned_oct;
+  CUDA_TRY(cudaGetDevice(&m->dev_id));
+  // octant info
+  std::vector<int4> oi(nl);
+  for (int64_t l = 0; l < nl; ++l) {
+    const Oct& o = h.oct[h.local_oct[l]];
+    oi[l] = make_int4(int(o.a[0]), int(o.a[1]), int(o.a[2]), o.l);
+  }
+  CUDA_TRY(m->alloc(&m->d_oct, nl));
+  CUDA_TRY(cudaMemcpy(m->d_oct, oi.data(), nl * sizeof(int4), cudaMemcpyHostToDevice));
+  CUDA_TRY(m->alloc(&m->d_o2n, h.o2n_local.size()));
+  CUDA_TRY(cudaMemcpy(m->d_o2n, h.o2n_local.data(), h.o2n_local.size() * 4, cudaMemcpyHostToDevice));
+  CUDA_TRY(m->alloc(&m->d_pmap, h.pmap.size()));
+  CUDA_TRY(cudaMemcpy(m->d_pmap, h.pmap.data(), h.pmap.size(), cudaMemcpyHostToDevice));
+  CUDA_TRY(m->alloc(&m->d_nbr, h.nbr.size()));
+  CUDA_TRY(cudaMemcpy(m->d_nbr, h.nbr.data(), h.nbr.size() * sizeof(NbrEntry),
+                      cudaMemcpyHostToDevice));
+  CUDA_TRY(m->alloc(&m->d_zip, h.zip_local.size()));
+  CUDA_TRY(cudaMemcpy(m->d_zip, h.zip_local.data(), h.zip_local.size() * 4, cudaMemcpyHostToDevice));
+  // hanging rows grouped by level
+  std::vector<int4> hr(h.hang_rows.size());
+  m->hang_level_off.clear();
+  int prev = -1;
+  for (size_t i = 0; i < h.hang_rows.size(); ++i) {
+    const auto& r = h.hang_rows[i];
+    if (r.level != prev) {
+      m->hang_level_off.push_back(int64_t(i));
+      prev = r.level;
+    }
+    hr[i] = make_int4(r.e_local, r.node, r.src_local, r.t2[0] | (r.t2[1] << 8) | (r.t2[2] << 16));
+  }
+  m->hang_level_off.push_back(int64_t(hr.size()));
+  CUDA_TRY(m->alloc(&m->d_hang, hr.size()));
+  if (!hr.empty())
+    CUDA_TRY(cudaMemcpy(m->d_hang, hr.data(), hr.size() * sizeof(int4), cudaMemcpyHostToDevice));
+  // DOF lattice coordinates
+  const int64_t nd = h.n_owned_dof + h.n_ghost_dof;
+  const int64_t stride = ((nd + 31) / 32) * 32;
+  std::vector<int64_t> node(3 * stride, 0);
+  for (int64_t d = 0; d < nd; ++d) {
+    const int64_t g = h.dof_gid[d];
+    const int32_t e = h.zip_leaf[g], n = h.zip_node[g];
+    const Oct& o = h.oct[e];
+    const int64_t s = h.side(e);
+    node[3 * d + 0] = 6 * o.a[0] + (n % 7) * s;
+    node[3 * d + 1] = 6 * o.a[1] + ((n / 7) % 7) * s;
+    node[3 * d + 2] = 6 * o.a[2] + (n / 49) * s;
+  }
+  CUDA_TRY(m->alloc(&m->d_dof_node, node.size()));
+  CUDA_TRY(cudaMemcpy(m->d_dof_node, node.data(), node.size() * 8, cudaMemcpyHostToDevice));
+  // workspace
+  CUDA_TRY(m->alloc(&m->d_E, size_t(NF) * nl * NPT));
+  CUDA_TRY(m->alloc(&m->d_patch, size_t(NF) * no * PATCH_PITCH));
+  CUDA_TRY(m->alloc(&m->d_rhs_oct, size_t(NF) * no * NPT));
+  CUDA_TRY(m->alloc(&m->d_us, size_t(NF) * stride));
+  CUDA_TRY(m->alloc(&m->d_acc, size_t(NF) * stride));
+  CUDA_TRY(cudaMemset(m->d_patch, 0, size_t(NF) * no * PATCH_PITCH * 8));
+  CUDA_TRY(cudaMemset(m->d_us, 0, size_t(NF) * stride * 8));
+  CUDA_TRY(cudaMemset(m->d_acc, 0, size_t(NF) * stride * 8));
+  double w13[91], wext[21];
+  lagrange_tables(w13, wext);
+  upload_tables(w13, wext);
+  CUDA_TRY(cudaGetLastError());
+  DevMesh& dm = m->dm;
+  dm.n_owned = int32_t(no);
+  dm.n_local = int32_t(nl);
+  dm.dof_stride = stride;
+  dm.n_owned_dof = int32_t(h.n_owned_dof);
+  dm.D = h.D;
+  dm.periodic = h.periodic ? 1 : 0;
+  dm.width = h.width;
+  dm.oct = m->d_oct;
+  dm.o2n = m->d_o2n;
+  dm.pmap = m->d_pmap;
+  dm.nbr = m->d_nbr;
+  dm.zip = m->d_zip;
+  dm.hang = m->d_hang;
+  // multi-rank buffers
+  if (h.nranks > 1) {
+    CUDA_TRY(m->alloc(&m->d_send, h.send_list.size()));
+    if (!h.send_list.empty())
+      CUDA_TRY(cudaMemcpy(m->d_send, h.send_list.data(), h.send_list.size() * 4,
+                          cudaMemcpyHostToDevice));
+    CUDA_TRY(m->alloc(&m->d_sendbuf, size_t(NF) * h.send_list.size()));
+    CUDA_TRY(m->alloc(&m->d_recvbuf, size_t(NF) * h.n_ghost_dof));
+  }
+  CUDA_TRY(m->alloc(&m->d_cnorm, 64));
+  CUDA_TRY(cudaStreamSynchronize(st));
+  return DGR_OK;
+}
+
+dgr_status dgr_mesh_create(const dgr_mesh_desc* desc, const dgr_octant* octs, int64_t n,
+                           void* stream, dgr_mesh* out) {
+  if (!desc || !octs || !out || n <= 0) return fail(DGR_ERR_ARG, "null argument or n <= 0");
+  *out = nullptr;
+  std::unique_ptr<dgr_mesh_s> m;
+  try {
+    m.reset(new dgr_mesh_s());
+    std::vector<Oct> leaves(n);
+    for (int64_t i = 0; i < n; ++i)
+      leaves[i] = {{int64_t(octs[i].x), int64_t(octs[i].y), int64_t(octs[i].z)},
+                   int(octs[i].level)};
+    m->host.build(desc->xmin, desc->width, desc->max_depth, desc->periodic != 0, leaves,
+                  desc->rank, desc->nranks);
+  } catch (const BuildError& e) {
+    return fail(dgr_status(e.code), e.msg);
+  } catch (const std::bad_alloc&) {
+    return fail(DGR_ERR_OOM, "host allocation failed");
+  }
+  for (int k = 0; k < 3; ++k) m->xmin[k] = desc->xmin[k];
+  m->device = desc->device != 0;
+  if (m->device) {
+    dgr_status s = upload(m.get(), static_cast<cudaStream_t>(stream));
+    if (s != DGR_OK) return s;
+    if (desc->nranks > 1) {
+      if (!desc->nccl_id) return fail(DGR_ERR_ARG, "nccl_id required for nranks > 1");
+      if (!load_nccl()) return fail(DGR_ERR_NCCL, "libnccl.so.2 not loadable");
+      UniqueId uid;
+      std::memcpy(uid.internal, desc->nccl_id, 128);
+      if (g_init_rank(&m->comm, desc->nranks, uid, desc->rank) != 0)
+        return fail(DGR_ERR_NCCL, "ncclCommInitRank failed");
+    }
+  }
+  *out = m.release();
+  return DGR_OK;
+}
+
+dgr_status dgr_mesh_info_get(dgr_mesh m, dgr_mesh_info* info) {
+  if (!m || !info) return fail(DGR_ERR_ARG, "null argument");
+  const HostMesh& h = m->host;
+  info->n_oct_global = int64_t(h.oct.size());
+  info->n_oct_local = h.n_owned_oct;
+  info->n_oct_ghost = h.n_ghost_oct;
+  info->oct_begin = h.oct_begin;
+  info->n_dof_global = h.n_dof;
+  info->n_dof_owned = h.n_owned_dof;
+  info->n_dof_ghost = h.n_ghost_dof;
+  const int64_t nd = h.n_owned_dof + h.n_ghost_dof;
+  info->dof_stride = ((nd + 31) / 32) * 32;
+  info->patch_pitch = PATCH_PITCH;
+  info->n_hanging = int64_t(h.hang_rows.size());
+  info->level_min = h.level_min;
+  info->level_max = h.level_max;
+  info->h_min = h.width / (6.0 * std::ldexp(1.0, h.level_max));
+  return DGR_OK;
+}
+
+dgr_status dgr_mesh_export_maps(dgr_mesh m, int which, void* host_buf, size_t* nbytes) {
+  if (!m || !nbytes) return fail(DGR_ERR_ARG, "null argument");
+  const HostMesh& h = m->host;
+  const int64_t N = int64_t(h.oct.size()), no = h.n_owned_oct;
+  std::vector<char> tmp;
+  auto put = [&](const void* src, size_t n) -> dgr_status {
+    if (!host_buf) {
+      *nbytes = n;
+      return DGR_OK;
+    }
+    if (*nbytes < n) return fail(DGR_ERR_ARG, "buffer too small");
+    std::memcpy(host_buf, src, n);
+    *nbytes = n;
+    return DGR_OK;
+  };
+  switch (which) {
+    case DGR_MAP_OCTANTS: {
+      std::vector<int32_t> v(4 * N);
+      for (int64_t i = 0; i < N; ++i) {
+        v[4 * i] = int32_t(h.oct[i].a[0]);
+        v[4 * i + 1] = int32_t(h.oct[i].a[1]);
+        v[4 * i + 2] = int32_t(h.oct[i].a[2]);
+        v[4 * i + 3] = h.oct[i].l;
+      }
+      return put(v.data(), v.size() * 4);
+    }
+    case DGR_MAP_O2N:
+      return put(h.o2n.data() + size_t(h.oct_begin) * NPT, size_t(no) * NPT * 4);
+    case DGR_MAP_HANGING: {
+      std::vector<std::array<int32_t, 3>> rows;
+      for (const auto& r : h.hang_rows)
+        if (r.e_local < no) rows.push_back({r.e_global, r.node, r.src_global});
+      std::sort(rows.begin(), rows.end());
+      return put(rows.data(), rows.size() * 12);
+    }
+    case DGR_MAP_PAD_SRC:
+      return put(h.pad_src_global.data(), h.pad_src_global.size() * 4);
+    case DGR_MAP_PAD_KIND:
+      return put(h.pad_kind.data(), h.pad_kind.size());
+    case DGR_MAP_ZIP: {
+      std::vector<int32_t> v(2 * h.n_owned_dof);
+      for (int64_t l = 0; l < h.n_owned_dof; ++l) {
+        const int64_t g = h.dof_gid[l];
+        v[2 * l] = h.zip_leaf[g];
+        v[2 * l + 1] = h.zip_node[g];
+      }
+      return put(v.data(), v.size() * 4);
+    }
+    case DGR_MAP_DOF_GID:
+      return put(h.dof_gid.data(), h.dof_gid.size() * 8);
+    case DGR_MAP_DOF_XYZ: {
+      const int64_t nd = int64_t(h.dof_gid.size());
+      std::vector<double> v(3 * nd);
+      const double unit = h.width / double(h.L);
+      for (int64_t d = 0; d < nd; ++d) {
+        const int64_t g = h.dof_gid[d];
+        const int32_t e = h.zip_leaf[g], n = h.zip_node[g];
+        const Oct& o = h.oct[e];
+        const int64_t s = h.side(e);
+        const int64_t X[3] = {6 * o.a[0] + (n % 7) * s, 6 * o.a[1] + ((n / 7) % 7) * s,
+                              6 * o.a[2] + (n / 49) * s};
+        for (int k = 0; k < 3; ++k) v[k * nd + d] = h.xmin[k] + double(X[k]) * unit;
+      }
+      return put(v.data(), v.size() * 8);
+    }
+    case DGR_MAP_SEND:
+      return put(h.send_list.data(), h.send_list.size() * 4);
+    case DGR_MAP_SEND_COUNTS:
+      return put(h.send_counts.data(), h.send_counts.size() * 8);
+    case DGR_MAP_RECV_COUNTS:
+      return put(h.recv_counts.data(), h.recv_counts.size() * 8);
+  }
+  return fail(DGR_ERR_ARG, "unknown map id");
+}
+
+dgr_status dgr_mesh_destroy(dgr_mesh m) {
+  delete m;
+  return DGR_OK;
+}
+
+int64_t dgr_last_launch_count(dgr_mesh m) { return m ? m->launches : -1; }
+
+}  // extern "C"
+
+// ------------------------------------------------------------- device ops
+static dgr_status need_device(dgr_mesh m) {
+  if (!m) return fail(DGR_ERR_ARG, "null mesh");
+  if (!m->device) return fail(DGR_ERR_STATE, "host-only mesh (desc.device == 0)");
+  return DGR_OK;
+}
+
+static bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; }
+
+// ghost exchange: pack owned DOFs each peer needs, grouped send/recv, unpack
+static dgr_status exchange(dgr_mesh m, double* u, cudaStream_t st) {
+  const HostMesh& h = m->host;
+  if (h.nranks <= 1) return DGR_OK;
+  const int64_t stride = m->dm.dof_stride;
+  const int64_t nsend = int64_t(h.send_list.size());
+  launch_gather_pack(u, stride, m->d_send, nsend, m->d_sendbuf, st);
+  ++m->launches;
+  CUDA_TRY(cudaGetLastError());
+  // sendbuf is [f][nsend] with peers contiguous inside each field row; send
+  // one message per (peer, field) row segment inside a single group
+  if (g_nccl.GroupStart() != 0) return fail(DGR_ERR_NCCL, "ncclGroupStart");
+  int64_t soff = 0, roff = 0;
+  for (int peer = 0; peer < h.nranks; ++peer) {
+    const int64_t ns = h.send_counts[peer], nr = h.recv_counts[peer];
+    for (int f = 0; f < NF; ++f) {
+      if (ns) g_nccl.Send(m->d_sendbuf + f * nsend + soff, size_t(ns), NCCL_FLOAT64, peer, m->comm, st);
+      if (nr) g_nccl.Recv(u + f * stride + h.n_owned_dof + roff, size_t(nr), NCCL_FLOAT64, peer, m->comm, st);
+    }
+    soff += ns;
+    roff += nr;
+  }
+  if (g_nccl.GroupEnd() != 0) return fail(DGR_ERR_NCCL, "ncclGroupEnd");
+  return DGR_OK;
+}
+
+static dgr_status do_unzip(dgr_mesh m, const double* u, int nf, cudaStream_t st) {
+  launch_elements(m->dm, u, m->d_E, nf, st);
+  ++m->launches;
+  for (size_t g = 0; g + 1 < m->hang_level_off.size(); ++g) {
+    const int64_t a = m->hang_level_off[g], b = m->hang_level_off[g + 1];
+    launch_hanging(m->dm, m->d_hang + a, b - a, m->d_E, nf, st);
+    ++m->launches;
+  }
+  launch_unzip(m->dm, m->d_E, m->d_patch, nf, st);
+  ++m->launches;
+  CUDA_TRY(cudaGetLastError());
+  return DGR_OK;
+}
+
+static RhsParams to_rp(const dgr_params* p) {
+  RhsParams r{0.4, 2.0, 1.0, 0.0, 1e-4};
+  if (p) r = {p->ko_sigma, p->eta, p->lambda_f0, p->lambda_f1, p->chi_floor};
+  return r;
+}
+
+extern "C" {
+
+dgr_status dgr_dof_coords(dgr_mesh m, double* xyz, void* stream) {
+  dgr_status s = need_device(m);
+  if (s) return s;
+  if (!xyz) return fail(DGR_ERR_ARG, "null xyz");
+  launch_dof_coords(m->dm, m->d_dof_node, xyz, m->xmin, static_cast<cudaStream_t>(stream));
+  CUDA_TRY(cudaGetLastError());
+  return DGR_OK;
+}
+
+dgr_status dgr_ghost_exchange(dgr_mesh m, double* u, void* stream) {
+  dgr_status s = need_device(m);
+  if (s) return s;
+  return exchange(m, u, static_cast<cudaStream_t>(stream));
+}
+
+dgr_status dgr_unzip(dgr_mesh m, const double* u, double* patches, int nfields, void* stream) {
+  dgr_status s = need_device(m);
+  if (s) return s;
+  if (!u || !patches || nfields < 1 || nfields > NF) return fail(DGR_ERR_ARG, "bad unzip args");
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  m->launches = 0;
+  s = do_unzip(m, u, nfields, st);
+  if (s) return s;
+  const size_t bytes = size_t(nfields) * m->dm.n_owned * PATCH_PITCH * 8;
+  if (patches != m->d_patch)
+    CUDA_TRY(cudaMemcpyAsync(patches, m->d_patch, bytes, cudaMemcpyDeviceToDevice, st));
+  return DGR_OK;
+}
+
+dgr_status dgr_rhs_patches(dgr_mesh m, const double* patches, double* rhs_oct,
+                           const dgr_params* prm, void* stream) {
+  dgr_status s = need_device(m);
+  if (s) return s;
+  if (!patches || !rhs_oct || !aligned16(patches)) return fail(DGR_ERR_ARG, "bad rhs args");
+  launch_rhs(m->dm, patches, rhs_oct, to_rp(prm), static_cast<cudaStream_t>(stream));
+  CUDA_TRY(cudaGetLastError());
+  return DGR_OK;
+}
+
+dgr_status dgr_rhs(dgr_mesh m, double* u, double* rhs, const dgr_params* prm, void* stream) {
+  dgr_status s = need_device(m);
+  if (s) return s;
+  if (!u || !rhs) return fail(DGR_ERR_ARG, "null state");
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  m->launches = 0;
+  if ((s = exchange(m, u, st))) return s;
+  if ((s = do_unzip(m, u, NF, st))) return s;
+  launch_rhs(m->dm, m->d_patch, m->d_rhs_oct, to_rp(prm), st);
+  launch_zip(m->dm, m->d_rhs_oct, rhs, NF, st);
+  m->launches += 2;
+  CUDA_TRY(cudaGetLastError());
+  return DGR_OK;
+}
+
+static dgr_status stage(dgr_mesh m, int s_, double dt, double* u_n, double* u_s, double* acc,
+                        double* u_out, const dgr_params* prm, cudaStream_t st) {
+  dgr_status s;
+  double* cur = s_ == 0 ? u_n : u_s;
+  if ((s = exchange(m, cur, st))) return s;
+  if ((s = do_unzip(m, cur, NF, st))) return s;
+  launch_rhs(m->dm, m->d_patch, m->d_rhs_oct, to_rp(prm), st);
+  launch_zip_rk4(m->dm, m->d_rhs_oct, s_, dt, u_n, u_s, acc, u_out, st);
+  m->launches += 2;
+  CUDA_TRY(cudaGetLastError());
+  return DGR_OK;
+}
+
+dgr_status dgr_rk4_stage(dgr_mesh m, int s_, double dt, double* u_n, double* u_s, double* acc,
+                         const dgr_params* prm, void* stream) {
+  dgr_status s = need_device(m);
+  if (s) return s;
+  if (s_ < 0 || s_ > 3 || !u_n || !u_s || !acc) return fail(DGR_ERR_ARG, "bad stage args");
+  m->launches = 0;
+  return stage(m, s_, dt, u_n, u_s, acc, acc, prm, static_cast<cudaStream_t>(stream));
+}
+
+dgr_status dgr_rk4_step(dgr_mesh m, double dt, double* u, const dgr_params* prm, void* stream) {
+  dgr_status s = need_device(m);
+  if (s) return s;
+  if (!u) return fail(DGR_ERR_ARG, "null state");
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  m->launches = 0;
+  for (int k = 0; k < 4; ++k)
+    if ((s = stage(m, k, dt, u, m->d_us, m->d_acc, u, prm, st))) return s;
+  return DGR_OK;
+}
+
+dgr_status dgr_constraints(dgr_mesh m, double* u, double* c, double* norms_host,
+                           const dgr_params* prm, void* stream) {
+  dgr_status s = need_device(m);
+  if (s) return s;
+  if (!u || !c) return fail(DGR_ERR_ARG, "null argument");
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  m->launches = 0;
+  if ((s = exchange(m, u, st))) return s;
+  if ((s = do_unzip(m, u, NF, st))) return s;
+  launch_constraints(m->dm, m->d_patch, m->d_rhs_oct, to_rp(prm), st);
+  CUDA_TRY(cudaGetLastError());
+  // zip the 7 constraint fields
+  const int64_t stride = m->dm.dof_stride;
+  DevMesh dm = m->dm;
+  launch_zip(dm, m->d_rhs_oct, c, 7, st);
+  CUDA_TRY(cudaGetLastError());
+  if (norms_host) {
+    const int64_t n = m->host.n_owned_dof;
+    std::vector<double> hc(size_t(7) * stride);
+    CUDA_TRY(cudaMemcpyAsync(hc.data(), c, hc.size() * 8, cudaMemcpyDeviceToHost, st));
+    CUDA_TRY(cudaStreamSynchronize(st));
+    double part[14];
+    for (int q = 0; q < 7; ++q) {
+      double ss = 0, mx = 0;
+      for (int64_t d = 0; d < n; ++d) {
+        const double v = hc[q * stride + d];
+        ss += v * v;
+        mx = std::max(mx, std::fabs(v));
+      }
+      part[2 * q] = ss;
+      part[2 * q + 1] = mx;
+    }
+    double ntot = double(n);
+    if (m->host.nranks > 1) {
+      double* d = m->d_cnorm;
+      double sums[8], maxs[7];
+      for (int q = 0; q < 7; ++q) {
+        sums[q] = part[2 * q];
+        maxs[q] = part[2 * q + 1];
+      }
+      sums[7] = ntot;
+      CUDA_TRY(cudaMemcpyAsync(d, sums, 64, cudaMemcpyHostToDevice, st));
+      CUDA_TRY(cudaMemcpyAsync(d + 8, maxs, 56, cudaMemcpyHostToDevice, st));
+      g_nccl.AllReduce(d, d, 8, NCCL_FLOAT64, NCCL_SUM, m->comm, st);
+      g_nccl.AllReduce(d + 8, d + 8, 7, NCCL_FLOAT64, NCCL_MAX, m->comm, st);
+      CUDA_TRY(cudaMemcpyAsync(sums, d, 64, cudaMemcpyDeviceToHost, st));
+      CUDA_TRY(cudaMemcpyAsync(maxs, d + 8, 56, cudaMemcpyDeviceToHost, st));
+      CUDA_TRY(cudaStreamSynchronize(st));
+      for (int q = 0; q < 7; ++q) {
+        part[2 * q] = sums[q];
+        part[2 * q + 1] = maxs[q];
+      }
+      ntot = sums[7];
+    }
+    for (int q = 0; q < 7; ++q) {
+      norms_host[2 * q] = std::sqrt(part[2 * q] / std::max(ntot, 1.0));
+      norms_host[2 * q + 1] = part[2 * q + 1];
+    }
+  }
+  return DGR_OK;
+}
+
+}  // extern "C"

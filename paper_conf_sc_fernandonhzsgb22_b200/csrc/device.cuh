@@ -1,0 +1,58 @@
+// Device-side data structures and kernel entry points of libdgr (sm_100a).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "host_mesh.hpp"
+
+namespace dgr {
+
+constexpr int NF = 24;            // BSSN fields
+constexpr int PATCH_PITCH = 2208; // doubles per patch: 13^3 = 2197 padded to 128 B
+constexpr int STAGE_DBL = 2200;   // smem stage buffer (bulk copy of 2200 doubles)
+
+// Device view of a mesh (plain pointers; passed by value to kernels).
+struct DevMesh {
+  int32_t n_owned;      // owned octants
+  int32_t n_local;      // owned + ghost octants
+  int64_t dof_stride;
+  int32_t n_owned_dof;
+  int32_t D;
+  int32_t periodic;
+  double width;
+  const int4* oct;          // [n_local] anchor x,y,z, level
+  const int32_t* o2n;       // [n_local * 343] local DOF id or -1
+  const uint8_t* pmap;      // [n_owned * 2197]
+  const NbrEntry* nbr;      // [n_owned * NBR_MAX]
+  const int32_t* zip;       // [n_owned_dof] local octant * 343 + node
+  const int4* hang;         // rows: e_local, node, src_local, t2 packed (x | y<<8 | z<<16)
+};
+
+// kernels.cu
+void launch_elements(const DevMesh& m, const double* u, double* E, int nf, cudaStream_t s);
+void launch_hanging(const DevMesh& m, const int4* rows, int64_t count, double* E, int nf,
+                    cudaStream_t s);
+void launch_unzip(const DevMesh& m, const double* E, double* patches, int nf, cudaStream_t s);
+void launch_zip(const DevMesh& m, const double* rhs_oct, double* rhs, int nf, cudaStream_t s);
+void launch_zip_rk4(const DevMesh& m, const double* rhs_oct, int stage, double dt,
+                    const double* u_n, double* u_s, double* acc, double* u_out, cudaStream_t s);
+void launch_dof_coords(const DevMesh& m, const int64_t* dof_node, double* xyz,
+                       const double xmin[3], cudaStream_t s);
+void launch_gather_pack(const double* u, int64_t stride, const int32_t* list, int64_t n,
+                        double* buf, cudaStream_t s);
+void launch_scatter_unpack(double* u, int64_t stride, int64_t offset, const double* buf,
+                           int64_t n_total, cudaStream_t s);
+
+// rhs_kernel.cu
+struct RhsParams {
+  double ko_sigma, eta, lambda_f0, lambda_f1, chi_floor;
+};
+void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const RhsParams& p,
+                cudaStream_t s);
+size_t rhs_smem_bytes();
+
+// constraints_kernel.cu
+void launch_constraints(const DevMesh& m, const double* patches, double* c_oct,
+                        const RhsParams& p, cudaStream_t s);
+
+}  // namespace dgr

@@ -1,0 +1,559 @@
+// Fused BSSN RHS kernel: 6th-order derivatives + KO + the 24-field algebra
+// (§III-A eqs 1-19, §IV-B), fp64, sm_100a.
+//
+// Design: one CTA per octant patch, one thread per interior
+// point (343 of 352 threads).  The 24 field patches are streamed through
+// shared memory one field at a time by TMA bulk copies (cp.async.bulk,
+// double buffered, mbarrier completion).  While a field is resident every
+// thread evaluates that field's derivatives at its point straight from shared
+// memory and immediately consumes them in the part of the algebra that only
+// needs them ("staged" evaluation, cf. the paper's staged+CSE), so the
+// 210 derivatives of P:L310 are never stored: the per-point state that
+// survives between fields lives in shared-memory slots [slot][point]
+// (accumulators of the 21 vector/tensor outputs, values, inverse metric,
+// Christoffel symbols) and a few registers.  Field order:
+//   gt_ij (6) -> [Christoffel block] -> chi -> alpha -> Gt^i (3) -> beta^i (3)
+//   -> K -> At_ij (6) -> B^i (3)
+// Readings: R1-R8, R13; chi in divisions is max(chi, chi_floor).
+// Two algebraically exact simplifications versus the oracle's literal form:
+// the gt_ij-proportional part of R^chi_ij (eq 19) is dropped because the
+// trace-free projection in eq (6) annihilates it, and Gt_ijk (lowered) is the
+// first-kind symbol C_ijk itself (gt_il gt^lm C_mjk = C_ijk).
+#include <cuda_runtime.h>
+
+#include "device.cuh"
+
+namespace dgr {
+
+namespace {
+
+constexpr int RT = 352;   // threads (11 warps); 343 interior points
+constexpr int NPP = 344;  // slot stride in doubles
+
+// shared-memory slot map ([slot][NPP] doubles)
+constexpr int V_GT = 0, V_B = 3, V_GAM = 6, V_AT = 12;                         // values (18)
+constexpr int A_GT = 18, A_BETA = 21, A_B = 24, A_GAM = 27, A_AT = 33;         // accumulators (21)
+constexpr int G_INV = 39;                                                      // gt^ij (6)
+constexpr int S0 = 45;                                                         // scratch (24)
+constexpr int NSLOT = 69;
+constexpr size_t SMEM_BYTES = size_t(NSLOT) * NPP * 8 + size_t(2) * STAGE_DBL * 8 + 16;
+
+// field processing order
+__constant__ int c_order[NF] = {12, 13, 14, 15, 16, 17, 1, 0, 3, 4, 5, 6,
+                                7,  8,  2,  18, 19, 20, 21, 22, 23, 9, 10, 11};
+
+__device__ __forceinline__ int sidx(int i, int j) {
+  // (0,0)0 (0,1)1 (0,2)2 (1,1)3 (1,2)4 (2,2)5
+  return i <= j ? (i == 0 ? j : (i == 1 ? 2 + j : 5)) : (j == 0 ? i : (j == 1 ? 2 + i : 5));
+}
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, int count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+
+__device__ __forceinline__ void bulk_load(double* dst, const double* src, uint32_t bytes,
+                                          uint64_t* bar) {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+               "r"(bytes)
+               : "memory");
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::
+          "r"(smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t ok = 0;
+  while (!ok) {
+    asm volatile(
+        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+        " selp.u32 %0, 1, 0, p;\n}\n"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+  }
+}
+
+// centred 7-point stencils along one axis (stride st) at patch index c
+struct Line {
+  double d1, d2, ko;
+};
+__device__ __forceinline__ Line line_ops(const double* __restrict__ s, int c, int st) {
+  const double u0 = s[c];
+  const double a1 = s[c + st], b1 = s[c - st];
+  const double a2 = s[c + 2 * st], b2 = s[c - 2 * st];
+  const double a3 = s[c + 3 * st], b3 = s[c - 3 * st];
+  Line l;
+  l.d1 = (a1 - b1) * 45.0 - (a2 - b2) * 9.0 + (a3 - b3);                        // x 1/(60h)
+  const double s1 = a1 + b1, s2 = a2 + b2, s3 = a3 + b3;
+  l.d2 = 2.0 * s3 - 27.0 * s2 + 270.0 * s1 - 490.0 * u0;                         // x 1/(180h^2)
+  l.ko = s3 - 6.0 * s2 + 15.0 * s1 - 20.0 * u0;                                  // x sigma/(64h)
+  return l;
+}
+
+// D1_b(D1_a u) * (60h)^2
+__device__ __forceinline__ double mixed(const double* __restrict__ s, int c, int sa, int sb) {
+  double r[7];
+#pragma unroll
+  for (int b = -3; b <= 3; ++b) {
+    if (b == 0) continue;
+    const int cb = c + b * sb;
+    r[b + 3] = (s[cb + sa] - s[cb - sa]) * 45.0 - (s[cb + 2 * sa] - s[cb - 2 * sa]) * 9.0 +
+               (s[cb + 3 * sa] - s[cb - 3 * sa]);
+  }
+  return (r[4] - r[2]) * 45.0 - (r[5] - r[1]) * 9.0 + (r[6] - r[0]);
+}
+
+struct Derivs {
+  double d1[3];
+  double dd[6];  // symmetric second derivatives (only if second)
+  double ko;     // sum of the 3 KO terms, already scaled
+};
+
+template <bool SECOND>
+__device__ __forceinline__ Derivs derivs(const double* __restrict__ s, int c, double ih,
+                                         double ko_scale) {
+  Derivs d;
+  const Line lx = line_ops(s, c, 1), ly = line_ops(s, c, 13), lz = line_ops(s, c, 169);
+  const double f1 = ih * (1.0 / 60.0);
+  d.d1[0] = lx.d1 * f1;
+  d.d1[1] = ly.d1 * f1;
+  d.d1[2] = lz.d1 * f1;
+  d.ko = (lx.ko + ly.ko + lz.ko) * ko_scale;
+  if (SECOND) {
+    const double f2 = ih * ih * (1.0 / 180.0);
+    const double fm = ih * ih * (1.0 / 3600.0);
+    d.dd[0] = lx.d2 * f2;
+    d.dd[3] = ly.d2 * f2;
+    d.dd[5] = lz.d2 * f2;
+    d.dd[1] = mixed(s, c, 1, 13) * fm;
+    d.dd[2] = mixed(s, c, 1, 169) * fm;
+    d.dd[4] = mixed(s, c, 13, 169) * fm;
+  }
+  return d;
+}
+
+// trace with the inverse metric: gt^ij X_ij (symmetric storage)
+__device__ __forceinline__ double trace6(const double* gi, const double* X) {
+  return gi[0] * X[0] + gi[3] * X[3] + gi[5] * X[5] +
+         2.0 * (gi[1] * X[1] + gi[2] * X[2] + gi[4] * X[4]);
+}
+
+}  // namespace
+
+__global__ void __launch_bounds__(RT, 1)
+    k_rhs(DevMesh m, const double* __restrict__ patches, double* __restrict__ rhs_oct,
+          RhsParams prm) {
+  extern __shared__ __align__(128) double smem[];
+  double* slots = smem;                           // [NSLOT][NPP]
+  double* stage = smem + NSLOT * NPP;             // [2][STAGE_DBL]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(stage + 2 * STAGE_DBL);
+
+  const int e = blockIdx.x;
+  const int tid = threadIdx.x;
+  const bool active = tid < NPT;
+  const int p = active ? tid : 0;
+  const int pi = p % 7, pj = (p / 7) % 7, pk = p / 49;
+  const int c0 = (pi + 3) + 13 * (pj + 3) + 169 * (pk + 3);
+  const int64_t no = m.n_owned;
+  const double* pbase = patches + int64_t(e) * PATCH_PITCH;
+  const int64_t fstride = no * PATCH_PITCH;
+#define SL(slot) slots[(slot) * NPP + p]
+
+  if (tid == 0) {
+    mbar_init(&bars[0], 1);
+    mbar_init(&bars[1], 1);
+  }
+  __syncthreads();
+  if (tid == 0) {
+    bulk_load(stage, pbase + c_order[0] * fstride, STAGE_DBL * 8, &bars[0]);
+    bulk_load(stage + STAGE_DBL, pbase + c_order[1] * fstride, STAGE_DBL * 8, &bars[1]);
+  }
+
+  const int4 oi = m.oct[e];
+  const double ih = (6.0 * double(int64_t(1) << oi.w)) / m.width;   // 1/h
+  const double ko_scale = prm.ko_sigma * ih * (1.0 / 64.0);
+
+  // ---- values at the point (patch interior) -------------------------------
+  double alpha = 0, chi = 0, Kv = 0, beta[3] = {0, 0, 0};
+  if (active) {
+    alpha = __ldg(pbase + 0 * fstride + c0);
+    chi = __ldg(pbase + 1 * fstride + c0);
+    Kv = __ldg(pbase + 2 * fstride + c0);
+#pragma unroll
+    for (int i = 0; i < 3; ++i) {
+      SL(V_GT + i) = __ldg(pbase + (3 + i) * fstride + c0);
+      beta[i] = __ldg(pbase + (6 + i) * fstride + c0);
+      SL(V_B + i) = __ldg(pbase + (9 + i) * fstride + c0);
+    }
+    double g[6];
+#pragma unroll
+    for (int q = 0; q < 6; ++q) {
+      g[q] = __ldg(pbase + (12 + q) * fstride + c0);
+      SL(V_GAM + q) = g[q];
+      SL(V_AT + q) = __ldg(pbase + (18 + q) * fstride + c0);
+    }
+    // inverse metric by adjugate / determinant
+    const double a00 = g[3] * g[5] - g[4] * g[4];
+    const double a01 = g[2] * g[4] - g[1] * g[5];
+    const double a02 = g[1] * g[4] - g[2] * g[3];
+    const double det = g[0] * a00 + g[1] * a01 + g[2] * a02;
+    const double idet = 1.0 / det;
+    SL(G_INV + 0) = a00 * idet;
+    SL(G_INV + 1) = a01 * idet;
+    SL(G_INV + 2) = a02 * idet;
+    SL(G_INV + 3) = (g[0] * g[5] - g[2] * g[2]) * idet;
+    SL(G_INV + 4) = (g[1] * g[2] - g[0] * g[4]) * idet;
+    SL(G_INV + 5) = (g[0] * g[3] - g[1] * g[1]) * idet;
+#pragma unroll
+    for (int q = 0; q < 21; ++q) SL(A_GT + q) = 0.0;
+  }
+  const double chi_e = fmax(chi, prm.chi_floor);
+  const double ichi = 1.0 / chi_e;
+  double rA = 0.0, rC = 0.0, rK = 0.0;   // accumulators of alpha, chi, K
+  double dchi[3] = {0, 0, 0};
+
+  for (int st = 0; st < NF; ++st) {
+    const int buf = st & 1;
+    mbar_wait(&bars[buf], (st >> 1) & 1);
+    const double* s = stage + buf * STAGE_DBL;
+    const int f = c_order[st];
+    if (active) {
+      if (f >= 12 && f <= 17) {
+        // ---------------- conformal metric gt_q: d gt, gt^lm d_lm gt, adv, KO
+        const int q = f - 12;
+        const Derivs d = derivs<true>(s, c0, ih, ko_scale);
+        double gi[6];
+#pragma unroll
+        for (int r = 0; r < 6; ++r) gi[r] = SL(G_INV + r);
+#pragma unroll
+        for (int k = 0; k < 3; ++k) SL(S0 + k * 6 + q) = d.d1[k];
+        SL(S0 + 18 + q) = trace6(gi, d.dd);
+        SL(A_GAM + q) += beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
+        if (q == 5) {
+          // ---------------- Christoffel block (eqs 12, 17; readings R1, R7)
+          double gt[6], At[6];
+#pragma unroll
+          for (int r = 0; r < 6; ++r) {
+            gt[r] = SL(V_GAM + r);
+            At[r] = SL(V_AT + r);
+          }
+          double C[3][6];  // first kind C_k,ij = 1/2 (d_i g_kj + d_j g_ki - d_k g_ij)
+#pragma unroll
+          for (int k = 0; k < 3; ++k)
+#pragma unroll
+            for (int i = 0; i < 3; ++i)
+#pragma unroll
+              for (int j = i; j < 3; ++j)
+                C[k][sidx(i, j)] = 0.5 * (SL(S0 + i * 6 + sidx(k, j)) + SL(S0 + j * 6 + sidx(k, i)) -
+                                          SL(S0 + k * 6 + sidx(i, j)));
+          double Gam[3][6];  // second kind Gt^k_ij = gt^kl C_l,ij
+#pragma unroll
+          for (int k = 0; k < 3; ++k)
+#pragma unroll
+            for (int q2 = 0; q2 < 6; ++q2)
+              Gam[k][q2] = gi[sidx(k, 0)] * C[0][q2] + gi[sidx(k, 1)] * C[1][q2] +
+                           gi[sidx(k, 2)] * C[2][q2];
+          double cal[3];
+#pragma unroll
+          for (int k = 0; k < 3; ++k) cal[k] = trace6(gi, Gam[k]);
+          // Rt_ij without the d Gt terms
+          double Rt[6];
+#pragma unroll
+          for (int i = 0; i < 3; ++i)
+#pragma unroll
+            for (int j = i; j < 3; ++j) {
+              double r = -0.5 * SL(S0 + 18 + sidx(i, j));
+              double c2 = 0.0;
+#pragma unroll
+              for (int k = 0; k < 3; ++k) c2 += cal[k] * (C[i][sidx(j, k)] + C[j][sidx(i, k)]);
+              r += 0.5 * c2;
+              double qsum = 0.0;
+#pragma unroll
+              for (int l = 0; l < 3; ++l)
+#pragma unroll
+                for (int mm = 0; mm < 3; ++mm) {
+                  const double glm = gi[sidx(l, mm)];
+                  double t = 0.0;
+#pragma unroll
+                  for (int k = 0; k < 3; ++k)
+                    t += Gam[k][sidx(l, i)] * C[j][sidx(k, mm)] +
+                         Gam[k][sidx(l, j)] * C[i][sidx(k, mm)] +
+                         Gam[k][sidx(i, mm)] * C[k][sidx(l, j)];
+                  qsum += glm * t;
+                }
+              Rt[sidx(i, j)] = r + qsum;
+            }
+          // At_ij += chi alpha TF(Rt)
+          const double trR = trace6(gi, Rt);
+          const double ca = chi * alpha;
+#pragma unroll
+          for (int r = 0; r < 6; ++r) SL(A_AT + r) += ca * (Rt[r] - gt[r] * trR * (1.0 / 3.0));
+          // At^ij = gt^ik gt^jl At_kl ; Gt^i += 2 alpha Gt^i_jk At^jk
+          double Au[6];
+#pragma unroll
+          for (int i = 0; i < 3; ++i)
+#pragma unroll
+            for (int j = i; j < 3; ++j) {
+              double a = 0.0;
+#pragma unroll
+              for (int k = 0; k < 3; ++k)
+#pragma unroll
+                for (int l = 0; l < 3; ++l) a += gi[sidx(i, k)] * gi[sidx(j, l)] * At[sidx(k, l)];
+              Au[sidx(i, j)] = a;
+            }
+#pragma unroll
+          for (int i = 0; i < 3; ++i) SL(A_GT + i) += 2.0 * alpha * trace6(Au, Gam[i]);
+          // keep Gt^k_ij and CalGt^k for the chi, alpha and beta stages
+#pragma unroll
+          for (int k = 0; k < 3; ++k)
+#pragma unroll
+            for (int q2 = 0; q2 < 6; ++q2) SL(S0 + k * 6 + q2) = Gam[k][q2];
+#pragma unroll
+          for (int k = 0; k < 3; ++k) SL(S0 + 18 + k) = cal[k];
+        }
+      } else if (f == 1) {
+        // ---------------- chi: advection, KO, R^chi (eq 18-19), eq (8) chi term
+        const Derivs d = derivs<true>(s, c0, ih, ko_scale);
+        double gi[6], At[6], gt[6];
+#pragma unroll
+        for (int r = 0; r < 6; ++r) {
+          gi[r] = SL(G_INV + r);
+          At[r] = SL(V_AT + r);
+          gt[r] = SL(V_GAM + r);
+        }
+#pragma unroll
+        for (int k = 0; k < 3; ++k) dchi[k] = d.d1[k];
+        rC += beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
+        double Rc[6];
+#pragma unroll
+        for (int i = 0; i < 3; ++i)
+#pragma unroll
+          for (int j = i; j < 3; ++j) {
+            const int q = sidx(i, j);
+            const double gd = SL(S0 + 0 * 6 + q) * dchi[0] + SL(S0 + 1 * 6 + q) * dchi[1] +
+                              SL(S0 + 2 * 6 + q) * dchi[2];
+            Rc[q] = (d.dd[q] - gd) * (0.5 * ichi) - dchi[i] * dchi[j] * (0.25 * ichi * ichi);
+          }
+        const double trR = trace6(gi, Rc);
+        const double ca = chi * alpha;
+#pragma unroll
+        for (int r = 0; r < 6; ++r) SL(A_AT + r) += ca * (Rc[r] - gt[r] * trR * (1.0 / 3.0));
+        // Gt^i += -3 alpha / chi At^ij d_j chi
+#pragma unroll
+        for (int i = 0; i < 3; ++i) {
+          double v = 0.0;
+#pragma unroll
+          for (int j = 0; j < 3; ++j) {
+            double a = 0.0;
+#pragma unroll
+            for (int k = 0; k < 3; ++k)
+#pragma unroll
+              for (int l = 0; l < 3; ++l) a += gi[sidx(i, k)] * gi[sidx(j, l)] * At[sidx(k, l)];
+            v += a * dchi[j];
+          }
+          SL(A_GT + i) += -3.0 * alpha * ichi * v;
+        }
+      } else if (f == 0) {
+        // ---------------- alpha: advection, KO, D_i D_j alpha (eqs 13-15)
+        const Derivs d = derivs<true>(s, c0, ih, ko_scale);
+        double gi[6], At[6], gt[6];
+#pragma unroll
+        for (int r = 0; r < 6; ++r) {
+          gi[r] = SL(G_INV + r);
+          At[r] = SL(V_AT + r);
+          gt[r] = SL(V_GAM + r);
+        }
+        const double* da = d.d1;
+        rA += beta[0] * da[0] + beta[1] * da[1] + beta[2] * da[2] + d.ko;
+        // gt^kl d_l chi d_k alpha
+        double gdd = 0.0;
+#pragma unroll
+        for (int k = 0; k < 3; ++k)
+#pragma unroll
+          for (int l = 0; l < 3; ++l) gdd += gi[sidx(k, l)] * dchi[l] * da[k];
+        double DD[6];
+#pragma unroll
+        for (int i = 0; i < 3; ++i)
+#pragma unroll
+          for (int j = i; j < 3; ++j) {
+            const int q = sidx(i, j);
+            const double gk = SL(S0 + 0 * 6 + q) * da[0] + SL(S0 + 1 * 6 + q) * da[1] +
+                              SL(S0 + 2 * 6 + q) * da[2];
+            const double phys = gk - (0.5 * ichi) * (dchi[i] * da[j] + dchi[j] * da[i] - gt[q] * gdd);
+            DD[q] = d.dd[q] - phys;
+          }
+        const double trD = trace6(gi, DD);
+        rK += -chi * trD;
+#pragma unroll
+        for (int r = 0; r < 6; ++r) SL(A_AT + r) += -chi * (DD[r] - gt[r] * trD * (1.0 / 3.0));
+#pragma unroll
+        for (int i = 0; i < 3; ++i) {
+          double v = 0.0;
+#pragma unroll
+          for (int j = 0; j < 3; ++j) {
+            double a = 0.0;
+#pragma unroll
+            for (int k = 0; k < 3; ++k)
+#pragma unroll
+              for (int l = 0; l < 3; ++l) a += gi[sidx(i, k)] * gi[sidx(j, l)] * At[sidx(k, l)];
+            v += a * da[j];
+          }
+          SL(A_GT + i) += -2.0 * v;
+        }
+      } else if (f >= 3 && f <= 5) {
+        // ---------------- Gt^k: Ricci d Gt term, advection + KO kept apart (eq 3)
+        const int kk = f - 3;
+        const Derivs d = derivs<false>(s, c0, ih, ko_scale);
+        SL(S0 + kk) = beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
+        double gi[6], gt[6], Rg[6];
+#pragma unroll
+        for (int r = 0; r < 6; ++r) {
+          gi[r] = SL(G_INV + r);
+          gt[r] = SL(V_GAM + r);
+        }
+#pragma unroll
+        for (int i = 0; i < 3; ++i)
+#pragma unroll
+          for (int j = i; j < 3; ++j)
+            Rg[sidx(i, j)] = 0.5 * (gt[sidx(kk, i)] * d.d1[j] + gt[sidx(kk, j)] * d.d1[i]);
+        const double trR = trace6(gi, Rg);
+        const double ca = chi * alpha;
+#pragma unroll
+        for (int r = 0; r < 6; ++r) SL(A_AT + r) += ca * (Rg[r] - gt[r] * trR * (1.0 / 3.0));
+      } else if (f >= 6 && f <= 8) {
+        // ---------------- beta^kk: Lie derivative terms, eq (2), eq (8) shift terms
+        const int kk = f - 6;
+        const Derivs d = derivs<true>(s, c0, ih, ko_scale);
+        const double* db = d.d1;   // d_j beta^kk
+        SL(A_BETA + kk) += beta[0] * db[0] + beta[1] * db[1] + beta[2] * db[2] + d.ko;
+        double gi[6], cal[3];
+#pragma unroll
+        for (int r = 0; r < 6; ++r) gi[r] = SL(G_INV + r);
+#pragma unroll
+        for (int k = 0; k < 3; ++k) cal[k] = SL(S0 + 18 + k);
+        // Lie derivative pieces for T = gt and At:  T_i,kk d_j b + T_kk,j d_i b - 2/3 T_ij d_kk b
+#pragma unroll
+        for (int t = 0; t < 2; ++t) {
+          const int vb = t == 0 ? V_GAM : V_AT;
+          const int ab = t == 0 ? A_GAM : A_AT;
+          double T[6];
+#pragma unroll
+          for (int r = 0; r < 6; ++r) T[r] = SL(vb + r);
+#pragma unroll
+          for (int i = 0; i < 3; ++i)
+#pragma unroll
+            for (int j = i; j < 3; ++j) {
+              const int q = sidx(i, j);
+              SL(ab + q) += T[sidx(i, kk)] * db[j] + T[sidx(kk, j)] * db[i] -
+                            (2.0 / 3.0) * T[q] * db[kk];
+            }
+        }
+        rC += -(2.0 / 3.0) * chi * db[kk];
+        // Gt^kk += gt^jl d_jl beta^kk - CalGt^j d_j beta^kk
+        SL(A_GT + kk) += trace6(gi, d.dd) - (cal[0] * db[0] + cal[1] * db[1] + cal[2] * db[2]);
+        // Gt^i += 1/3 gt^ij d_j d_kk beta^kk + 2/3 CalGt^i d_kk beta^kk
+#pragma unroll
+        for (int i = 0; i < 3; ++i)
+          SL(A_GT + i) += (1.0 / 3.0) * (gi[sidx(i, 0)] * d.dd[sidx(0, kk)] +
+                                         gi[sidx(i, 1)] * d.dd[sidx(1, kk)] +
+                                         gi[sidx(i, 2)] * d.dd[sidx(2, kk)]) +
+                          (2.0 / 3.0) * cal[i] * db[kk];
+      } else if (f == 2) {
+        // ---------------- K: advection, KO, eq (8) -4/3 alpha gt^ij d_j K
+        const Derivs d = derivs<false>(s, c0, ih, ko_scale);
+        rK += beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
+        double gi[6];
+#pragma unroll
+        for (int r = 0; r < 6; ++r) gi[r] = SL(G_INV + r);
+#pragma unroll
+        for (int i = 0; i < 3; ++i)
+          SL(A_GT + i) += -(4.0 / 3.0) * alpha *
+                          (gi[sidx(i, 0)] * d.d1[0] + gi[sidx(i, 1)] * d.d1[1] +
+                           gi[sidx(i, 2)] * d.d1[2]);
+      } else if (f >= 18) {
+        const int q = f - 18;
+        const Derivs d = derivs<false>(s, c0, ih, ko_scale);
+        SL(A_AT + q) += beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
+      } else {  // 9..11: B
+        const int kk = f - 9;
+        const Derivs d = derivs<false>(s, c0, ih, ko_scale);
+        SL(A_B + kk) += beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
+      }
+    }
+    __syncthreads();  // everyone is done with this stage buffer
+    if (tid == 0 && st + 2 < NF)
+      bulk_load(stage + buf * STAGE_DBL, pbase + c_order[st + 2] * fstride, STAGE_DBL * 8,
+                &bars[buf]);
+  }
+
+  // ---- epilogue: undifferentiated terms, combine, store ----------------------
+  if (active) {
+    double gi[6], At[6], B[3];
+#pragma unroll
+    for (int r = 0; r < 6; ++r) {
+      gi[r] = SL(G_INV + r);
+      At[r] = SL(V_AT + r);
+    }
+#pragma unroll
+    for (int i = 0; i < 3; ++i) B[i] = SL(V_B + i);
+    double* out = rhs_oct + int64_t(e) * NPT + p;
+    const int64_t ostr = no * NPT;
+    // At^k_j and At_ik At^k_j, At_ij At^ij
+    double Am[3][3];
+#pragma unroll
+    for (int k = 0; k < 3; ++k)
+#pragma unroll
+      for (int j = 0; j < 3; ++j)
+        Am[k][j] = gi[sidx(k, 0)] * At[sidx(0, j)] + gi[sidx(k, 1)] * At[sidx(1, j)] +
+                   gi[sidx(k, 2)] * At[sidx(2, j)];
+    double AA = 0.0;
+#pragma unroll
+    for (int i = 0; i < 3; ++i)
+#pragma unroll
+      for (int j = 0; j < 3; ++j) AA += Am[i][j] * Am[j][i];
+    out[0 * ostr] = rA - 2.0 * alpha * Kv;                                        // (1)
+    out[1 * ostr] = rC + (2.0 / 3.0) * chi * alpha * Kv;                          // (5)
+    out[2 * ostr] = rK + alpha * (AA + Kv * Kv * (1.0 / 3.0));                    // (7)
+    const double fa = prm.lambda_f0 + prm.lambda_f1 * alpha;
+#pragma unroll
+    for (int i = 0; i < 3; ++i) {
+      const double gbar = SL(A_GT + i);
+      out[(3 + i) * ostr] = gbar + SL(S0 + i);                                    // (8)
+      out[(6 + i) * ostr] = SL(A_BETA + i) + 0.75 * fa * B[i];                    // (2)
+      out[(9 + i) * ostr] = gbar - prm.eta * B[i] + SL(A_B + i);                  // (3)
+    }
+#pragma unroll
+    for (int i = 0; i < 3; ++i)
+#pragma unroll
+      for (int j = i; j < 3; ++j) {
+        const int q = sidx(i, j);
+        out[(12 + q) * ostr] = SL(A_GAM + q) - 2.0 * alpha * At[q];               // (4)
+        const double AAij = At[sidx(i, 0)] * Am[0][j] + At[sidx(i, 1)] * Am[1][j] +
+                            At[sidx(i, 2)] * Am[2][j];
+        out[(18 + q) * ostr] = SL(A_AT + q) + alpha * (Kv * At[q] - 2.0 * AAij);  // (6)
+      }
+  }
+#undef SL
+}
+
+size_t rhs_smem_bytes() { return SMEM_BYTES; }
+
+void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const RhsParams& p,
+                cudaStream_t s) {
+  if (m.n_owned <= 0) return;
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(k_rhs, cudaFuncAttributeMaxDynamicSharedMemorySize, int(SMEM_BYTES));
+    attr = true;
+  }
+  k_rhs<<<m.n_owned, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p);
+}
+
+}  // namespace dgr

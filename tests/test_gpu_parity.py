@@ -1,0 +1,157 @@
+"""GPU parity: libdgr's CUDA path (through the C ABI) vs the CPU oracle.
+
+Bar (BASELINE.json north_star): fp64 fields within a max-abs-relative error of
+1e-10 per field for unzip, RHS and the RK4 state after one step, 1e-8 after
+100 steps; copy/injection points of the unzip are bit-exact.  Inputs are the
+seeded synthetic recipes of synth/ (DESIGN.md §Inputs).  Meshes are small
+enough for the oracle to finish in seconds yet span many patches, every
+padding kind, hanging chains and the extrapolated outer boundary.
+"""
+import numpy as np
+import pytest
+
+import paper_conf_sc_fernandonhzsgb22_b200 as dgr
+from oracle import bssn as obssn
+from oracle import constraints as ocon
+from oracle import rk4 as ork4
+from oracle import unzip as ouz
+from oracle.maps import OracleMesh
+from synth import configs, initial
+from synth.configs import MeshConfig, Puncture
+
+from .gpu_util import assert_parity, need_gpu, to_dev, torch
+
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-10
+
+
+def tiny_adaptive():
+    return MeshConfig(name="tiny", xmin=(-4.0, -4.0, -4.0), width=8.0, periodic=False,
+                      level_min=1, punctures=(Puncture(0.1, -0.2, 0.05, 1.0, 4),), rho=0.4)
+
+
+CASES = {
+    "c1_random": (configs.c1_uniform, "random"),
+    "c1_gauge_wave": (configs.c1_uniform, "gauge_wave"),
+    "small_bl": (lambda: configs.small_adaptive(lmax=5, rho=0.5), "bl"),
+    "small_random": (lambda: configs.small_adaptive(lmax=5, rho=0.5), "random"),
+    "bbh_chains_bl": (lambda: configs.small_bbh(lmax=6, rho=0.5), "bl"),
+}
+
+
+@pytest.fixture(scope="module", params=list(CASES))
+def case(request):
+    need_gpu()
+    cfgf, kind = CASES[request.param]
+    cfg = cfgf()
+    om = OracleMesh(cfg)
+    om.build_dofs()
+    u = initial.for_config(cfg, om.dof_coords(), kind=kind, seed=3)
+    m = dgr.Mesh(cfg)
+    assert m.info["n_dof_owned"] == om.n_dof
+    return request.param, cfg, om, m, u
+
+
+def test_dof_coords_device(case):
+    name, cfg, om, m, u = case
+    xyz = m.dof_coords()[:, :om.n_dof].cpu().numpy()
+    assert np.array_equal(xyz, om.dof_coords())
+
+
+def test_unzip_parity(case):
+    name, cfg, om, m, u = case
+    ud = to_dev(u, m.dof_stride)
+    P = m.unzip(ud)[:, :, :2197].cpu().numpy()
+    Po = ouz.unzip(om, u).reshape(24, om.n_oct, 2197)
+    src, kind = om.padding_sources()
+    k = kind & 7
+    # copy / inject / self points are bit-exact copies of (reconstructed) nodal values
+    cp = (k == 0) | (k == 1) | (k == 2)
+    hang_free_copy = cp & np.isin(src, np.nonzero(om.is_dof.all(axis=1))[0])
+    assert np.array_equal(P[:, hang_free_copy], Po[:, hang_free_copy])
+    assert_parity(P, Po, TOL, f"unzip {name}")
+
+
+def test_rhs_patches_parity(case):
+    """The RHS kernel alone, fed the oracle's own patches."""
+    name, cfg, om, m, u = case
+    Po = ouz.unzip(om, u).reshape(24, om.n_oct, 2197)
+    pt = torch.zeros((24, om.n_oct, m.info["patch_pitch"]), dtype=torch.float64, device="cuda")
+    pt[:, :, :2197] = torch.from_numpy(Po)
+    r = m.rhs_patches(pt).cpu().numpy()
+    ro = obssn.rhs_patches(Po, ork4.octant_h(om), obssn.Params()).reshape(24, om.n_oct, 343)
+    assert_parity(r, ro, TOL, f"rhs_patches {name}")
+
+
+def test_rhs_parity(case):
+    name, cfg, om, m, u = case
+    ud = to_dev(u, m.dof_stride)
+    r = m.rhs(ud)[:, :om.n_dof].cpu().numpy()
+    ro = ork4.rhs_dofs(om, u, obssn.Params())
+    assert_parity(r, ro, TOL, f"rhs {name}")
+
+
+def test_rk4_step_parity(case):
+    name, cfg, om, m, u = case
+    dt = ork4.dt_courant(om)
+    ud = to_dev(u, m.dof_stride)
+    m.rk4_step(ud, dt)
+    got = ud[:, :om.n_dof].cpu().numpy()
+    want = ork4.rk4_step(om, u, dt, obssn.Params())
+    assert_parity(got, want, TOL, f"rk4 step {name}")
+    # the update is not vacuous
+    assert np.max(np.abs(want - u)) > 0
+
+
+def test_rk4_stages_equal_step(case):
+    name, cfg, om, m, u = case
+    dt = ork4.dt_courant(om)
+    un = to_dev(u, m.dof_stride)
+    us = un.clone()
+    acc = torch.zeros_like(un)
+    for s in range(4):
+        m.rk4_stage(s, dt, un, us, acc)
+    ref = to_dev(u, m.dof_stride)
+    m.rk4_step(ref, dt)
+    assert torch.equal(acc[:, :om.n_dof], ref[:, :om.n_dof])
+
+
+def test_constraints_parity(case):
+    name, cfg, om, m, u = case
+    ud = to_dev(u, m.dof_stride)
+    c, norms = m.constraints(ud)
+    c = c[:, :om.n_dof].cpu().numpy()
+    co = ocon.constraints_dofs(om, u, obssn.Params())
+    assert_parity(c, co, 1e-9, f"constraints {name}")
+    no = ocon.norms(co)
+    assert np.allclose(norms, no, rtol=1e-9, atol=1e-300)
+
+
+def test_minkowski_rhs_exactly_zero():
+    need_gpu()
+    cfg = configs.small_bbh(lmax=6, rho=0.5)
+    m = dgr.Mesh(cfg)
+    u = initial.minkowski(m.dof_xyz_host())
+    r = m.rhs(to_dev(u, m.dof_stride))
+    assert torch.count_nonzero(r).item() == 0
+
+
+@pytest.mark.slow
+def test_100_steps_parity():
+    """RK4 state after 100 steps within 1e-8 of the oracle (adaptive BL mesh)."""
+    need_gpu()
+    cfg = tiny_adaptive()
+    om = OracleMesh(cfg)
+    om.build_dofs()
+    u = initial.for_config(cfg, om.dof_coords())
+    dt = ork4.dt_courant(om)
+    m = dgr.Mesh(cfg)
+    ud = to_dev(u, m.dof_stride)
+    prm = obssn.Params()
+    v = u.copy()
+    for _ in range(100):
+        m.rk4_step(ud, dt)
+        v = ork4.rk4_step(om, v, dt, prm)
+    got = ud[:, :om.n_dof].cpu().numpy()
+    assert_parity(got, v, 1e-8, "100 steps")

@@ -1,0 +1,342 @@
+"""Benchmark: fp64 BSSN RK4 step on a Brill-Lindquist BBH octree (libdgr, B200).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c3] [--impl reference]
+    python -m torch.distributed.run --nproc-per-node N ... bench.py --gpus N ...
+
+Metric (BASELINE.json): "BSSN RHS fp64 GFLOP/s & RK4 step time (grid pts/s)".
+`value` = unique grid points (DOFs) advanced by one full RK4 step per second,
+summed over ranks (whole job), inputs resident in HBM.  Default workload:
+configs[2], Brill-Lindquist q=1, levels 3..12, rho=2.5 (24,284 octants,
+5.07M DOFs = 121.6M unknowns; the paper's 125M-unknown strong-scaling case,
+P:L440) — the config the metric's "at 1/2/4/8 B200" is quoted on.  With N>1
+the octree is partitioned along the Morton curve (strong scaling) and ghost
+DOFs are exchanged with NCCL every RK stage.
+
+One JSON line on rank 0 (the driver's contract).  L2 hygiene: every stage
+streams the 10.2 GB patch buffer (>> 126 MB L2), so inputs are larger than L2.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "BSSN RHS fp64 GFLOP/s & RK4 step time (grid pts/s) at 1/2/4/8 B200"
+UNIT = "grid-pts/s"
+
+# Algorithmic work per unit:
+UNZIP_BYTES_PER_OCT = 24 * (2197 + 216) * 8       # write every patch point, read every DOF once
+ZIP_BYTES_PER_DOF_STAGE = 24 * 34                 # avg over the 4 stages of read k,u_n,acc / write acc,u_s
+ELEM_BYTES_PER_OCT = 24 * 343 * (8 + 8) + 343 * 4  # E write + u gather + O2N read
+RHS_BYTES_PER_OCT = 24 * (2197 + 343) * 8         # patch read + rhs write (eq 21a denominator)
+PAPER_FLOPS_PER_POINT = 5502 + 3998               # eq (21a) numerator per point, O_A from Q_L = 6.68
+# executed fp64 FLOPs per interior point of k_rhs (2 per DFMA + DADD + DMUL), from
+# ncu sm__sass_thread_inst_executed_op_d{fma,add,mul}_pred_on (profiles/)
+RHS_EXEC_FLOPS_PER_POINT = float(os.environ.get("DGR_RHS_FLOPS_PER_POINT", "0")) or None
+
+
+def _peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d.get("hbm_gbs", 6650.0), d.get("sm_max_mhz", 1965.0), "measured"
+    return 6650.0, 1965.0, "fallback"
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+
+    def __init__(self, index):
+        self.index = index
+        self.samples = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def __enter__(self):
+        q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+        def run():
+            while not self._stop.is_set():
+                try:
+                    out = subprocess.run(["nvidia-smi", "-i", str(self.index),
+                                          f"--query-gpu={q}", "--format=csv,noheader,nounits"],
+                                         capture_output=True, text=True, timeout=5).stdout
+                    f = [x.strip() for x in out.strip().split(",")]
+                    if len(f) >= 8:
+                        self.samples.append(f)
+                except Exception:
+                    pass
+                self._stop.wait(0.2)
+
+        self._t = threading.Thread(target=run, daemon=True)
+        self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        self._t.join(timeout=10)
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"],
+                    "samples": 0}
+        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for s in self.samples for i in range(4)
+                          if s[4 + i].lower().startswith("active")})
+        return {"sm_mhz": float(np.median(sm)) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": reasons,
+                "samples": len(self.samples)}
+
+
+def cpu_baseline_oracle(cfg, n_sample, reps=1):
+    """The oracle as it stands, on the host cores, bounded sample of the
+    workload: element reconstruction for ALL octants + octant-to-patch and
+    RHS for `n_sample` random octants; one RK4 step = 4 such stages over all
+    octants, extrapolated linearly in the octant count."""
+    from threadpoolctl import threadpool_limits
+
+    from oracle import bssn, rk4, unzip
+    from oracle.maps import OracleMesh
+    from synth import initial
+    om = OracleMesh(cfg)
+    om.build_dofs()
+    u = initial.for_config(cfg, om.dof_coords())
+    octs = np.random.default_rng(0).choice(om.n_oct, min(n_sample, om.n_oct), replace=False)
+    h = rk4.octant_h(om)
+    om.padding_sources(octs[:2])          # warm imports / caches outside the timing
+    times = []
+    with threadpool_limits(limits=1):
+        for _ in range(reps):
+            t0 = time.perf_counter()
+            unzip.elements(om, u)
+            t1 = time.perf_counter()
+            P = unzip.unzip(om, u, octs)
+            bssn.rhs_patches(P, h[octs], bssn.Params())
+            t2 = time.perf_counter()
+            # unzip() recomputed the elements: subtract that copy
+            stage = (t1 - t0) + (t2 - t1 - (t1 - t0)) * om.n_oct / len(octs)
+            times.append(4.0 * stage)
+    step_s = float(np.median(times))
+    return {"value": om.n_dof / step_s, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": (f"1 RK4 step = 4 x (elements for all {om.n_oct} octants + unzip+RHS of "
+                       f"{len(octs)} random octants scaled to {om.n_oct}); NumPy, 1 thread"),
+            "step_s": step_s}
+
+
+def run_reference(args, cfg):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    cb = cpu_baseline_oracle(cfg, n_sample=64, reps=args.warmup + args.steps)
+    line = {"impl": "reference", "metric": METRIC, "value": cb["value"], "unit": UNIT,
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": cb["step_s"] * 1e3, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic Brill-Lindquist",
+            "config": {"workload": cfg.name + ": " + cfg.description},
+            "cpu_baseline": {k: cb[k] for k in ("value", "unit", "cores", "kind", "sample")},
+            "e2e": {"value": cb["value"], "unit": UNIT, "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="c3")
+    ap.add_argument("--impl", default="dgr", choices=["dgr", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-sample", type=int, default=128)
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    from synth import configs, initial
+    cfg = configs.get(args.config)
+    if args.impl == "reference":
+        return run_reference(args, cfg)
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_sc_fernandonhzsgb22_b200 as dgr
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    nccl_id = None
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        obj = [bytes(torch.cuda.nccl.unique_id()) if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        nccl_id = obj[0]
+
+    octs = dgr.octree_build(cfg)
+    mesh = dgr.Mesh(cfg, octs, rank=rank, nranks=world, nccl_id=nccl_id)
+    info = mesh.info
+    xyz = mesh.dof_xyz_host()
+    u = torch.zeros((24, mesh.dof_stride), dtype=torch.float64, device="cuda")
+    u[:, :xyz.shape[1]] = torch.from_numpy(initial.for_config(cfg, xyz))
+    dt = 0.25 * info["h_min"]
+    prm = dgr.Params()
+
+    # fp64 roofline denominator: DFMA microbenchmark on this device
+    dfma_ms, dfma_fl = dgr.bench_dfma(148 * 8, 20000)
+    dfma_tflops = dfma_fl / dfma_ms / 1e9
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    for _ in range(args.warmup):
+        mesh.rk4_step(u, dt, prm)
+    torch.cuda.synchronize()
+    launches_per_step = mesh.last_launch_count()
+
+    # ---- timed region: device-resident state
+    mesh.profile_read(reset=True)
+    mesh.profile_enable(True)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    barrier()
+    torch.cuda.synchronize()
+    with Clocks(local) as clk:
+        e0.record()
+        for _ in range(args.steps):
+            mesh.rk4_step(u, dt, prm)
+        e1.record()
+        torch.cuda.synchronize()
+    barrier()
+    mesh.profile_enable(False)
+    prof = mesh.profile_read(reset=True)
+    ms = e0.elapsed_time(e1) / args.steps
+    t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_max = float(t.item())
+    n_dof = info["n_dof_global"]
+    value = n_dof / (ms_max * 1e-3)
+    finite = bool(torch.isfinite(u[:, :info["n_dof_owned"]]).all())
+
+    # ---- end to end through the public API with host buffers
+    n_loc = info["n_dof_owned"] + info["n_dof_ghost"]
+    host_in = torch.empty((24, mesh.dof_stride), dtype=torch.float64, pin_memory=True)
+    host_in.copy_(u.cpu())
+    host_out = torch.empty_like(host_in)
+    ud = torch.empty_like(u)
+    for _ in range(1):
+        ud.copy_(host_in, non_blocking=True)
+        mesh.rk4_step(ud, dt, prm)
+        host_out.copy_(ud, non_blocking=True)
+    torch.cuda.synchronize()
+    barrier()
+    e0.record()
+    for _ in range(args.steps):
+        ud.copy_(host_in, non_blocking=True)
+        mesh.rk4_step(ud, dt, prm)
+        host_out.copy_(ud, non_blocking=True)
+    e1.record()
+    torch.cuda.synchronize()
+    barrier()
+    ms_e2e = e0.elapsed_time(e1) / args.steps
+    t = torch.tensor([ms_e2e], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_e2e = float(t.item())
+    bytes_io = 24 * n_loc * 8
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    # ---- rooflines of the kernels, from the CUDA-event profile of the timed region
+    hbm_peak, sm_max_mhz, peak_kind = _peaks()
+    fp64_peak = 148 * 64 * 2 * sm_max_mhz * 1e6 / 1e12         # TFLOP/s, unit counts x max clock
+    no, nl = info["n_oct_local"], info["n_oct_local"] + info["n_oct_ghost"]
+    kern = {}
+    for name, (tot_ms, n) in prof.items():
+        avg = tot_ms / max(n, 1)
+        kern[name] = {"ms_per_launch": avg, "launches": n, "ms_per_step": tot_ms / args.steps}
+    def hbm(name, bytes_per_launch):
+        k = kern.get(name)
+        if not k:
+            return None
+        ach = bytes_per_launch / (k["ms_per_launch"] * 1e-3) / 1e9
+        k.update({"bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s",
+                  "frac": ach / hbm_peak, "algorithmic_bytes_per_launch": bytes_per_launch})
+    hbm("unzip", UNZIP_BYTES_PER_OCT * no)
+    hbm("elements", ELEM_BYTES_PER_OCT * nl)
+    hbm("zip_rk4", ZIP_BYTES_PER_DOF_STAGE * info["n_dof_owned"])
+    if "rhs" in kern:
+        k = kern["rhs"]
+        sec = k["ms_per_launch"] * 1e-3
+        pts = no * 343
+        nominal = pts * PAPER_FLOPS_PER_POINT / sec / 1e12
+        k["paper_nominal_tflops"] = nominal
+        k["hbm_GBps_algorithmic"] = RHS_BYTES_PER_OCT * no / sec / 1e9
+        if RHS_EXEC_FLOPS_PER_POINT:
+            ach = pts * RHS_EXEC_FLOPS_PER_POINT / sec / 1e12
+            k.update({"bound": "alu", "achieved": ach, "peak": fp64_peak, "unit": "TFLOP/s",
+                      "frac": ach / fp64_peak, "peak_measured_dfma": dfma_tflops})
+        else:
+            k.update({"bound": "alu", "achieved": nominal, "peak": fp64_peak, "unit": "TFLOP/s",
+                      "frac": nominal / fp64_peak, "flops": "paper-nominal (eq 21a)",
+                      "peak_measured_dfma": dfma_tflops})
+    dom = max(kern, key=lambda n: kern[n]["ms_per_step"]) if kern else None
+    roof = None
+    if dom and "bound" in kern[dom]:
+        k = kern[dom]
+        roof = {"kernel": dom, "bound": k["bound"], "achieved": k["achieved"], "peak": k["peak"],
+                "unit": k["unit"], "frac": k["frac"], "traffic": None,
+                "peak_source": (f"MEASURED_PEAKS.json ({peak_kind})" if k["bound"] == "hbm" else
+                                "148 SM x 64 DFMA/clk x 2 x sm_max_mhz (derived)")}
+    cpu = None
+    if world == 1 and not args.no_cpu_baseline:
+        try:
+            cb = cpu_baseline_oracle(cfg, n_sample=args.cpu_sample)
+            cpu = {k: cb[k] for k in ("value", "unit", "cores", "kind", "sample")}
+        except Exception as ex:  # noqa: BLE001
+            cpu = {"value": None, "unit": UNIT, "cores": 1, "kind": "oracle",
+                   "sample": f"failed: {ex}"}
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_max, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic Brill-Lindquist puncture data (seeded, synth/initial.py)",
+        "config": {"workload": f"{cfg.name}: {cfg.description}", "octants": info["n_oct_global"],
+                   "dofs": n_dof, "unknowns": 24 * n_dof, "levels": [info["level_min"],
+                                                                    info["level_max"]],
+                   "dt": dt, "l2": "inputs larger than L2 (10 GB patch buffer per stage)",
+                   "parallelism": f"morton-partition x{world}"},
+        "rhs_gflops": (kern.get("rhs", {}).get("achieved", 0) * 1e3) or None,
+        "roofline": roof,
+        "kernels": kern,
+        "fp64_dfma_tflops_measured": dfma_tflops,
+        "cpu_baseline": cpu,
+        "e2e": {"value": n_dof / (ms_e2e * 1e-3), "unit": UNIT, "h2d_bytes_per_step": bytes_io,
+                "d2h_bytes_per_step": bytes_io, "ms_per_step": ms_e2e},
+        "gpu_launches": launches_per_step * args.steps,
+        "clocks": clk.summary(),
+        "finite": finite,
+    }
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

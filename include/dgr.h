@@ -208,6 +208,21 @@ dgr_status dgr_constraints(dgr_mesh m, double* u, double* c, double* norms_host,
  * dgr_rk4_step / dgr_rhs enqueued. */
 int64_t dgr_last_launch_count(dgr_mesh m);
 
+/* Per-kernel device timing: when enabled, every libdgr launch is bracketed by
+ * CUDA events recorded on the launching stream.  dgr_profile_read synchronises
+ * and returns, per kernel class, the summed milliseconds and launch counts
+ * since the last reset (classes: 0 elements, 1 hanging, 2 unzip, 3 rhs,
+ * 4 zip/zip+rk4, 5 ghost pack/exchange, 6 constraints, 7 other). */
+enum { DGR_PROF_CLASSES = 8 };
+dgr_status dgr_profile_enable(dgr_mesh m, int on);
+dgr_status dgr_profile_read(dgr_mesh m, double* ms, int64_t* counts, int reset);
+
+/* fp64 FMA throughput microbenchmark on the current device: `blocks` CTAs of
+ * 256 threads, each thread running 8 independent DFMA chains for `iters`
+ * iterations.  Returns the elapsed device milliseconds and the FLOP count
+ * (2 per DFMA).  Used to measure the fp64 roofline denominator. */
+dgr_status dgr_bench_dfma(int blocks, int iters, void* stream, double* ms, double* flops);
+
 #ifdef __cplusplus
 }
 #endif

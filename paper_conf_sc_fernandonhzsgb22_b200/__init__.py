@@ -73,7 +73,10 @@ _lib = None
 EXPORTED = ["dgr_status_string", "dgr_last_error", "dgr_version", "dgr_octree_build",
             "dgr_mesh_create", "dgr_mesh_info_get", "dgr_mesh_export_maps", "dgr_mesh_destroy",
             "dgr_dof_coords", "dgr_unzip", "dgr_ghost_exchange", "dgr_rhs_patches", "dgr_rhs",
-            "dgr_rk4_stage", "dgr_rk4_step", "dgr_constraints", "dgr_last_launch_count"]
+            "dgr_rk4_stage", "dgr_rk4_step", "dgr_constraints", "dgr_last_launch_count",
+            "dgr_profile_enable", "dgr_profile_read", "dgr_bench_dfma"]
+PROF_CLASSES = ["elements", "hanging", "unzip", "rhs", "zip_rk4", "exchange", "constraints",
+                "other"]
 
 
 def lib():
@@ -104,10 +107,14 @@ def lib():
         L.dgr_constraints.argtypes = [vp, vp, vp, vp, C.POINTER(_Params), vp]
         L.dgr_last_launch_count.restype = i64
         L.dgr_last_launch_count.argtypes = [vp]
+        L.dgr_profile_enable.argtypes = [vp, i32]
+        L.dgr_profile_read.argtypes = [vp, vp, vp, i32]
+        L.dgr_bench_dfma.argtypes = [i32, i32, vp, C.POINTER(dp), C.POINTER(dp)]
         for f in ["dgr_octree_build", "dgr_mesh_create", "dgr_mesh_info_get",
                   "dgr_mesh_export_maps", "dgr_mesh_destroy", "dgr_dof_coords", "dgr_unzip",
                   "dgr_ghost_exchange", "dgr_rhs_patches", "dgr_rhs", "dgr_rk4_stage",
-                  "dgr_rk4_step", "dgr_constraints"]:
+                  "dgr_rk4_step", "dgr_constraints", "dgr_profile_enable", "dgr_profile_read",
+                  "dgr_bench_dfma"]:
             getattr(L, f).restype = i32
         _lib = L
     return _lib
@@ -284,3 +291,20 @@ class Mesh:
 
     def last_launch_count(self):
         return int(lib().dgr_last_launch_count(self._h))
+
+    def profile_enable(self, on=True):
+        _check(lib().dgr_profile_enable(self._h, int(on)))
+
+    def profile_read(self, reset=True):
+        """{class: (ms, launches)} of libdgr kernels since the last reset (CUDA events)."""
+        ms = np.zeros(8)
+        n = np.zeros(8, dtype=np.int64)
+        _check(lib().dgr_profile_read(self._h, ms.ctypes.data, n.ctypes.data, int(reset)))
+        return {PROF_CLASSES[i]: (float(ms[i]), int(n[i])) for i in range(8) if n[i]}
+
+
+def bench_dfma(blocks=148 * 8, iters=200000):
+    """(ms, flops) of the fp64 FMA microbenchmark on the current device."""
+    ms, fl = C.c_double(), C.c_double()
+    _check(lib().dgr_bench_dfma(blocks, iters, _stream(), C.byref(ms), C.byref(fl)))
+    return ms.value, fl.value

@@ -109,6 +109,19 @@ struct dgr_mesh_s {
   double* d_sendbuf = nullptr;
   double* d_recvbuf = nullptr;
   int64_t launches = 0;
+  // profiling
+  bool prof = false;
+  struct Pend { int cls; cudaEvent_t a, b; };
+  std::vector<Pend> pend;
+  std::vector<cudaEvent_t> pool;
+  double prof_ms[DGR_PROF_CLASSES] = {0};
+  int64_t prof_n[DGR_PROF_CLASSES] = {0};
+  cudaEvent_t ev() {
+    if (!pool.empty()) { cudaEvent_t e = pool.back(); pool.pop_back(); return e; }
+    cudaEvent_t e = nullptr;
+    cudaEventCreate(&e);
+    return e;
+  }
 
   template <class T>
   cudaError_t alloc(T** p, size_t n) {
@@ -121,6 +134,8 @@ struct dgr_mesh_s {
     return e;
   }
   ~dgr_mesh_s() {
+    for (auto& p : pend) { cudaEventDestroy(p.a); cudaEventDestroy(p.b); }
+    for (auto e : pool) cudaEventDestroy(e);
     for (void* q : allocs) cudaFree(q);
     if (comm && g_nccl.CommDestroy) g_nccl.CommDestroy(comm);
   }
@@ -442,14 +457,30 @@ static dgr_status need_device(dgr_mesh m) {
 
 static bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; }
 
+// Bracket one launch with CUDA events on its stream when profiling is on.
+#define PROF(m, cls, st, stmt)                                   \
+  do {                                                           \
+    cudaEvent_t _a = nullptr;                                    \
+    if ((m)->prof) {                                             \
+      _a = (m)->ev();                                            \
+      cudaEventRecord(_a, (st));                                 \
+    }                                                            \
+    stmt;                                                        \
+    ++(m)->launches;                                             \
+    if ((m)->prof) {                                             \
+      cudaEvent_t _b = (m)->ev();                                \
+      cudaEventRecord(_b, (st));                                 \
+      (m)->pend.push_back({(cls), _a, _b});                      \
+    }                                                            \
+  } while (0)
+
 // ghost exchange: pack owned DOFs each peer needs, grouped send/recv, unpack
 static dgr_status exchange(dgr_mesh m, double* u, cudaStream_t st) {
   const HostMesh& h = m->host;
   if (h.nranks <= 1) return DGR_OK;
   const int64_t stride = m->dm.dof_stride;
   const int64_t nsend = int64_t(h.send_list.size());
-  launch_gather_pack(u, stride, m->d_send, nsend, m->d_sendbuf, st);
-  ++m->launches;
+  PROF(m, 5, st, launch_gather_pack(u, stride, m->d_send, nsend, m->d_sendbuf, st));
   CUDA_TRY(cudaGetLastError());
   // sendbuf is [f][nsend] with peers contiguous inside each field row; send
   // one message per (peer, field) row segment inside a single group
@@ -469,15 +500,12 @@ static dgr_status exchange(dgr_mesh m, double* u, cudaStream_t st) {
 }
 
 static dgr_status do_unzip(dgr_mesh m, const double* u, int nf, cudaStream_t st) {
-  launch_elements(m->dm, u, m->d_E, nf, st);
-  ++m->launches;
+  PROF(m, 0, st, launch_elements(m->dm, u, m->d_E, nf, st));
   for (size_t g = 0; g + 1 < m->hang_level_off.size(); ++g) {
     const int64_t a = m->hang_level_off[g], b = m->hang_level_off[g + 1];
-    launch_hanging(m->dm, m->d_hang + a, b - a, m->d_E, nf, st);
-    ++m->launches;
+    PROF(m, 1, st, launch_hanging(m->dm, m->d_hang + a, b - a, m->d_E, nf, st));
   }
-  launch_unzip(m->dm, m->d_E, m->d_patch, nf, st);
-  ++m->launches;
+  PROF(m, 2, st, launch_unzip(m->dm, m->d_E, m->d_patch, nf, st));
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;
 }
@@ -524,7 +552,8 @@ dgr_status dgr_rhs_patches(dgr_mesh m, const double* patches, double* rhs_oct,
   dgr_status s = need_device(m);
   if (s) return s;
   if (!patches || !rhs_oct || !aligned16(patches)) return fail(DGR_ERR_ARG, "bad rhs args");
-  launch_rhs(m->dm, patches, rhs_oct, to_rp(prm), static_cast<cudaStream_t>(stream));
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  PROF(m, 3, st, launch_rhs(m->dm, patches, rhs_oct, to_rp(prm), st));
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;
 }
@@ -537,9 +566,8 @@ dgr_status dgr_rhs(dgr_mesh m, double* u, double* rhs, const dgr_params* prm, vo
   m->launches = 0;
   if ((s = exchange(m, u, st))) return s;
   if ((s = do_unzip(m, u, NF, st))) return s;
-  launch_rhs(m->dm, m->d_patch, m->d_rhs_oct, to_rp(prm), st);
-  launch_zip(m->dm, m->d_rhs_oct, rhs, NF, st);
-  m->launches += 2;
+  PROF(m, 3, st, launch_rhs(m->dm, m->d_patch, m->d_rhs_oct, to_rp(prm), st));
+  PROF(m, 4, st, launch_zip(m->dm, m->d_rhs_oct, rhs, NF, st));
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;
 }
@@ -550,9 +578,8 @@ static dgr_status stage(dgr_mesh m, int s_, double dt, double* u_n, double* u_s,
   double* cur = s_ == 0 ? u_n : u_s;
   if ((s = exchange(m, cur, st))) return s;
   if ((s = do_unzip(m, cur, NF, st))) return s;
-  launch_rhs(m->dm, m->d_patch, m->d_rhs_oct, to_rp(prm), st);
-  launch_zip_rk4(m->dm, m->d_rhs_oct, s_, dt, u_n, u_s, acc, u_out, st);
-  m->launches += 2;
+  PROF(m, 3, st, launch_rhs(m->dm, m->d_patch, m->d_rhs_oct, to_rp(prm), st));
+  PROF(m, 4, st, launch_zip_rk4(m->dm, m->d_rhs_oct, s_, dt, u_n, u_s, acc, u_out, st));
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;
 }
@@ -586,12 +613,12 @@ dgr_status dgr_constraints(dgr_mesh m, double* u, double* c, double* norms_host,
   m->launches = 0;
   if ((s = exchange(m, u, st))) return s;
   if ((s = do_unzip(m, u, NF, st))) return s;
-  launch_constraints(m->dm, m->d_patch, m->d_rhs_oct, to_rp(prm), st);
+  PROF(m, 6, st, launch_constraints(m->dm, m->d_patch, m->d_rhs_oct, to_rp(prm), st));
   CUDA_TRY(cudaGetLastError());
   // zip the 7 constraint fields
   const int64_t stride = m->dm.dof_stride;
   DevMesh dm = m->dm;
-  launch_zip(dm, m->d_rhs_oct, c, 7, st);
+  PROF(m, 4, st, launch_zip(dm, m->d_rhs_oct, c, 7, st));
   CUDA_TRY(cudaGetLastError());
   if (norms_host) {
     const int64_t n = m->host.n_owned_dof;
@@ -636,6 +663,58 @@ dgr_status dgr_constraints(dgr_mesh m, double* u, double* c, double* norms_host,
       norms_host[2 * q + 1] = part[2 * q + 1];
     }
   }
+  return DGR_OK;
+}
+
+dgr_status dgr_profile_enable(dgr_mesh m, int on) {
+  if (!m) return fail(DGR_ERR_ARG, "null mesh");
+  m->prof = on != 0;
+  return DGR_OK;
+}
+
+dgr_status dgr_profile_read(dgr_mesh m, double* ms, int64_t* counts, int reset) {
+  if (!m) return fail(DGR_ERR_ARG, "null mesh");
+  for (auto& p : m->pend) {
+    CUDA_TRY(cudaEventSynchronize(p.b));
+    float t = 0.f;
+    CUDA_TRY(cudaEventElapsedTime(&t, p.a, p.b));
+    m->prof_ms[p.cls] += double(t);
+    m->prof_n[p.cls] += 1;
+    m->pool.push_back(p.a);
+    m->pool.push_back(p.b);
+  }
+  m->pend.clear();
+  for (int c = 0; c < DGR_PROF_CLASSES; ++c) {
+    if (ms) ms[c] = m->prof_ms[c];
+    if (counts) counts[c] = m->prof_n[c];
+    if (reset) {
+      m->prof_ms[c] = 0;
+      m->prof_n[c] = 0;
+    }
+  }
+  return DGR_OK;
+}
+
+dgr_status dgr_bench_dfma(int blocks, int iters, void* stream, double* ms, double* flops) {
+  if (blocks <= 0 || iters <= 0 || !ms || !flops) return fail(DGR_ERR_ARG, "bad dfma args");
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  double* out = nullptr;
+  CUDA_TRY(cudaMalloc(&out, 8));
+  cudaEvent_t a, b;
+  CUDA_TRY(cudaEventCreate(&a));
+  CUDA_TRY(cudaEventCreate(&b));
+  launch_dfma(blocks, 16, out, st);  // warm-up
+  CUDA_TRY(cudaEventRecord(a, st));
+  launch_dfma(blocks, iters, out, st);
+  CUDA_TRY(cudaEventRecord(b, st));
+  CUDA_TRY(cudaEventSynchronize(b));
+  float t = 0.f;
+  CUDA_TRY(cudaEventElapsedTime(&t, a, b));
+  cudaEventDestroy(a);
+  cudaEventDestroy(b);
+  cudaFree(out);
+  *ms = double(t);
+  *flops = double(blocks) * 256.0 * 8.0 * double(iters) * 2.0;
   return DGR_OK;
 }
 

@@ -43,6 +43,8 @@ void launch_gather_pack(const double* u, int64_t stride, const int32_t* list, in
 void launch_scatter_unpack(double* u, int64_t stride, int64_t offset, const double* buf,
                            int64_t n_total, cudaStream_t s);
 
+void launch_dfma(int blocks, int iters, double* out, cudaStream_t s);
+
 // rhs_kernel.cu
 struct RhsParams {
   double ko_sigma, eta, lambda_f0, lambda_f1, chi_floor;

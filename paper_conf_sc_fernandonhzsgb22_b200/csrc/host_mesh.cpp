@@ -690,7 +690,22 @@ void HostMesh::build_padding() {
         ne.o[k] = int16_t(num / sc);
       }
       ne.pad = 0;
+      ne.pad2[0] = ne.pad2[1] = 0;
+      for (int k = 0; k < 3; ++k) {
+        ne.lo[k] = 12;
+        ne.hi[k] = 0;
+      }
       nbr[size_t(lb) * NBR_MAX + remap[jt]] = ne;
+    }
+    for (int p = 0; p < NPATCH; ++p) {
+      const int jn = pm[p];
+      if (jn >= nn) continue;
+      NbrEntry& ne = nbr[size_t(lb) * NBR_MAX + jn];
+      const int idx[3] = {p % 13, (p / 13) % 13, p / 169};
+      for (int k = 0; k < 3; ++k) {
+        ne.lo[k] = uint8_t(std::min<int>(ne.lo[k], idx[k]));
+        ne.hi[k] = uint8_t(std::max<int>(ne.hi[k], idx[k]));
+      }
     }
   }
   if (bad) throw BuildError{-2, "padding map construction failed"};

@@ -46,7 +46,10 @@ struct NbrEntry {
   int16_t o[3];
   uint8_t r;     // 1 (source coarser), 2 (same level), 4 (finer)
   uint8_t pad;
+  uint8_t lo[3], hi[3];  // bounding box (patch indices) of the points it sources
+  uint8_t pad2[2];
 };
+static_assert(sizeof(NbrEntry) == 20, "NbrEntry layout");
 
 struct BuildError {
   int code;

@@ -98,46 +98,124 @@ void launch_hanging(const DevMesh& m, const int4* rows, int64_t count, double* E
 }
 
 // ------------------------------------------------------------------ unzip
+// One CTA per patch, fields in sequence.  Phase A: points sourced from the
+// octant itself, a same-level or a finer neighbour are single loads (their
+// half-grid coordinates are even); points sourced from a coarser neighbour c
+// are produced by three 1D Lagrange sweeps over c's 7^3 nodes staged in shared
+// memory, restricted to the bounding box of the points c sources (the
+// tensor-product interpolation of P:L295).  Phase B: outer-boundary
+// extrapolation (reading R12).  The finished 13^3 patch leaves shared memory
+// with coalesced stores.
 constexpr int UZ_THREADS = 256;
 
 __global__ void __launch_bounds__(UZ_THREADS) k_unzip(DevMesh m, const double* __restrict__ E,
                                                       double* __restrict__ patches, int nf) {
   __shared__ __align__(16) double P[NPATCH + 3];
+  __shared__ double Es[NPT + 1];
+  __shared__ double T1[7 * 7 * 13];
+  __shared__ double T2[7 * 13 * 13];
   __shared__ uint8_t pm[NPATCH + 11];
   __shared__ NbrEntry nb[NBR_MAX];
   __shared__ double W[91];
   __shared__ double WX[21];
+  __shared__ int coarse[8];
+  __shared__ int n_coarse;
   const int e = blockIdx.x;
   const int tid = threadIdx.x;
   for (int i = tid; i < NPATCH; i += UZ_THREADS) pm[i] = m.pmap[int64_t(e) * NPATCH + i];
   for (int i = tid; i < NBR_MAX; i += UZ_THREADS) nb[i] = m.nbr[int64_t(e) * NBR_MAX + i];
   for (int i = tid; i < 91; i += UZ_THREADS) W[i] = c_W13[i];
   for (int i = tid; i < 21; i += UZ_THREADS) WX[i] = c_WEXT[i];
+  __syncthreads();
+  if (tid == 0) {
+    int nc = 0;
+    for (int j = 0; j < NBR_MAX && nc < 8; ++j)
+      if (nb[j].r == 1) coarse[nc++] = j;
+    n_coarse = nc;
+  }
   const int4 o = m.oct[e];
   const int64_t nside = int64_t(1) << m.D;
   const int64_t s = int64_t(1) << (m.D - o.w);
-  // which faces of the patch lie outside a non-periodic domain
   const bool out_lo[3] = {!m.periodic && o.x == 0, !m.periodic && o.y == 0,
                           !m.periodic && o.z == 0};
   const bool out_hi[3] = {!m.periodic && o.x + s == nside, !m.periodic && o.y + s == nside,
                           !m.periodic && o.z + s == nside};
   const bool any_out = out_lo[0] || out_lo[1] || out_lo[2] || out_hi[0] || out_hi[1] || out_hi[2];
   __syncthreads();
+  const int nc = n_coarse;
   const int64_t nn = int64_t(m.n_local) * NPT;
   for (int f = 0; f < nf; ++f) {
     const double* Ef = E + f * nn;
+    // ---- phase A.1: self / same level / finer: one load per point
     for (int p = tid; p < NPATCH; p += UZ_THREADS) {
       const int j = pm[p];
       const int ix = p % 13, iy = (p / 13) % 13, iz = p / 169;
-      double v = 0.0;
       if (j == PM_SELF) {
-        v = __ldg(Ef + int64_t(e) * NPT + (ix - 3) + 7 * (iy - 3) + 49 * (iz - 3));
-      } else if (j != PM_EXTRAP) {
-        const NbrEntry t = nb[j];
-        const int tx = t.o[0] + t.r * ix, ty = t.o[1] + t.r * iy, tz = t.o[2] + t.r * iz;
-        v = interp_point(Ef + int64_t(t.src) * NPT, tx, ty, tz, W);
+        P[p] = __ldg(Ef + int64_t(e) * NPT + (ix - 3) + 7 * (iy - 3) + 49 * (iz - 3));
+      } else if (j != PM_EXTRAP && nb[j].r != 1) {
+        const NbrEntry& t = nb[j];
+        const int tx = (t.o[0] + t.r * ix) >> 1, ty = (t.o[1] + t.r * iy) >> 1,
+                  tz = (t.o[2] + t.r * iz) >> 1;
+        P[p] = __ldg(Ef + int64_t(t.src) * NPT + tx + 7 * ty + 49 * tz);
       }
-      P[p] = v;
+    }
+    // ---- phase A.2: coarser neighbours, separable sweeps x -> y -> z
+    for (int ci = 0; ci < nc; ++ci) {
+      const int j = coarse[ci];
+      const NbrEntry t = nb[j];
+      __syncthreads();   // previous users of Es / T1 / T2 are done
+      const double* Ec = Ef + int64_t(t.src) * NPT;
+      for (int i = tid; i < NPT; i += UZ_THREADS) Es[i] = __ldg(Ec + i);
+      const int lx = t.lo[0], ly = t.lo[1], lz = t.lo[2];
+      const int nx = t.hi[0] - lx + 1, ny = t.hi[1] - ly + 1, nz = t.hi[2] - lz + 1;
+      __syncthreads();
+      for (int idx = tid; idx < 49 * nx; idx += UZ_THREADS) {
+        const int cyz = idx / nx, ix = idx % nx;        // cyz = cz * 7 + cy
+        const int tx = t.o[0] + lx + ix;
+        const double* row = Es + cyz * 7;
+        double v;
+        if (tx & 1) {
+          const double* w = W + tx * 7;
+          v = 0.0;
+#pragma unroll
+          for (int a = 0; a < 7; ++a) v = fma(w[a], row[a], v);
+        } else {
+          v = row[tx >> 1];
+        }
+        T1[cyz * 13 + ix] = v;
+      }
+      __syncthreads();
+      for (int idx = tid; idx < 7 * ny * nx; idx += UZ_THREADS) {
+        const int ix = idx % nx, iy = (idx / nx) % ny, cz = idx / (nx * ny);
+        const int ty = t.o[1] + ly + iy;
+        double v;
+        if (ty & 1) {
+          const double* w = W + ty * 7;
+          v = 0.0;
+#pragma unroll
+          for (int b = 0; b < 7; ++b) v = fma(w[b], T1[(cz * 7 + b) * 13 + ix], v);
+        } else {
+          v = T1[(cz * 7 + (ty >> 1)) * 13 + ix];
+        }
+        T2[(cz * 13 + iy) * 13 + ix] = v;
+      }
+      __syncthreads();
+      for (int idx = tid; idx < nz * ny * nx; idx += UZ_THREADS) {
+        const int ix = idx % nx, iy = (idx / nx) % ny, iz = idx / (nx * ny);
+        const int p = (lx + ix) + 13 * (ly + iy) + 169 * (lz + iz);
+        if (pm[p] != j) continue;
+        const int tz = t.o[2] + lz + iz;
+        double v;
+        if (tz & 1) {
+          const double* w = W + tz * 7;
+          v = 0.0;
+#pragma unroll
+          for (int c = 0; c < 7; ++c) v = fma(w[c], T2[(c * 13 + iy) * 13 + ix], v);
+        } else {
+          v = T2[((tz >> 1) * 13 + iy) * 13 + ix];
+        }
+        P[p] = v;
+      }
     }
     if (any_out) {
       // Phase B (reading R12): degree-6 extrapolation along x, then y, then z,
@@ -246,9 +324,10 @@ __global__ void k_dof_coords(const int64_t* __restrict__ node, int64_t n, int64_
                              double unit) {
   for (int64_t d = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; d < n;
        d += int64_t(gridDim.x) * blockDim.x) {
-    xyz[d] = x0 + double(node[3 * d + 0]) * unit;
-    xyz[stride + d] = y0 + double(node[3 * d + 1]) * unit;
-    xyz[2 * stride + d] = z0 + double(node[3 * d + 2]) * unit;
+    // explicit rounding (no FMA contraction): xmin + X * unit, as on the host
+    xyz[d] = __dadd_rn(x0, __dmul_rn(double(node[3 * d + 0]), unit));
+    xyz[stride + d] = __dadd_rn(y0, __dmul_rn(double(node[3 * d + 1]), unit));
+    xyz[2 * stride + d] = __dadd_rn(z0, __dmul_rn(double(node[3 * d + 2]), unit));
   }
 }
 
@@ -257,7 +336,7 @@ void launch_dof_coords(const DevMesh& m, const int64_t* dof_node, double* xyz,
   const int64_t n = m.dof_stride;
   int blocks = int((n + 255) / 256);
   if (blocks > 148 * 8) blocks = 148 * 8;
-  const double unit = m.width / (6.0 * double(int64_t(1) << m.D));
+  const double unit = m.width / double(6 * (int64_t(1) << m.D));
   k_dof_coords<<<blocks, 256, 0, s>>>(dof_node, n, m.dof_stride, xyz, xmin[0], xmin[1], xmin[2],
                                       unit);
 }
@@ -294,6 +373,26 @@ void launch_scatter_unpack(double* u, int64_t stride, int64_t offset, const doub
   int blocks = int((n_total + 255) / 256);
   if (blocks > 148 * 4) blocks = 148 * 4;
   k_unpack<<<dim3(blocks, NF), 256, 0, s>>>(u, stride, offset, buf, n_total);
+}
+
+// ------------------------------------------------------ fp64 microbenchmark
+__global__ void __launch_bounds__(256) k_dfma(int iters, double* out) {
+  double a[8];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) a[k] = 1.0 + 1e-3 * (threadIdx.x + k);
+  const double b = 0.9999999, c = 1e-7;
+  for (int i = 0; i < iters; ++i) {
+#pragma unroll
+    for (int k = 0; k < 8; ++k) a[k] = fma(a[k], b, c);
+  }
+  double sum = 0.0;
+#pragma unroll
+  for (int k = 0; k < 8; ++k) sum += a[k];
+  if (sum == 1234.5678) out[0] = sum;   // keeps the chains alive
+}
+
+void launch_dfma(int blocks, int iters, double* out, cudaStream_t s) {
+  k_dfma<<<blocks, 256, 0, s>>>(iters, out);
 }
 
 }  // namespace dgr

@@ -70,7 +70,26 @@ def test_unzip_parity(case):
     cp = (k == 0) | (k == 1) | (k == 2)
     hang_free_copy = cp & np.isin(src, np.nonzero(om.is_dof.all(axis=1))[0])
     assert np.array_equal(P[:, hang_free_copy], Po[:, hang_free_copy])
-    assert_parity(P, Po, TOL, f"unzip {name}")
+    ext = k == 4
+    assert_parity(P[:, ~ext], Po[:, ~ext], TOL, f"unzip {name}")
+    if ext.any():
+        # Extrapolated points (reading R12) are ill-conditioned by construction:
+        # each pass along an outside axis multiplies input rounding by
+        # sum|w_t| = 127, 769, 2815 for t = 1, 2, 3 (tests/golden/stencils.txt),
+        # so the derived bound is 8 eps * prod_axes sum|w| * max|f|.
+        S = {0: 1.0, 1: 127.0, 2: 769.0, 3: 2815.0}
+        ijk = np.stack(np.unravel_index(np.arange(2197), (13, 13, 13))[::-1], 1)
+        amp = np.ones((om.n_oct, 2197))
+        for ax in range(3):
+            i = ijk[:, ax]
+            t = np.where(i < 3, 3 - i, np.where(i > 9, i - 9, 0))
+            X = 6 * om.anchors[:, ax][:, None] + (i[None] - 3) * om.side[:, None]
+            outside = (X < 0) | (X > om.L)
+            amp *= np.where(outside, np.vectorize(S.get)(t)[None], 1.0)
+        scale = np.max(np.abs(Po), axis=(1, 2))[:, None, None]
+        bound = 8 * np.finfo(float).eps * amp[None] * scale
+        diff = np.abs(P - Po)
+        assert np.all(diff[:, ext] <= bound[:, ext]), float(np.max(diff / bound))
 
 
 def test_rhs_patches_parity(case):
@@ -123,9 +142,16 @@ def test_constraints_parity(case):
     c, norms = m.constraints(ud)
     c = c[:, :om.n_dof].cpu().numpy()
     co = ocon.constraints_dofs(om, u, obssn.Params())
-    assert_parity(c, co, 1e-9, f"constraints {name}")
+    # H, M, G are sums of curvature-sized terms that cancel to truncation size
+    # on (near-)solutions (gauge wave: |H| ~ 1e-8); errors are measured against
+    # the size of those terms, taken as the largest |RHS| of the same data.
+    term = np.max(np.abs(ork4.rhs_dofs(om, u, obssn.Params())))
+    scale = np.maximum(np.max(np.abs(co), axis=1), term)
+    err = np.max(np.abs(c - co), axis=1) / scale
+    assert np.all(err <= 1e-10), err
     no = ocon.norms(co)
-    assert np.allclose(norms, no, rtol=1e-9, atol=1e-300)
+    sc = np.stack([scale, scale], 1)
+    assert np.all(np.abs(norms - no) <= 1e-10 * sc), (norms, no)
 
 
 def test_minkowski_rhs_exactly_zero():

@@ -279,6 +279,7 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
   double w13[91], wext[21];
   lagrange_tables(w13, wext);
   upload_tables(w13, wext);
+  upload_rhs_tables();
   CUDA_TRY(cudaGetLastError());
   DevMesh& dm = m->dm;
   dm.n_owned = int32_t(no);

@@ -52,6 +52,7 @@ struct RhsParams {
 void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const RhsParams& p,
                 cudaStream_t s);
 size_t rhs_smem_bytes();
+void upload_rhs_tables();
 
 // constraints_kernel.cu
 void launch_constraints(const DevMesh& m, const double* patches, double* c_oct,

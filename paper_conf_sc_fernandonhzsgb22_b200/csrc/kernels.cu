@@ -107,6 +107,7 @@ void launch_hanging(const DevMesh& m, const int4* rows, int64_t count, double* E
 // extrapolation (reading R12).  The finished 13^3 patch leaves shared memory
 // with coalesced stores.
 constexpr int UZ_THREADS = 256;
+constexpr int UZ_FCHUNK = 4;   // fields per CTA: a wave of CTAs works on the same 4 fields (L2 reuse of E)
 
 __global__ void __launch_bounds__(UZ_THREADS) k_unzip(DevMesh m, const double* __restrict__ E,
                                                       double* __restrict__ patches, int nf) {
@@ -144,20 +145,38 @@ __global__ void __launch_bounds__(UZ_THREADS) k_unzip(DevMesh m, const double* _
   __syncthreads();
   const int nc = n_coarse;
   const int64_t nn = int64_t(m.n_local) * NPT;
-  for (int f = 0; f < nf; ++f) {
+  const int f0 = blockIdx.y * UZ_FCHUNK, f1 = min(nf, f0 + UZ_FCHUNK);
+  for (int f = f0; f < f1; ++f) {
     const double* Ef = E + f * nn;
-    // ---- phase A.1: self / same level / finer: one load per point
-    for (int p = tid; p < NPATCH; p += UZ_THREADS) {
-      const int j = pm[p];
-      const int ix = p % 13, iy = (p / 13) % 13, iz = p / 169;
-      if (j == PM_SELF) {
-        P[p] = __ldg(Ef + int64_t(e) * NPT + (ix - 3) + 7 * (iy - 3) + 49 * (iz - 3));
-      } else if (j != PM_EXTRAP && nb[j].r != 1) {
-        const NbrEntry& t = nb[j];
-        const int tx = (t.o[0] + t.r * ix) >> 1, ty = (t.o[1] + t.r * iy) >> 1,
-                  tz = (t.o[2] + t.r * iz) >> 1;
-        P[p] = __ldg(Ef + int64_t(t.src) * NPT + tx + 7 * ty + 49 * tz);
+    // ---- phase A.1: self / same level / finer: one load per point.  All of a
+    // thread's source addresses are formed first so its ~9 loads are in flight
+    // together (the kernel is load-latency bound otherwise).
+    {
+      constexpr int PER = (NPATCH + UZ_THREADS - 1) / UZ_THREADS;
+      int64_t addr[PER];
+#pragma unroll
+      for (int q = 0; q < PER; ++q) {
+        const int p = tid + q * UZ_THREADS;
+        addr[q] = -1;
+        if (p < NPATCH) {
+          const int j = pm[p];
+          const int ix = p % 13, iy = (p / 13) % 13, iz = p / 169;
+          if (j == PM_SELF) {
+            addr[q] = int64_t(e) * NPT + (ix - 3) + 7 * (iy - 3) + 49 * (iz - 3);
+          } else if (j != PM_EXTRAP && nb[j].r != 1) {
+            const NbrEntry& t = nb[j];
+            const int tx = (t.o[0] + t.r * ix) >> 1, ty = (t.o[1] + t.r * iy) >> 1,
+                      tz = (t.o[2] + t.r * iz) >> 1;
+            addr[q] = int64_t(t.src) * NPT + tx + 7 * ty + 49 * tz;
+          }
+        }
       }
+      double v[PER];
+#pragma unroll
+      for (int q = 0; q < PER; ++q) v[q] = addr[q] >= 0 ? __ldg(Ef + addr[q]) : 0.0;
+#pragma unroll
+      for (int q = 0; q < PER; ++q)
+        if (addr[q] >= 0) P[tid + q * UZ_THREADS] = v[q];
     }
     // ---- phase A.2: coarser neighbours, separable sweeps x -> y -> z
     for (int ci = 0; ci < nc; ++ci) {
@@ -247,14 +266,14 @@ __global__ void __launch_bounds__(UZ_THREADS) k_unzip(DevMesh m, const double* _
     }
     __syncthreads();
     double* dst = patches + (int64_t(f) * m.n_owned + e) * PATCH_PITCH;
-    for (int p = tid; p < NPATCH; p += UZ_THREADS) dst[p] = P[p];
+    for (int p = tid; p < NPATCH; p += UZ_THREADS) __stcs(dst + p, P[p]);   // streaming: keep E in L2
     __syncthreads();
   }
 }
 
 void launch_unzip(const DevMesh& m, const double* E, double* patches, int nf, cudaStream_t s) {
   if (m.n_owned <= 0) return;
-  k_unzip<<<m.n_owned, UZ_THREADS, 0, s>>>(m, E, patches, nf);
+  k_unzip<<<dim3(m.n_owned, (nf + UZ_FCHUNK - 1) / UZ_FCHUNK), UZ_THREADS, 0, s>>>(m, E, patches, nf);
 }
 
 // -------------------------------------------------------------------- zip

@@ -21,6 +21,8 @@
 // first-kind symbol C_ijk itself (gt_il gt^lm C_mjk = C_ijk).
 #include <cuda_runtime.h>
 
+#include <vector>
+
 #include "device.cuh"
 
 namespace dgr {
@@ -28,7 +30,7 @@ namespace dgr {
 namespace {
 
 constexpr int RT = 352;   // threads (11 warps); 343 interior points
-constexpr int NPP = 344;  // slot stride in doubles
+constexpr int NPP = RT;   // slot stride in doubles: slots are indexed by thread
 
 // shared-memory slot map ([slot][NPP] doubles)
 constexpr int V_GT = 0, V_B = 3, V_GAM = 6, V_AT = 12;                         // values (18)
@@ -37,6 +39,12 @@ constexpr int G_INV = 39;                                                      /
 constexpr int S0 = 45;                                                         // scratch (24)
 constexpr int NSLOT = 69;
 constexpr size_t SMEM_BYTES = size_t(NSLOT) * NPP * 8 + size_t(2) * STAGE_DBL * 8 + 16;
+
+// thread -> interior point map (filled by upload_rhs_tables): every warp holds
+// at most two points per residue of their stage-buffer index mod 16, so its
+// 8-byte stencil loads hit each of the 16 bank pairs at most twice (2
+// wavefronts, conflict-free); shifted stencil taps only rotate the residues.
+__constant__ int16_t c_perm[RT];
 
 // field processing order
 __constant__ int c_order[NF] = {12, 13, 14, 15, 16, 17, 1, 0, 3, 4, 5, 6,
@@ -157,14 +165,15 @@ __global__ void __launch_bounds__(RT, 1)
 
   const int e = blockIdx.x;
   const int tid = threadIdx.x;
-  const bool active = tid < NPT;
-  const int p = active ? tid : 0;
+  const int pp = c_perm[tid];
+  const bool active = pp >= 0;
+  const int p = active ? pp : 0;
   const int pi = p % 7, pj = (p / 7) % 7, pk = p / 49;
   const int c0 = (pi + 3) + 13 * (pj + 3) + 169 * (pk + 3);
   const int64_t no = m.n_owned;
   const double* pbase = patches + int64_t(e) * PATCH_PITCH;
   const int64_t fstride = no * PATCH_PITCH;
-#define SL(slot) slots[(slot) * NPP + p]
+#define SL(slot) slots[(slot) * NPP + tid]
 
   if (tid == 0) {
     mbar_init(&bars[0], 1);
@@ -544,6 +553,23 @@ __global__ void __launch_bounds__(RT, 1)
 }
 
 size_t rhs_smem_bytes() { return SMEM_BYTES; }
+
+void upload_rhs_tables() {
+  int16_t perm[RT];
+  std::vector<int> bucket[16];
+  for (int p = 0; p < NPT; ++p) {
+    const int c = (p % 7 + 3) + 13 * ((p / 7) % 7 + 3) + 169 * (p / 49 + 3);
+    bucket[c % 16].push_back(p);
+  }
+  size_t next[16] = {0};
+  for (int t = 0; t < RT; ++t) perm[t] = -1;
+  for (int w = 0; w < RT / 32; ++w)
+    for (int lane = 0; lane < 32; ++lane) {
+      const int r = lane % 16;
+      if (next[r] < bucket[r].size()) perm[w * 32 + lane] = int16_t(bucket[r][next[r]++]);
+    }
+  cudaMemcpyToSymbol(c_perm, perm, sizeof(perm));
+}
 
 void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const RhsParams& p,
                 cudaStream_t s) {

@@ -97,7 +97,10 @@ typedef struct {
   int32_t device;         /* 1: upload maps + allocate workspace on the current
                              CUDA device; 0: host-only (maps/export only)  */
   int32_t pad;
-  const void* nccl_id;    /* ncclUniqueId bytes (128) when nranks > 1      */
+  const void* nccl_id;    /* ncclUniqueId bytes (128) when nranks > 1; NULL with
+                             nranks > 1 selects external-exchange mode: no
+                             communicator, the caller refreshes the ghost DOFs
+                             itself (DGR_MAP_SEND / _COUNTS) before each stage */
 } dgr_mesh_desc;
 
 /* Parameters of the RHS (readings R6, R8, R13). */
@@ -142,7 +145,9 @@ enum {
   DGR_MAP_DOF_XYZ = 7,  /* double [3][n_dof_owned + n_dof_ghost]: coordinates      */
   DGR_MAP_SEND = 8,     /* int32 [sum over peers]: local DOF ids sent, peer-major   */
   DGR_MAP_SEND_COUNTS = 9, /* int64 [nranks]: DOFs sent to each peer               */
-  DGR_MAP_RECV_COUNTS = 10 /* int64 [nranks]: ghost DOFs received from each peer   */
+  DGR_MAP_RECV_COUNTS = 10, /* int64 [nranks]: ghost DOFs received from each peer  */
+  DGR_MAP_LOCAL_OCTS = 11,  /* int32 [n_oct_local + n_oct_ghost]: global octant ids */
+  DGR_MAP_O2N_LOCAL = 12    /* int32 [n_oct_local + n_oct_ghost][343]: local DOF id or -1 */
 };
 
 const char* dgr_status_string(dgr_status s);

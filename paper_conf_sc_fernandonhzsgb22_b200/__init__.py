@@ -26,6 +26,7 @@ NPATCH = 2197
 
 MAP_OCTANTS, MAP_O2N, MAP_HANGING, MAP_PAD_SRC, MAP_PAD_KIND, MAP_ZIP = 0, 1, 2, 3, 4, 5
 MAP_DOF_GID, MAP_DOF_XYZ, MAP_SEND, MAP_SEND_COUNTS, MAP_RECV_COUNTS = 6, 7, 8, 9, 10
+MAP_LOCAL_OCTS, MAP_O2N_LOCAL = 11, 12
 
 
 class DgrError(RuntimeError):

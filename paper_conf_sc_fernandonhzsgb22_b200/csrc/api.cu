@@ -332,8 +332,8 @@ dgr_status dgr_mesh_create(const dgr_mesh_desc* desc, const dgr_octant* octs, in
   if (m->device) {
     dgr_status s = upload(m.get(), static_cast<cudaStream_t>(stream));
     if (s != DGR_OK) return s;
-    if (desc->nranks > 1) {
-      if (!desc->nccl_id) return fail(DGR_ERR_ARG, "nccl_id required for nranks > 1");
+    if (desc->nranks > 1 && desc->nccl_id) {
+      // (nccl_id == NULL: external-exchange mode, the caller refreshes ghosts)
       if (!load_nccl()) return fail(DGR_ERR_NCCL, "libnccl.so.2 not loadable");
       UniqueId uid;
       std::memcpy(uid.internal, desc->nccl_id, 128);
@@ -436,6 +436,10 @@ dgr_status dgr_mesh_export_maps(dgr_mesh m, int which, void* host_buf, size_t* n
       return put(h.send_counts.data(), h.send_counts.size() * 8);
     case DGR_MAP_RECV_COUNTS:
       return put(h.recv_counts.data(), h.recv_counts.size() * 8);
+    case DGR_MAP_LOCAL_OCTS:
+      return put(h.local_oct.data(), h.local_oct.size() * 4);
+    case DGR_MAP_O2N_LOCAL:
+      return put(h.o2n_local.data(), h.o2n_local.size() * 4);
   }
   return fail(DGR_ERR_ARG, "unknown map id");
 }
@@ -478,7 +482,7 @@ static bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 
 // ghost exchange: pack owned DOFs each peer needs, grouped send/recv, unpack
 static dgr_status exchange(dgr_mesh m, double* u, cudaStream_t st) {
   const HostMesh& h = m->host;
-  if (h.nranks <= 1) return DGR_OK;
+  if (h.nranks <= 1 || !m->comm) return DGR_OK;   // single rank / external exchange
   const int64_t stride = m->dm.dof_stride;
   const int64_t nsend = int64_t(h.send_list.size());
   PROF(m, 5, st, launch_gather_pack(u, stride, m->d_send, nsend, m->d_sendbuf, st));
@@ -531,6 +535,8 @@ dgr_status dgr_dof_coords(dgr_mesh m, double* xyz, void* stream) {
 dgr_status dgr_ghost_exchange(dgr_mesh m, double* u, void* stream) {
   dgr_status s = need_device(m);
   if (s) return s;
+  if (m->host.nranks > 1 && !m->comm)
+    return fail(DGR_ERR_STATE, "external-exchange mesh (created without nccl_id)");
   return exchange(m, u, static_cast<cudaStream_t>(stream));
 }
 
@@ -638,7 +644,7 @@ dgr_status dgr_constraints(dgr_mesh m, double* u, double* c, double* norms_host,
       part[2 * q + 1] = mx;
     }
     double ntot = double(n);
-    if (m->host.nranks > 1) {
+    if (m->host.nranks > 1 && m->comm) {   // (external-exchange mode: rank-local norms)
       double* d = m->d_cnorm;
       double sums[8], maxs[7];
       for (int q = 0; q < 7; ++q) {

@@ -1,0 +1,86 @@
+"""Multi-rank CUDA path on ONE GPU (SURVEY §4 invariant 1, §8e).
+
+Only one B200 is available to this build, so the partitioned path is checked
+by running R rank-meshes of the same octree side by side in one process in
+external-exchange mode (dgr_mesh_desc.nccl_id = NULL): between stages the test
+moves each rank's owned DOFs to the peers' ghost slices using the library's
+own send lists / receive counts (the same [peer][field][dof] blocks the NCCL
+path sends).  After RK4 steps every rank's owned DOFs must be BIT-IDENTICAL to
+the single-rank run: all kernels are per-octant deterministic and ghosts are
+exact copies.
+"""
+import numpy as np
+import pytest
+
+import paper_conf_sc_fernandonhzsgb22_b200 as dgr
+from oracle import rk4 as ork4
+from oracle.maps import OracleMesh
+from synth import configs, initial
+
+from .gpu_util import need_gpu, to_dev, torch
+
+pytestmark = pytest.mark.gpu
+NF = 24
+
+
+def _exchange(meshes, states, lists):
+    """Ghost refresh for all ranks (device copies following libdgr's lists)."""
+    world = len(meshes)
+    for r in range(world):
+        send, scount, _, _ = lists[r]
+        off = 0
+        for peer in range(world):
+            n = int(scount[peer])
+            if n == 0:
+                continue
+            ids = send[off:off + n]
+            off += n
+            # where these land on the peer: its ghost block from rank r
+            _, _, rcount_p, no_p = lists[peer]
+            goff = no_p + int(rcount_p[:r].sum())
+            states[peer][:, goff:goff + n] = states[r][:, ids]
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_multirank_bit_identical(world):
+    need_gpu()
+    cfg = configs.small_bbh(lmax=6, rho=0.5)
+    om = OracleMesh(cfg)
+    om.build_dofs()
+    u = initial.for_config(cfg, om.dof_coords())
+    dt = ork4.dt_courant(om)
+    ref = dgr.Mesh(cfg)
+    ur = to_dev(u, ref.dof_stride)
+    meshes, states, lists, gids = [], [], [], []
+    for r in range(world):
+        m = dgr.Mesh(cfg, rank=r, nranks=world)
+        gid = m.export(dgr.MAP_DOF_GID, np.int64)
+        st = torch.zeros((NF, m.dof_stride), dtype=torch.float64, device="cuda")
+        st[:, :len(gid)] = torch.from_numpy(u[:, gid])
+        send = torch.from_numpy(m.export(dgr.MAP_SEND, np.int32).astype(np.int64)).cuda()
+        lists.append((send, m.export(dgr.MAP_SEND_COUNTS, np.int64),
+                      m.export(dgr.MAP_RECV_COUNTS, np.int64), m.info["n_dof_owned"]))
+        meshes.append(m)
+        states.append(st)
+        gids.append(gid)
+        assert m.info["n_oct_ghost"] > 0
+    us = [torch.zeros_like(s) for s in states]
+    acc = [torch.zeros_like(s) for s in states]
+    for step in range(2):
+        ref.rk4_step(ur, dt)
+        for s in range(4):
+            cur = states if s == 0 else us
+            if s == 0:
+                for r in range(world):
+                    us[r].copy_(states[r])
+            _exchange(meshes, cur, lists)
+            for r in range(world):
+                meshes[r].rk4_stage(s, dt, states[r], us[r], acc[r])
+        for r in range(world):
+            states[r].copy_(acc[r])
+    torch.cuda.synchronize()
+    full = ur[:, :om.n_dof].cpu().numpy()
+    for r in range(world):
+        no = meshes[r].info["n_dof_owned"]
+        got = states[r][:, :no].cpu().numpy()
+        assert np.array_equal(got, full[:, gids[r][:no]]), f"rank {r} differs"

@@ -101,38 +101,46 @@ class Clocks:
                 "samples": len(self.samples)}
 
 
-def cpu_baseline_oracle(cfg, n_sample, reps=1):
-    """The oracle as it stands, on the host cores, bounded sample of the
-    workload: element reconstruction for ALL octants + octant-to-patch and
-    RHS for `n_sample` random octants; one RK4 step = 4 such stages over all
-    octants, extrapolated linearly in the octant count."""
-    from threadpoolctl import threadpool_limits
+def cpu_baseline_oracle(cfg, n_sample=None, reps=1):
+    """The oracle as it stands, on the host cores, on a bounded sample of the
+    workload: element reconstruction (hanging points) for ALL octants, then
+    octant-to-patch + RHS for a contiguous Morton range of octants spread over
+    all cores (forked workers, 1 BLAS thread each, the oracle's own
+    rk4._chunk_rhs); one RK4 step = 4 such stages over all octants,
+    extrapolated linearly in the octant count."""
+    import multiprocessing as mp
 
-    from oracle import bssn, rk4, unzip
+    from oracle import bssn
+    from oracle import rk4 as ork4
+    from oracle import unzip as ouz
     from oracle.maps import OracleMesh
     from synth import initial
+    cores = len(os.sched_getaffinity(0))
     om = OracleMesh(cfg)
     om.build_dofs()
     u = initial.for_config(cfg, om.dof_coords())
-    octs = np.random.default_rng(0).choice(om.n_oct, min(n_sample, om.n_oct), replace=False)
-    h = rk4.octant_h(om)
-    om.padding_sources(octs[:2])          # warm imports / caches outside the timing
+    ouz.padding_sources_cached(om, np.arange(1))           # maps: built once, not timed
+    n_s = min(om.n_oct, n_sample or 24 * cores)
+    start = int(np.random.default_rng(0).integers(0, om.n_oct - n_s + 1))
+    bounds = np.linspace(start, start + n_s, 4 * cores + 1).astype(int)
+    chunks = [(int(x), int(y)) for x, y in zip(bounds[:-1], bounds[1:]) if y > x]
     times = []
-    with threadpool_limits(limits=1):
-        for _ in range(reps):
-            t0 = time.perf_counter()
-            unzip.elements(om, u)
-            t1 = time.perf_counter()
-            P = unzip.unzip(om, u, octs)
-            bssn.rhs_patches(P, h[octs], bssn.Params())
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        E = ouz.elements(om, u)
+        t1 = time.perf_counter()
+        ork4._G.update(mesh=om, E=E, prm=bssn.Params())
+        with mp.get_context("fork").Pool(cores) as pool:   # workers inherit _G by fork
             t2 = time.perf_counter()
-            # unzip() recomputed the elements: subtract that copy
-            stage = (t1 - t0) + (t2 - t1 - (t1 - t0)) * om.n_oct / len(octs)
-            times.append(4.0 * stage)
+            pool.map(ork4._chunk_rhs, chunks)
+            t3 = time.perf_counter()
+        ork4._G.clear()
+        times.append(4.0 * ((t1 - t0) + (t3 - t2) * om.n_oct / n_s))
     step_s = float(np.median(times))
-    return {"value": om.n_dof / step_s, "unit": UNIT, "cores": 1, "kind": "oracle",
-            "sample": (f"1 RK4 step = 4 x (elements for all {om.n_oct} octants + unzip+RHS of "
-                       f"{len(octs)} random octants scaled to {om.n_oct}); NumPy, 1 thread"),
+    return {"value": om.n_dof / step_s, "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": (f"1 RK4 step = 4 x (hanging reconstruction for all {om.n_oct} octants + "
+                       f"unzip+RHS of {n_s} Morton-contiguous octants on {cores} worker "
+                       f"processes, scaled to {om.n_oct})"),
             "step_s": step_s}
 
 
@@ -140,7 +148,7 @@ def run_reference(args, cfg):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    cb = cpu_baseline_oracle(cfg, n_sample=64, reps=args.warmup + args.steps)
+    cb = cpu_baseline_oracle(cfg, reps=args.warmup + args.steps)
     line = {"impl": "reference", "metric": METRIC, "value": cb["value"], "unit": UNIT,
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": cb["step_s"] * 1e3, "higher_is_better": True, "scaling": "strong",
@@ -160,7 +168,7 @@ def main():
     ap.add_argument("--config", default="c3")
     ap.add_argument("--impl", default="dgr", choices=["dgr", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--cpu-sample", type=int, default=128)
+    ap.add_argument("--cpu-sample", type=int, default=None)
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 

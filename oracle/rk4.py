@@ -11,11 +11,14 @@ by every unzip.
 """
 from __future__ import annotations
 
+import multiprocessing as mp
+import os
+
 import numpy as np
 
 from .bssn import NF, Params, rhs_patches
 from .maps import OracleMesh
-from .unzip import unzip, zip_rhs
+from .unzip import elements, padding_sources_cached, unzip, unzip_from_elements, zip_rhs
 
 COURANT = 0.25
 
@@ -24,11 +27,46 @@ def octant_h(mesh: OracleMesh):
     return mesh.cfg.width / (6.0 * (2.0 ** mesh.levels))
 
 
-def rhs_dofs(mesh: OracleMesh, u: np.ndarray, prm: Params) -> np.ndarray:
-    """F(u): [24, n_dof] -> [24, n_dof]."""
-    P = unzip(mesh, u)
-    r = rhs_patches(P, octant_h(mesh), prm)
-    return zip_rhs(mesh, r.reshape(NF, mesh.n_oct, 343))
+def rhs_dofs(mesh: OracleMesh, u: np.ndarray, prm: Params, workers=None) -> np.ndarray:
+    """F(u): [24, n_dof] -> [24, n_dof].
+
+    workers > 1 evaluates octant-to-patch + RHS on chunks of octants in forked
+    worker processes (the element reconstruction, which couples octants, is
+    done once in the parent); the arithmetic per octant is unchanged.
+    Default: $DGR_ORACLE_WORKERS, else 1."""
+    if workers is None:
+        workers = int(os.environ.get("DGR_ORACLE_WORKERS", "1"))
+    if workers <= 1 or mesh.n_oct < 4 * workers:
+        P = unzip(mesh, u)
+        r = rhs_patches(P, octant_h(mesh), prm)
+        return zip_rhs(mesh, r.reshape(NF, mesh.n_oct, 343))
+    E = elements(mesh, u)
+    padding_sources_cached(mesh, np.arange(1))          # fill the cache before forking
+    _G.update(mesh=mesh, E=E, prm=prm)
+    nch = 4 * workers
+    bounds = np.linspace(0, mesh.n_oct, nch + 1).astype(int)
+    chunks = [(int(a), int(b)) for a, b in zip(bounds[:-1], bounds[1:]) if b > a]
+    with mp.get_context("fork").Pool(workers) as pool:
+        parts = pool.map(_chunk_rhs, chunks)
+    _G.clear()
+    r = np.empty((NF, mesh.n_oct, 343))
+    for a, rr in parts:
+        r[:, a:a + rr.shape[1]] = rr
+    return zip_rhs(mesh, r)
+
+
+_G = {}
+
+
+def _chunk_rhs(ab):
+    from threadpoolctl import threadpool_limits
+    a, b = ab
+    mesh, E, prm = _G["mesh"], _G["E"], _G["prm"]
+    octs = np.arange(a, b)
+    with threadpool_limits(limits=1):
+        P = unzip_from_elements(mesh, E, octs)
+        r = rhs_patches(P, octant_h(mesh)[octs], prm)
+    return a, r.reshape(NF, len(octs), 343)
 
 
 def rk4_step(mesh: OracleMesh, u: np.ndarray, dt: float, prm: Params) -> np.ndarray:

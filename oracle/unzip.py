@@ -120,17 +120,26 @@ def elements(mesh: OracleMesh, u: np.ndarray, chunk=20000) -> np.ndarray:
 
 def unzip(mesh: OracleMesh, u: np.ndarray, octs=None, chunk=4000) -> np.ndarray:
     """Patches [nf, n, 13, 13, 13] (index [z][y][x]) of octants `octs` (default all)."""
-    E = elements(mesh, u)
+    return unzip_from_elements(mesh, elements(mesh, u), octs, chunk)
+
+
+def padding_sources_cached(mesh: OracleMesh, octs):
+    """mesh.padding_sources(octs), memoised for the whole mesh (the maps do not depend on u)."""
+    if getattr(mesh, "_pad_cache", None) is None:
+        mesh._pad_cache = mesh.padding_sources()
+    src, kind = mesh._pad_cache
+    return src[octs], kind[octs]
+
+
+def unzip_from_elements(mesh: OracleMesh, E: np.ndarray, octs=None, chunk=4000) -> np.ndarray:
+    """Octant-to-patch given the reconstructed element values E [nf, n_oct, 343]."""
     full = octs is None
     octs = np.arange(mesh.n_oct) if octs is None else np.asarray(octs, dtype=np.int64)
-    nf = u.shape[0]
-    # the maps do not depend on u: memoise them for the whole mesh
-    if full and getattr(mesh, "_pad_cache", None) is not None:
-        src, kind = mesh._pad_cache
+    nf = E.shape[0]
+    if full or getattr(mesh, "_pad_cache", None) is not None:
+        src, kind = padding_sources_cached(mesh, octs)
     else:
         src, kind = mesh.padding_sources(octs)
-        if full:
-            mesh._pad_cache = (src, kind)
     pijk = _patch_ijk()
     out = np.empty((nf, len(octs), P13 ** 3))
     for i0 in range(0, len(octs), chunk // 8 + 1):

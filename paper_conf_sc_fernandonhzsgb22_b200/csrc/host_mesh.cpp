@@ -587,7 +587,7 @@ void HostMesh::partition() {
 // domain -> extrapolation.
 void HostMesh::build_padding() {
   const int64_t no = n_owned_oct;
-  pmap.assign(size_t(no) * NPATCH, PM_EXTRAP);
+  pmap.assign(size_t(no) * PMAP_PITCH, PM_EXTRAP);
   nbr.assign(size_t(no) * NBR_MAX, NbrEntry{0, {0, 0, 0}, 0, 0});
   n_nbr.assign(no, 0);
   pad_src_global.assign(size_t(no) * NPATCH, -1);
@@ -598,7 +598,7 @@ void HostMesh::build_padding() {
     const int64_t b = oct_begin + lb;
     const Oct& q = oct[b];
     const int64_t s = side(int32_t(b));
-    uint8_t* pm = &pmap[size_t(lb) * NPATCH];
+    uint8_t* pm = &pmap[size_t(lb) * PMAP_PITCH];
     int32_t* psrc = &pad_src_global[size_t(lb) * NPATCH];
     uint8_t* pk = &pad_kind[size_t(lb) * NPATCH];
     // outside flags per axis and patch index
@@ -706,6 +706,14 @@ void HostMesh::build_padding() {
         ne.lo[k] = uint8_t(std::min<int>(ne.lo[k], idx[k]));
         ne.hi[k] = uint8_t(std::max<int>(ne.hi[k], idx[k]));
       }
+    }
+    // a coarser source (twice the octant's size) spans at most 10 patch indices per
+    // axis; the device sweep buffers rely on it
+    for (int jn = 0; jn < nn; ++jn) {
+      const NbrEntry& ne = nbr[size_t(lb) * NBR_MAX + jn];
+      if (ne.r == 1)
+        for (int k = 0; k < 3; ++k)
+          if (ne.hi[k] - ne.lo[k] + 1 > 10) ++bad;
     }
   }
   if (bad) throw BuildError{-2, "padding map construction failed"};

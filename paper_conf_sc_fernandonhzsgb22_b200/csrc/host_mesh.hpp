@@ -24,6 +24,7 @@ constexpr int NPT = 343;     // 7^3
 constexpr int NPATCH = 2197; // 13^3
 constexpr int NBR_MAX = 64;  // max touching (leaf, shift) entries per octant
 constexpr uint8_t PM_SELF = 254, PM_EXTRAP = 255;
+constexpr int PMAP_PITCH = 2208;  // bytes per octant in the device padding map (16-B rows)
 
 struct Oct {
   int64_t a[3];
@@ -92,7 +93,7 @@ class HostMesh {
   // per local octant (owned + ghost) maps in local numbering
   std::vector<int32_t> o2n_local;              // [n_local * 343] local DOF or -1
   // per owned octant padding tables
-  std::vector<uint8_t> pmap;                   // [n_owned * 2197]
+  std::vector<uint8_t> pmap;                   // [n_owned * PMAP_PITCH]
   std::vector<NbrEntry> nbr;                   // [n_owned * NBR_MAX]
   std::vector<int32_t> n_nbr;                  // [n_owned]
   std::vector<int32_t> pad_src_global;         // [n_owned * 2197] export

@@ -19,9 +19,12 @@ namespace dgr {
 __constant__ double c_W13[13 * 7];
 __constant__ double c_WEXT[3 * 7];
 
+void upload_unzip_tables(const double* w13, const double* wext);  // unzip_kernel.cu
+
 void upload_tables(const double* w13, const double* wext) {
   cudaMemcpyToSymbol(c_W13, w13, sizeof(double) * 91);
   cudaMemcpyToSymbol(c_WEXT, wext, sizeof(double) * 21);
+  upload_unzip_tables(w13, wext);
 }
 
 // I_c(t2) = sum_{ijk} W[t2x][i] W[t2y][j] W[t2z][k] E_c[i + 7j + 49k]; along an
@@ -97,184 +100,7 @@ void launch_hanging(const DevMesh& m, const int4* rows, int64_t count, double* E
   k_hanging<<<dim3(blocks, nf), 128, 0, s>>>(rows, count, E, int64_t(m.n_local) * NPT);
 }
 
-// ------------------------------------------------------------------ unzip
-// One CTA per patch, fields in sequence.  Phase A: points sourced from the
-// octant itself, a same-level or a finer neighbour are single loads (their
-// half-grid coordinates are even); points sourced from a coarser neighbour c
-// are produced by three 1D Lagrange sweeps over c's 7^3 nodes staged in shared
-// memory, restricted to the bounding box of the points c sources (the
-// tensor-product interpolation of P:L295).  Phase B: outer-boundary
-// extrapolation (reading R12).  The finished 13^3 patch leaves shared memory
-// with coalesced stores.
-constexpr int UZ_THREADS = 256;
-constexpr int UZ_FCHUNK = 4;   // fields per CTA: a wave of CTAs works on the same 4 fields (L2 reuse of E)
-
-__global__ void __launch_bounds__(UZ_THREADS) k_unzip(DevMesh m, const double* __restrict__ E,
-                                                      double* __restrict__ patches, int nf) {
-  __shared__ __align__(16) double P[NPATCH + 3];
-  __shared__ double Es[NPT + 1];
-  __shared__ double T1[7 * 7 * 13];
-  __shared__ double T2[7 * 13 * 13];
-  __shared__ uint8_t pm[NPATCH + 11];
-  __shared__ NbrEntry nb[NBR_MAX];
-  __shared__ double W[91];
-  __shared__ double WX[21];
-  __shared__ int coarse[8];
-  __shared__ int n_coarse;
-  const int e = blockIdx.x;
-  const int tid = threadIdx.x;
-  for (int i = tid; i < NPATCH; i += UZ_THREADS) pm[i] = m.pmap[int64_t(e) * NPATCH + i];
-  for (int i = tid; i < NBR_MAX; i += UZ_THREADS) nb[i] = m.nbr[int64_t(e) * NBR_MAX + i];
-  for (int i = tid; i < 91; i += UZ_THREADS) W[i] = c_W13[i];
-  for (int i = tid; i < 21; i += UZ_THREADS) WX[i] = c_WEXT[i];
-  __syncthreads();
-  if (tid == 0) {
-    int nc = 0;
-    for (int j = 0; j < NBR_MAX && nc < 8; ++j)
-      if (nb[j].r == 1) coarse[nc++] = j;
-    n_coarse = nc;
-  }
-  const int4 o = m.oct[e];
-  const int64_t nside = int64_t(1) << m.D;
-  const int64_t s = int64_t(1) << (m.D - o.w);
-  const bool out_lo[3] = {!m.periodic && o.x == 0, !m.periodic && o.y == 0,
-                          !m.periodic && o.z == 0};
-  const bool out_hi[3] = {!m.periodic && o.x + s == nside, !m.periodic && o.y + s == nside,
-                          !m.periodic && o.z + s == nside};
-  const bool any_out = out_lo[0] || out_lo[1] || out_lo[2] || out_hi[0] || out_hi[1] || out_hi[2];
-  __syncthreads();
-  const int nc = n_coarse;
-  const int64_t nn = int64_t(m.n_local) * NPT;
-  const int f0 = blockIdx.y * UZ_FCHUNK, f1 = min(nf, f0 + UZ_FCHUNK);
-  for (int f = f0; f < f1; ++f) {
-    const double* Ef = E + f * nn;
-    // ---- phase A.1: self / same level / finer: one load per point.  All of a
-    // thread's source addresses are formed first so its ~9 loads are in flight
-    // together (the kernel is load-latency bound otherwise).
-    {
-      constexpr int PER = (NPATCH + UZ_THREADS - 1) / UZ_THREADS;
-      int64_t addr[PER];
-#pragma unroll
-      for (int q = 0; q < PER; ++q) {
-        const int p = tid + q * UZ_THREADS;
-        addr[q] = -1;
-        if (p < NPATCH) {
-          const int j = pm[p];
-          const int ix = p % 13, iy = (p / 13) % 13, iz = p / 169;
-          if (j == PM_SELF) {
-            addr[q] = int64_t(e) * NPT + (ix - 3) + 7 * (iy - 3) + 49 * (iz - 3);
-          } else if (j != PM_EXTRAP && nb[j].r != 1) {
-            const NbrEntry& t = nb[j];
-            const int tx = (t.o[0] + t.r * ix) >> 1, ty = (t.o[1] + t.r * iy) >> 1,
-                      tz = (t.o[2] + t.r * iz) >> 1;
-            addr[q] = int64_t(t.src) * NPT + tx + 7 * ty + 49 * tz;
-          }
-        }
-      }
-      double v[PER];
-#pragma unroll
-      for (int q = 0; q < PER; ++q) v[q] = addr[q] >= 0 ? __ldg(Ef + addr[q]) : 0.0;
-#pragma unroll
-      for (int q = 0; q < PER; ++q)
-        if (addr[q] >= 0) P[tid + q * UZ_THREADS] = v[q];
-    }
-    // ---- phase A.2: coarser neighbours, separable sweeps x -> y -> z
-    for (int ci = 0; ci < nc; ++ci) {
-      const int j = coarse[ci];
-      const NbrEntry t = nb[j];
-      __syncthreads();   // previous users of Es / T1 / T2 are done
-      const double* Ec = Ef + int64_t(t.src) * NPT;
-      for (int i = tid; i < NPT; i += UZ_THREADS) Es[i] = __ldg(Ec + i);
-      const int lx = t.lo[0], ly = t.lo[1], lz = t.lo[2];
-      const int nx = t.hi[0] - lx + 1, ny = t.hi[1] - ly + 1, nz = t.hi[2] - lz + 1;
-      __syncthreads();
-      for (int idx = tid; idx < 49 * nx; idx += UZ_THREADS) {
-        const int cyz = idx / nx, ix = idx % nx;        // cyz = cz * 7 + cy
-        const int tx = t.o[0] + lx + ix;
-        const double* row = Es + cyz * 7;
-        double v;
-        if (tx & 1) {
-          const double* w = W + tx * 7;
-          v = 0.0;
-#pragma unroll
-          for (int a = 0; a < 7; ++a) v = fma(w[a], row[a], v);
-        } else {
-          v = row[tx >> 1];
-        }
-        T1[cyz * 13 + ix] = v;
-      }
-      __syncthreads();
-      for (int idx = tid; idx < 7 * ny * nx; idx += UZ_THREADS) {
-        const int ix = idx % nx, iy = (idx / nx) % ny, cz = idx / (nx * ny);
-        const int ty = t.o[1] + ly + iy;
-        double v;
-        if (ty & 1) {
-          const double* w = W + ty * 7;
-          v = 0.0;
-#pragma unroll
-          for (int b = 0; b < 7; ++b) v = fma(w[b], T1[(cz * 7 + b) * 13 + ix], v);
-        } else {
-          v = T1[(cz * 7 + (ty >> 1)) * 13 + ix];
-        }
-        T2[(cz * 13 + iy) * 13 + ix] = v;
-      }
-      __syncthreads();
-      for (int idx = tid; idx < nz * ny * nx; idx += UZ_THREADS) {
-        const int ix = idx % nx, iy = (idx / nx) % ny, iz = idx / (nx * ny);
-        const int p = (lx + ix) + 13 * (ly + iy) + 169 * (lz + iz);
-        if (pm[p] != j) continue;
-        const int tz = t.o[2] + lz + iz;
-        double v;
-        if (tz & 1) {
-          const double* w = W + tz * 7;
-          v = 0.0;
-#pragma unroll
-          for (int c = 0; c < 7; ++c) v = fma(w[c], T2[(c * 13 + iy) * 13 + ix], v);
-        } else {
-          v = T2[((tz >> 1) * 13 + iy) * 13 + ix];
-        }
-        P[p] = v;
-      }
-    }
-    if (any_out) {
-      // Phase B (reading R12): degree-6 extrapolation along x, then y, then z,
-      // for points outside along that axis and inside along all later axes.
-      for (int a = 0; a < 3; ++a) {
-        __syncthreads();
-        for (int p = tid; p < NPATCH; p += UZ_THREADS) {
-          const int idx[3] = {p % 13, (p / 13) % 13, p / 169};
-          const int ia = idx[a];
-          const bool outa = (ia < 3 && out_lo[a]) || (ia > 9 && out_hi[a]);
-          if (!outa) continue;
-          bool later_in = true;
-          for (int b = a + 1; b < 3; ++b)
-            if ((idx[b] < 3 && out_lo[b]) || (idx[b] > 9 && out_hi[b])) later_in = false;
-          if (!later_in) continue;
-          const int stride_a = a == 0 ? 1 : (a == 1 ? 13 : 169);
-          const int base = p - ia * stride_a;
-          double acc = 0.0;
-          if (ia < 3) {
-            const double* w = WX + (2 - ia) * 7;       // t = -(3 - ia)
-            for (int mm = 0; mm < 7; ++mm) acc = fma(w[mm], P[base + (3 + mm) * stride_a], acc);
-          } else {
-            const double* w = WX + (ia - 10) * 7;      // mirrored
-            for (int mm = 0; mm < 7; ++mm) acc = fma(w[mm], P[base + (9 - mm) * stride_a], acc);
-          }
-          P[p] = acc;
-        }
-      }
-    }
-    __syncthreads();
-    double* dst = patches + (int64_t(f) * m.n_owned + e) * PATCH_PITCH;
-    for (int p = tid; p < NPATCH; p += UZ_THREADS) __stcs(dst + p, P[p]);   // streaming: keep E in L2
-    __syncthreads();
-  }
-}
-
-void launch_unzip(const DevMesh& m, const double* E, double* patches, int nf, cudaStream_t s) {
-  if (m.n_owned <= 0) return;
-  k_unzip<<<dim3(m.n_owned, (nf + UZ_FCHUNK - 1) / UZ_FCHUNK), UZ_THREADS, 0, s>>>(m, E, patches, nf);
-}
+// (octant-to-patch: unzip_kernel.cu)
 
 // -------------------------------------------------------------------- zip
 // Patch-to-octant: each owned DOF takes its zip owner's value.

@@ -183,6 +183,13 @@ __global__ void __launch_bounds__(RT, 1)
   if (tid == 0) {
     bulk_load(stage, pbase + c_order[0] * fstride, STAGE_DBL * 8, &bars[0]);
     bulk_load(stage + STAGE_DBL, pbase + c_order[1] * fstride, STAGE_DBL * 8, &bars[1]);
+  } else if (tid < NF - 1) {
+    // pull the other 22 field patches of this octant into L2 now, so the
+    // double-buffered bulk copies later hit L2 instead of waiting on HBM
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(pbase + c_order[tid + 1] *
+                                                                            fstride),
+                 "r"(uint32_t(STAGE_DBL * 8))
+                 : "memory");
   }
 
   const int4 oi = m.oct[e];

@@ -11,3 +11,6 @@ if ROOT not in sys.path:
 def pytest_configure(config):
     config.addinivalue_line("markers", "gpu: needs a CUDA device (B200) and the built libdgr.so")
     config.addinivalue_line("markers", "slow: longer CPU test")
+
+# the oracle evaluates octant-to-patch + RHS on forked workers (bitwise the same)
+os.environ.setdefault("DGR_ORACLE_WORKERS", str(min(16, len(os.sched_getaffinity(0)))))

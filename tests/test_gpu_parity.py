@@ -7,6 +7,8 @@ seeded synthetic recipes of synth/ (DESIGN.md §Inputs).  Meshes are small
 enough for the oracle to finish in seconds yet span many patches, every
 padding kind, hanging chains and the extrapolated outer boundary.
 """
+import os
+
 import numpy as np
 import pytest
 
@@ -17,18 +19,13 @@ from oracle import rk4 as ork4
 from oracle import unzip as ouz
 from oracle.maps import OracleMesh
 from synth import configs, initial
-from synth.configs import MeshConfig, Puncture
+from synth.configs import MeshConfig
 
 from .gpu_util import assert_parity, need_gpu, to_dev, torch
 
 pytestmark = pytest.mark.gpu
 
 TOL = 1e-10
-
-
-def tiny_adaptive():
-    return MeshConfig(name="tiny", xmin=(-4.0, -4.0, -4.0), width=8.0, periodic=False,
-                      level_min=1, punctures=(Puncture(0.1, -0.2, 0.05, 1.0, 4),), rho=0.4)
 
 
 CASES = {
@@ -163,14 +160,29 @@ def test_minkowski_rhs_exactly_zero():
     assert torch.count_nonzero(r).item() == 0
 
 
-@pytest.mark.slow
-def test_100_steps_parity():
-    """RK4 state after 100 steps within 1e-8 of the oracle (adaptive BL mesh)."""
+LONG_RUNS = {
+    # stable evolutions only: a perturbation test (tools/growth.py) shows that
+    # these amplify a 1e-13 relative perturbation by < 1e6 over 100 steps, so
+    # last-bit differences between two correct implementations stay < 1e-8;
+    # under-resolved punctures near an extrapolated boundary (e.g. a 176-octant
+    # [-4,4]^3 mesh: 1e-13 -> 5e-2) are chaotic and cannot meet any such bar.
+    "u2_random": (lambda: MeshConfig(name="u2", xmin=(-0.5, -0.5, -0.5), width=1.0,
+                                     periodic=True, level_min=2), "random", False),
+    "bbh_chains_bl": (lambda: configs.small_bbh(lmax=6, rho=0.5), "bl", True),
+}
+
+
+@pytest.mark.parametrize("name", list(LONG_RUNS))
+def test_100_steps_parity(name):
+    """RK4 state after 100 steps within 1e-8 of the oracle."""
     need_gpu()
-    cfg = tiny_adaptive()
+    cfgf, kind, slow = LONG_RUNS[name]
+    if slow and not os.environ.get("DGR_SLOW_TESTS"):
+        pytest.skip("set DGR_SLOW_TESTS=1 (oracle: ~400 RHS evaluations on 428 octants)")
+    cfg = cfgf()
     om = OracleMesh(cfg)
     om.build_dofs()
-    u = initial.for_config(cfg, om.dof_coords())
+    u = initial.for_config(cfg, om.dof_coords(), kind=kind, seed=5)
     dt = ork4.dt_courant(om)
     m = dgr.Mesh(cfg)
     ud = to_dev(u, m.dof_stride)
@@ -180,4 +192,5 @@ def test_100_steps_parity():
         m.rk4_step(ud, dt)
         v = ork4.rk4_step(om, v, dt, prm)
     got = ud[:, :om.n_dof].cpu().numpy()
-    assert_parity(got, v, 1e-8, "100 steps")
+    assert np.max(np.abs(v - u)) > 1e-3            # the state really evolved
+    assert_parity(got, v, 1e-8, f"100 steps {name}")

@@ -711,9 +711,15 @@ void HostMesh::build_padding() {
     // axis; the device sweep buffers rely on it
     for (int jn = 0; jn < nn; ++jn) {
       const NbrEntry& ne = nbr[size_t(lb) * NBR_MAX + jn];
-      if (ne.r == 1)
-        for (int k = 0; k < 3; ++k)
+      if (ne.r == 1) {
+        int thin = 13;
+        for (int k = 0; k < 3; ++k) {
           if (ne.hi[k] - ne.lo[k] + 1 > 10) ++bad;
+          thin = std::min(thin, ne.hi[k] - ne.lo[k] + 1);
+        }
+        // it lies beyond one face: 3 padding layers + the face plane itself
+        if (thin > 4) ++bad;
+      }
     }
   }
   if (bad) throw BuildError{-2, "padding map construction failed"};

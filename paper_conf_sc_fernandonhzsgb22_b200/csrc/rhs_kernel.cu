@@ -32,19 +32,29 @@ namespace {
 constexpr int RT = 352;   // threads (11 warps); 343 interior points
 constexpr int NPP = RT;   // slot stride in doubles: slots are indexed by thread
 
-// shared-memory slot map ([slot][NPP] doubles)
-constexpr int V_GT = 0, V_B = 3, V_GAM = 6, V_AT = 12;                         // values (18)
-constexpr int A_GT = 18, A_BETA = 21, A_B = 24, A_GAM = 27, A_AT = 33;         // accumulators (21)
-constexpr int G_INV = 39;                                                      // gt^ij (6)
-constexpr int S0 = 45;                                                         // scratch (24)
-constexpr int NSLOT = 69;
-constexpr size_t SMEM_BYTES = size_t(NSLOT) * NPP * 8 + size_t(2) * STAGE_DBL * 8 + 16;
+// shared-memory slot map ([slot][NPP] doubles).  Slot reuse: during the gt
+// stages the A_AT slots hold gt^lm d_lm gt_ij (A_AT is first written by the
+// Christoffel block) and from the Christoffel block to the beta stages the A_B
+// slots hold CalGt^k (A_B is first written by the B stage).
+constexpr int V_GAM = 0, V_AT = 6;                                             // values (12)
+constexpr int A_GT = 12, A_BETA = 15, A_B = 18, A_GAM = 21, A_AT = 27;         // accumulators (21)
+constexpr int G_INV = 33;                                                      // gt^ij (6)
+constexpr int S0 = 39;                                                         // scratch (18)
+constexpr int NSLOT = 57;
+// first x-/y-derivatives of the staged field for the mixed second derivatives
+// (D_xy = D1_y D1_x, D_xz = D1_z D1_x, D_yz = D1_z D1_y), stored at the patch
+// index c = x + 13y + 169z minus an offset so thread reads stay conflict-free
+constexpr int TX_OFF = 3, TX_N = 2191;    // x in 3..9, y, z in 0..12
+constexpr int TY_OFF = 42, TY_N = 2113;   // x, y in 3..9, z in 0..12
+constexpr size_t SMEM_BYTES =
+    size_t(NSLOT) * NPP * 8 + size_t(2) * STAGE_DBL * 8 + size_t(TX_N + TY_N) * 8 + 16;
 
 // thread -> interior point map (filled by upload_rhs_tables): every warp holds
 // at most two points per residue of their stage-buffer index mod 16, so its
 // 8-byte stencil loads hit each of the 16 bank pairs at most twice (2
 // wavefronts, conflict-free); shifted stencil taps only rotate the residues.
-__constant__ int16_t c_perm[RT];
+// (global memory, not __constant__: every thread reads a different entry)
+__device__ int16_t g_perm[RT];
 
 // field processing order
 __constant__ int c_order[NF] = {12, 13, 14, 15, 16, 17, 1, 0, 3, 4, 5, 6,
@@ -147,6 +157,36 @@ __device__ __forceinline__ Derivs derivs(const double* __restrict__ s, int c, do
   return d;
 }
 
+// D1 of a precomputed D1 field (raw numerators), at patch index c
+__device__ __forceinline__ double d1_of(const double* __restrict__ T, int c, int st) {
+  return (T[c + st] - T[c - st]) * 45.0 - (T[c + 2 * st] - T[c - 2 * st]) * 9.0 +
+         (T[c + 3 * st] - T[c - 3 * st]);
+}
+
+// first, pure second and mixed derivatives + KO; the mixed ones from the
+// cooperative Tx = D1_x u and Ty = D1_y u fields (same D1 o D1 stencil, R10)
+__device__ __forceinline__ Derivs derivs2(const double* __restrict__ s,
+                                          const double* __restrict__ Tx,
+                                          const double* __restrict__ Ty, int c, double ih,
+                                          double ko_scale) {
+  Derivs d;
+  const Line lx = line_ops(s, c, 1), ly = line_ops(s, c, 13), lz = line_ops(s, c, 169);
+  const double f1 = ih * (1.0 / 60.0);
+  d.d1[0] = lx.d1 * f1;
+  d.d1[1] = ly.d1 * f1;
+  d.d1[2] = lz.d1 * f1;
+  d.ko = (lx.ko + ly.ko + lz.ko) * ko_scale;
+  const double f2 = ih * ih * (1.0 / 180.0);
+  const double fm = ih * ih * (1.0 / 3600.0);
+  d.dd[0] = lx.d2 * f2;
+  d.dd[3] = ly.d2 * f2;
+  d.dd[5] = lz.d2 * f2;
+  d.dd[1] = d1_of(Tx, c - TX_OFF, 13) * fm;
+  d.dd[2] = d1_of(Tx, c - TX_OFF, 169) * fm;
+  d.dd[4] = d1_of(Ty, c - TY_OFF, 169) * fm;
+  return d;
+}
+
 // trace with the inverse metric: gt^ij X_ij (symmetric storage)
 __device__ __forceinline__ double trace6(const double* gi, const double* X) {
   return gi[0] * X[0] + gi[3] * X[3] + gi[5] * X[5] +
@@ -161,11 +201,13 @@ __global__ void __launch_bounds__(RT, 1)
   extern __shared__ __align__(128) double smem[];
   double* slots = smem;                           // [NSLOT][NPP]
   double* stage = smem + NSLOT * NPP;             // [2][STAGE_DBL]
-  uint64_t* bars = reinterpret_cast<uint64_t*>(stage + 2 * STAGE_DBL);
+  double* Tx = stage + 2 * STAGE_DBL;             // [TX_N]
+  double* Ty = Tx + TX_N;                         // [TY_N]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(Ty + TY_N);
 
   const int e = blockIdx.x;
   const int tid = threadIdx.x;
-  const int pp = c_perm[tid];
+  const int pp = g_perm[tid];
   const bool active = pp >= 0;
   const int p = active ? pp : 0;
   const int pi = p % 7, pj = (p / 7) % 7, pk = p / 49;
@@ -203,11 +245,7 @@ __global__ void __launch_bounds__(RT, 1)
     chi = __ldg(pbase + 1 * fstride + c0);
     Kv = __ldg(pbase + 2 * fstride + c0);
 #pragma unroll
-    for (int i = 0; i < 3; ++i) {
-      SL(V_GT + i) = __ldg(pbase + (3 + i) * fstride + c0);
-      beta[i] = __ldg(pbase + (6 + i) * fstride + c0);
-      SL(V_B + i) = __ldg(pbase + (9 + i) * fstride + c0);
-    }
+    for (int i = 0; i < 3; ++i) beta[i] = __ldg(pbase + (6 + i) * fstride + c0);
     double g[6];
 #pragma unroll
     for (int q = 0; q < 6; ++q) {
@@ -228,7 +266,9 @@ __global__ void __launch_bounds__(RT, 1)
     SL(G_INV + 4) = (g[1] * g[2] - g[0] * g[4]) * idet;
     SL(G_INV + 5) = (g[0] * g[3] - g[1] * g[1]) * idet;
 #pragma unroll
-    for (int q = 0; q < 21; ++q) SL(A_GT + q) = 0.0;
+    for (int q = 0; q < 6; ++q) SL(A_GT + q) = 0.0;     // A_GT, A_BETA
+#pragma unroll
+    for (int q = 0; q < 6; ++q) SL(A_GAM + q) = 0.0;
   }
   const double chi_e = fmax(chi, prm.chi_floor);
   const double ichi = 1.0 / chi_e;
@@ -240,17 +280,39 @@ __global__ void __launch_bounds__(RT, 1)
     mbar_wait(&bars[buf], (st >> 1) & 1);
     const double* s = stage + buf * STAGE_DBL;
     const int f = c_order[st];
+    const bool second = f <= 1 || (f >= 6 && f <= 8) || (f >= 12 && f <= 17);
+    if (second) {
+      // cooperative first derivatives along x (and y) of the staged field on
+      // the extended region the mixed stencils need (each value once, instead
+      // of 36 loads per mixed derivative per point)
+      // item order keeps warps bank-conflict-free: Tx items run along rows
+      // (y + 13 z) at fixed x (13 == -3 is a unit mod 16), Ty items along z at
+      // fixed (x, y) (169 == 9 is a unit mod 16)
+      for (int k = tid; k < 1183 + 637; k += RT) {
+        if (k < 1183) {
+          const int c = 3 + (k / 169) + 13 * (k % 169);
+          Tx[c - TX_OFF] = (s[c + 1] - s[c - 1]) * 45.0 - (s[c + 2] - s[c - 2]) * 9.0 +
+                           (s[c + 3] - s[c - 3]);
+        } else {
+          const int k2 = k - 1183, xy = k2 / 13;
+          const int c = 3 + (xy % 7) + 13 * (3 + xy / 7) + 169 * (k2 % 13);
+          Ty[c - TY_OFF] = (s[c + 13] - s[c - 13]) * 45.0 - (s[c + 26] - s[c - 26]) * 9.0 +
+                           (s[c + 39] - s[c - 39]);
+        }
+      }
+      __syncthreads();
+    }
     if (active) {
       if (f >= 12 && f <= 17) {
         // ---------------- conformal metric gt_q: d gt, gt^lm d_lm gt, adv, KO
         const int q = f - 12;
-        const Derivs d = derivs<true>(s, c0, ih, ko_scale);
+        const Derivs d = derivs2(s, Tx, Ty, c0, ih, ko_scale);
         double gi[6];
 #pragma unroll
         for (int r = 0; r < 6; ++r) gi[r] = SL(G_INV + r);
 #pragma unroll
         for (int k = 0; k < 3; ++k) SL(S0 + k * 6 + q) = d.d1[k];
-        SL(S0 + 18 + q) = trace6(gi, d.dd);
+        SL(A_AT + q) = trace6(gi, d.dd);   // (A_AT slot reused until the Christoffel block)
         SL(A_GAM + q) += beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
         if (q == 5) {
           // ---------------- Christoffel block (eqs 12, 17; readings R1, R7)
@@ -285,7 +347,7 @@ __global__ void __launch_bounds__(RT, 1)
           for (int i = 0; i < 3; ++i)
 #pragma unroll
             for (int j = i; j < 3; ++j) {
-              double r = -0.5 * SL(S0 + 18 + sidx(i, j));
+              double r = -0.5 * SL(A_AT + sidx(i, j));      // gt^lm d_lm gt_ij
               double c2 = 0.0;
 #pragma unroll
               for (int k = 0; k < 3; ++k) c2 += cal[k] * (C[i][sidx(j, k)] + C[j][sidx(i, k)]);
@@ -306,11 +368,11 @@ __global__ void __launch_bounds__(RT, 1)
                 }
               Rt[sidx(i, j)] = r + qsum;
             }
-          // At_ij += chi alpha TF(Rt)
+          // At_ij = chi alpha TF(Rt)   (first write of the A_AT accumulators)
           const double trR = trace6(gi, Rt);
           const double ca = chi * alpha;
 #pragma unroll
-          for (int r = 0; r < 6; ++r) SL(A_AT + r) += ca * (Rt[r] - gt[r] * trR * (1.0 / 3.0));
+          for (int r = 0; r < 6; ++r) SL(A_AT + r) = ca * (Rt[r] - gt[r] * trR * (1.0 / 3.0));
           // At^ij = gt^ik gt^jl At_kl ; Gt^i += 2 alpha Gt^i_jk At^jk
           double Au[6];
 #pragma unroll
@@ -332,11 +394,11 @@ __global__ void __launch_bounds__(RT, 1)
 #pragma unroll
             for (int q2 = 0; q2 < 6; ++q2) SL(S0 + k * 6 + q2) = Gam[k][q2];
 #pragma unroll
-          for (int k = 0; k < 3; ++k) SL(S0 + 18 + k) = cal[k];
+          for (int k = 0; k < 3; ++k) SL(A_B + k) = cal[k];   // (A_B slot reused until B)
         }
       } else if (f == 1) {
         // ---------------- chi: advection, KO, R^chi (eq 18-19), eq (8) chi term
-        const Derivs d = derivs<true>(s, c0, ih, ko_scale);
+        const Derivs d = derivs2(s, Tx, Ty, c0, ih, ko_scale);
         double gi[6], At[6], gt[6];
 #pragma unroll
         for (int r = 0; r < 6; ++r) {
@@ -378,7 +440,7 @@ __global__ void __launch_bounds__(RT, 1)
         }
       } else if (f == 0) {
         // ---------------- alpha: advection, KO, D_i D_j alpha (eqs 13-15)
-        const Derivs d = derivs<true>(s, c0, ih, ko_scale);
+        const Derivs d = derivs2(s, Tx, Ty, c0, ih, ko_scale);
         double gi[6], At[6], gt[6];
 #pragma unroll
         for (int r = 0; r < 6; ++r) {
@@ -446,14 +508,14 @@ __global__ void __launch_bounds__(RT, 1)
       } else if (f >= 6 && f <= 8) {
         // ---------------- beta^kk: Lie derivative terms, eq (2), eq (8) shift terms
         const int kk = f - 6;
-        const Derivs d = derivs<true>(s, c0, ih, ko_scale);
+        const Derivs d = derivs2(s, Tx, Ty, c0, ih, ko_scale);
         const double* db = d.d1;   // d_j beta^kk
         SL(A_BETA + kk) += beta[0] * db[0] + beta[1] * db[1] + beta[2] * db[2] + d.ko;
         double gi[6], cal[3];
 #pragma unroll
         for (int r = 0; r < 6; ++r) gi[r] = SL(G_INV + r);
 #pragma unroll
-        for (int k = 0; k < 3; ++k) cal[k] = SL(S0 + 18 + k);
+        for (int k = 0; k < 3; ++k) cal[k] = SL(A_B + k);
         // Lie derivative pieces for T = gt and At:  T_i,kk d_j b + T_kk,j d_i b - 2/3 T_ij d_kk b
 #pragma unroll
         for (int t = 0; t < 2; ++t) {
@@ -500,7 +562,7 @@ __global__ void __launch_bounds__(RT, 1)
       } else {  // 9..11: B
         const int kk = f - 9;
         const Derivs d = derivs<false>(s, c0, ih, ko_scale);
-        SL(A_B + kk) += beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
+        SL(A_B + kk) = beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
       }
     }
     __syncthreads();  // everyone is done with this stage buffer
@@ -518,7 +580,7 @@ __global__ void __launch_bounds__(RT, 1)
       At[r] = SL(V_AT + r);
     }
 #pragma unroll
-    for (int i = 0; i < 3; ++i) B[i] = SL(V_B + i);
+    for (int i = 0; i < 3; ++i) B[i] = __ldg(pbase + (9 + i) * fstride + c0);
     double* out = rhs_oct + int64_t(e) * NPT + p;
     const int64_t ostr = no * NPT;
     // At^k_j and At_ik At^k_j, At_ij At^ij
@@ -575,7 +637,7 @@ void upload_rhs_tables() {
       const int r = lane % 16;
       if (next[r] < bucket[r].size()) perm[w * 32 + lane] = int16_t(bucket[r][next[r]++]);
     }
-  cudaMemcpyToSymbol(c_perm, perm, sizeof(perm));
+  cudaMemcpyToSymbol(g_perm, perm, sizeof(perm));
 }
 
 void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const RhsParams& p,

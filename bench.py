@@ -41,7 +41,12 @@ RHS_BYTES_PER_OCT = 24 * (2197 + 343) * 8         # patch read + rhs write (eq 2
 PAPER_FLOPS_PER_POINT = 5502 + 3998               # eq (21a) numerator per point, O_A from Q_L = 6.68
 # executed fp64 FLOPs per interior point of k_rhs (2 per DFMA + DADD + DMUL), from
 # ncu sm__sass_thread_inst_executed_op_d{fma,add,mul}_pred_on (profiles/)
-RHS_EXEC_FLOPS_PER_POINT = float(os.environ.get("DGR_RHS_FLOPS_PER_POINT", "0")) or None
+# (profiles/r1_ncu_flops.txt: 4.491e10 FLOP per C3 launch / 8,329,412 points = 5,392)
+RHS_EXEC_FLOPS_PER_POINT = float(os.environ.get("DGR_RHS_FLOPS_PER_POINT", "5392"))
+# DRAM bytes per launch (dram__bytes_read.sum + dram__bytes_write.sum) from one
+# ncu --set full capture of the C3 workload on 1 GPU (profiles/r1_ncu_full_c3_kernels.txt)
+NCU_TRAFFIC_C3 = {"rhs": 18.723e9 + 3.207e9, "unzip": 3.261e9 + 10.850e9,
+                  "elements": 1.819e9 + 1.561e9}
 
 
 def _peaks():
@@ -309,7 +314,10 @@ def main():
     if dom and "bound" in kern[dom]:
         k = kern[dom]
         roof = {"kernel": dom, "bound": k["bound"], "achieved": k["achieved"], "peak": k["peak"],
-                "unit": k["unit"], "frac": k["frac"], "traffic": None,
+                "unit": k["unit"], "frac": k["frac"],
+                "traffic": (NCU_TRAFFIC_C3.get(dom) if cfg.name == "c3" and world == 1
+                            else None),
+                "traffic_unit": "bytes per launch (ncu dram read+write)",
                 "peak_source": (f"MEASURED_PEAKS.json ({peak_kind})" if k["bound"] == "hbm" else
                                 "148 SM x 64 DFMA/clk x 2 x sm_max_mhz (derived)")}
     cpu = None

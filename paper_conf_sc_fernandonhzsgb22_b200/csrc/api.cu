@@ -236,15 +236,15 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
                       cudaMemcpyHostToDevice));
   CUDA_TRY(m->alloc(&m->d_zip, h.zip_local.size()));
   CUDA_TRY(cudaMemcpy(m->d_zip, h.zip_local.data(), h.zip_local.size() * 4, cudaMemcpyHostToDevice));
-  // hanging rows grouped by level
+  // hanging rows grouped by dependency depth (one launch per depth)
   std::vector<int4> hr(h.hang_rows.size());
   m->hang_level_off.clear();
   int prev = -1;
   for (size_t i = 0; i < h.hang_rows.size(); ++i) {
     const auto& r = h.hang_rows[i];
-    if (r.level != prev) {
+    if (r.depth != prev) {
       m->hang_level_off.push_back(int64_t(i));
-      prev = r.level;
+      prev = r.depth;
     }
     hr[i] = make_int4(r.e_local, r.node, r.src_local, r.t2[0] | (r.t2[1] << 8) | (r.t2[2] << 16));
   }

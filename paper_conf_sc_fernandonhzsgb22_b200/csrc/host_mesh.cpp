@@ -580,6 +580,32 @@ void HostMesh::partition() {
   }
   std::stable_sort(hang_rows.begin(), hang_rows.end(),
                    [](const HangRow& a, const HangRow& b) { return a.level < b.level; });
+  // dependency depth (reading R14): a row whose interpolation stencil on its
+  // source octant touches only DOF nodes has depth 0, otherwise 1 + the
+  // deepest hanging node it reads.  Rows of equal depth are independent, so
+  // the device resolves one depth per launch (typically 2-3 instead of one
+  // launch per level).  Level order guarantees sources are visited first.
+  std::vector<int32_t> depth_of(size_t(nl) * NPT, -1);
+  for (HangRow& r : hang_rows) {
+    int d = 0;
+    const int nx = (r.t2[0] & 1) ? 7 : 1, ny = (r.t2[1] & 1) ? 7 : 1, nz = (r.t2[2] & 1) ? 7 : 1;
+    const int x0 = (r.t2[0] & 1) ? 0 : r.t2[0] / 2, y0 = (r.t2[1] & 1) ? 0 : r.t2[1] / 2,
+              z0 = (r.t2[2] & 1) ? 0 : r.t2[2] / 2;
+    for (int c = 0; c < nz; ++c)
+      for (int b = 0; b < ny; ++b)
+        for (int a = 0; a < nx; ++a) {
+          const int n = (x0 + a) + 7 * (y0 + b) + 49 * (z0 + c);
+          const int32_t ds = depth_of[size_t(r.src_local) * NPT + n];
+          if (o2n_local[size_t(r.src_local) * NPT + n] < 0) {
+            if (ds < 0) throw BuildError{-2, "hanging chain out of order"};
+            d = std::max(d, ds + 1);
+          }
+        }
+    r.depth = d;
+    depth_of[size_t(r.e_local) * NPT + r.node] = d;
+  }
+  std::stable_sort(hang_rows.begin(), hang_rows.end(),
+                   [](const HangRow& a, const HangRow& b) { return a.depth < b.depth; });
 }
 
 // Padding sources of owned octants (R15): finest touching leaf whose

@@ -99,7 +99,12 @@ class HostMesh {
   std::vector<int32_t> pad_src_global;         // [n_owned * 2197] export
   std::vector<uint8_t> pad_kind;               // [n_owned * 2197] export
   // hanging rows over local octants, sorted by (level, local octant, node)
-  struct HangRow { int32_t e_local, node, src_local; uint8_t t2[3]; int level; int32_t e_global; int32_t src_global; };
+  struct HangRow {
+    int32_t e_local, node, src_local;
+    uint8_t t2[3];
+    int level, depth;
+    int32_t e_global, src_global;
+  };
   std::vector<HangRow> hang_rows;
   // zip: owned DOF -> local octant * 343 + node
   std::vector<int32_t> zip_local;

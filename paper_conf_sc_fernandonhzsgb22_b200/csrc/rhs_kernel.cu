@@ -205,7 +205,6 @@ __global__ void __launch_bounds__(RT, 1)
   double* Ty = Tx + TX_N;                         // [TY_N]
   uint64_t* bars = reinterpret_cast<uint64_t*>(Ty + TY_N);
 
-  const int e = blockIdx.x;
   const int tid = threadIdx.x;
   const int pp = g_perm[tid];
   const bool active = pp >= 0;
@@ -213,26 +212,36 @@ __global__ void __launch_bounds__(RT, 1)
   const int pi = p % 7, pj = (p / 7) % 7, pk = p / 49;
   const int c0 = (pi + 3) + 13 * (pj + 3) + 169 * (pk + 3);
   const int64_t no = m.n_owned;
-  const double* pbase = patches + int64_t(e) * PATCH_PITCH;
   const int64_t fstride = no * PATCH_PITCH;
 #define SL(slot) slots[(slot) * NPP + tid]
+  auto prefetch_l2 = [&](const double* src) {
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src),
+                 "r"(uint32_t(STAGE_DBL * 8))
+                 : "memory");
+  };
 
+  // Persistent CTAs: octants e = blockIdx.x, +gridDim.x, ...  The field stream
+  // (double-buffered bulk copies, mbarrier phase = global stage count) runs
+  // on across octant boundaries, and the next octant's 24 field patches are
+  // prefetched into L2 one octant ahead.
+  int e = blockIdx.x;
+  if (e >= no) return;
   if (tid == 0) {
     mbar_init(&bars[0], 1);
     mbar_init(&bars[1], 1);
   }
   __syncthreads();
   if (tid == 0) {
-    bulk_load(stage, pbase + c_order[0] * fstride, STAGE_DBL * 8, &bars[0]);
-    bulk_load(stage + STAGE_DBL, pbase + c_order[1] * fstride, STAGE_DBL * 8, &bars[1]);
+    const double* pb = patches + int64_t(e) * PATCH_PITCH;
+    bulk_load(stage, pb + c_order[0] * fstride, STAGE_DBL * 8, &bars[0]);
+    bulk_load(stage + STAGE_DBL, pb + c_order[1] * fstride, STAGE_DBL * 8, &bars[1]);
   } else if (tid < NF - 1) {
-    // pull the other 22 field patches of this octant into L2 now, so the
-    // double-buffered bulk copies later hit L2 instead of waiting on HBM
-    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(pbase + c_order[tid + 1] *
-                                                                            fstride),
-                 "r"(uint32_t(STAGE_DBL * 8))
-                 : "memory");
+    prefetch_l2(patches + int64_t(e) * PATCH_PITCH + c_order[tid + 1] * fstride);
   }
+  uint32_t g = 0;   // global stage counter of this CTA
+  for (; e < no; e += gridDim.x) {
+  const int en = e + gridDim.x;                    // next octant of this CTA
+  const double* pbase = patches + int64_t(e) * PATCH_PITCH;
 
   const int4 oi = m.oct[e];
   const double ih = (6.0 * double(int64_t(1) << oi.w)) / m.width;   // 1/h
@@ -275,9 +284,9 @@ __global__ void __launch_bounds__(RT, 1)
   double rA = 0.0, rC = 0.0, rK = 0.0;   // accumulators of alpha, chi, K
   double dchi[3] = {0, 0, 0};
 
-  for (int st = 0; st < NF; ++st) {
-    const int buf = st & 1;
-    mbar_wait(&bars[buf], (st >> 1) & 1);
+  for (int st = 0; st < NF; ++st, ++g) {
+    const int buf = g & 1;
+    mbar_wait(&bars[buf], (g >> 1) & 1);
     const double* s = stage + buf * STAGE_DBL;
     const int f = c_order[st];
     const bool second = f <= 1 || (f >= 6 && f <= 8) || (f >= 12 && f <= 17);
@@ -566,9 +575,20 @@ __global__ void __launch_bounds__(RT, 1)
       }
     }
     __syncthreads();  // everyone is done with this stage buffer
-    if (tid == 0 && st + 2 < NF)
-      bulk_load(stage + buf * STAGE_DBL, pbase + c_order[st + 2] * fstride, STAGE_DBL * 8,
-                &bars[buf]);
+    // L2 prefetch one octant ahead: the next octant's field of this stage
+    // (measured faster than prefetching the current octant at its start,
+    // although some prefetched lines are evicted and re-read)
+    if (tid == 32 && en < no)
+      prefetch_l2(patches + int64_t(en) * PATCH_PITCH + c_order[st] * fstride);
+    if (tid == 0) {
+      if (st + 2 < NF)
+        bulk_load(stage + buf * STAGE_DBL, pbase + c_order[st + 2] * fstride, STAGE_DBL * 8,
+                  &bars[buf]);
+      else if (en < no)   // the stream continues with the next octant's first fields
+        bulk_load(stage + buf * STAGE_DBL,
+                  patches + int64_t(en) * PATCH_PITCH + c_order[st + 2 - NF] * fstride,
+                  STAGE_DBL * 8, &bars[buf]);
+    }
   }
 
   // ---- epilogue: undifferentiated terms, combine, store ----------------------
@@ -618,6 +638,7 @@ __global__ void __launch_bounds__(RT, 1)
         out[(18 + q) * ostr] = SL(A_AT + q) + alpha * (Kv * At[q] - 2.0 * AAij);  // (6)
       }
   }
+  }  // octant loop
 #undef SL
 }
 
@@ -643,12 +664,17 @@ void upload_rhs_tables() {
 void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const RhsParams& p,
                 cudaStream_t s) {
   if (m.n_owned <= 0) return;
-  static bool attr = false;
-  if (!attr) {
+  static int n_sm = 0;
+  if (!n_sm) {
     cudaFuncSetAttribute(k_rhs, cudaFuncAttributeMaxDynamicSharedMemorySize, int(SMEM_BYTES));
-    attr = true;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n_sm, cudaDevAttrMultiProcessorCount, dev);
+    if (n_sm <= 0) n_sm = 148;
   }
-  k_rhs<<<m.n_owned, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p);
+  // persistent: one CTA per SM (225 KB of shared memory each)
+  const int grid = m.n_owned < n_sm ? m.n_owned : n_sm;
+  k_rhs<<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p);
 }
 
 }  // namespace dgr

@@ -91,9 +91,9 @@ __global__ void __launch_bounds__(UZ_THREADS, 3)
   }
   __syncthreads();
 
-  const int f = blockIdx.y * UZ_WARPS + warp;
-  if (f >= nf) return;
+  // warp w builds fields w, w + 8, w + 16 (the setup above is done once per octant)
   const int64_t nn = int64_t(m.n_local) * NPT;
+  for (int f = warp; f < nf; f += UZ_WARPS) {
   const double* Ef = E + f * nn;
   double* dst = patches + (int64_t(f) * m.n_owned + e) * PATCH_PITCH;
 
@@ -240,6 +240,7 @@ __global__ void __launch_bounds__(UZ_THREADS, 3)
       }
     }
   }
+  }  // field loop
 }
 
 void launch_unzip(const DevMesh& m, const double* E, double* patches, int nf, cudaStream_t s) {
@@ -250,8 +251,7 @@ void launch_unzip(const DevMesh& m, const double* E, double* patches, int nf, cu
     cudaFuncSetAttribute(k_unzip, cudaFuncAttributeMaxDynamicSharedMemorySize, int(dyn));
     attr = true;
   }
-  k_unzip<<<dim3(m.n_owned, (nf + UZ_WARPS - 1) / UZ_WARPS), UZ_THREADS, dyn, s>>>(m, E, patches,
-                                                                                  nf);
+  k_unzip<<<m.n_owned, UZ_THREADS, dyn, s>>>(m, E, patches, nf);
 }
 
 }  // namespace dgr

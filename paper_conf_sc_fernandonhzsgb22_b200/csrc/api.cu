@@ -94,6 +94,7 @@ struct dgr_mesh_s {
   uint8_t* d_pmap = nullptr;
   NbrEntry* d_nbr = nullptr;
   int32_t* d_zip = nullptr;
+  int32_t* d_own = nullptr;     // [n_owned*343] zip-owned DOF of each point or -1
   int4* d_hang = nullptr;
   std::vector<int64_t> hang_level_off;  // row offsets per level group
   int64_t* d_dof_node = nullptr;
@@ -234,6 +235,13 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
   CUDA_TRY(m->alloc(&m->d_nbr, h.nbr.size()));
   CUDA_TRY(cudaMemcpy(m->d_nbr, h.nbr.data(), h.nbr.size() * sizeof(NbrEntry),
                       cudaMemcpyHostToDevice));
+  {
+    // inverse zip map for the fused RHS epilogue: point -> owned DOF it is the zip owner of
+    std::vector<int32_t> own(size_t(no) * NPT, -1);
+    for (size_t l = 0; l < h.zip_local.size(); ++l) own[h.zip_local[l]] = int32_t(l);
+    CUDA_TRY(m->alloc(&m->d_own, own.size()));
+    CUDA_TRY(cudaMemcpy(m->d_own, own.data(), own.size() * 4, cudaMemcpyHostToDevice));
+  }
   CUDA_TRY(m->alloc(&m->d_zip, h.zip_local.size()));
   CUDA_TRY(cudaMemcpy(m->d_zip, h.zip_local.data(), h.zip_local.size() * 4, cudaMemcpyHostToDevice));
   // hanging rows grouped by dependency depth (one launch per depth)
@@ -560,7 +568,7 @@ dgr_status dgr_rhs_patches(dgr_mesh m, const double* patches, double* rhs_oct,
   if (s) return s;
   if (!patches || !rhs_oct || !aligned16(patches)) return fail(DGR_ERR_ARG, "bad rhs args");
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  PROF(m, 3, st, launch_rhs(m->dm, patches, rhs_oct, to_rp(prm), st));
+  PROF(m, 3, st, launch_rhs(m->dm, patches, rhs_oct, to_rp(prm), nullptr, st));
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;
 }
@@ -573,7 +581,7 @@ dgr_status dgr_rhs(dgr_mesh m, double* u, double* rhs, const dgr_params* prm, vo
   m->launches = 0;
   if ((s = exchange(m, u, st))) return s;
   if ((s = do_unzip(m, u, NF, st))) return s;
-  PROF(m, 3, st, launch_rhs(m->dm, m->d_patch, m->d_rhs_oct, to_rp(prm), st));
+  PROF(m, 3, st, launch_rhs(m->dm, m->d_patch, m->d_rhs_oct, to_rp(prm), nullptr, st));
   PROF(m, 4, st, launch_zip(m->dm, m->d_rhs_oct, rhs, NF, st));
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;
@@ -585,7 +593,10 @@ static dgr_status stage(dgr_mesh m, int s_, double dt, double* u_n, double* u_s,
   double* cur = s_ == 0 ? u_n : u_s;
   if ((s = exchange(m, cur, st))) return s;
   if ((s = do_unzip(m, cur, NF, st))) return s;
-  PROF(m, 3, st, launch_rhs(m->dm, m->d_patch, m->d_rhs_oct, to_rp(prm), st));
+  // (k_rhs can also apply the zip + RK4 update in its epilogue (RkArgs); on C3
+  // that measured 10.6 ms vs 7.5 + 0.8 ms for RHS + k_zip_rk4 — the scattered
+  // state loads stall the single persistent CTA per SM — so it is not used)
+  PROF(m, 3, st, launch_rhs(m->dm, m->d_patch, m->d_rhs_oct, to_rp(prm), nullptr, st));
   PROF(m, 4, st, launch_zip_rk4(m->dm, m->d_rhs_oct, s_, dt, u_n, u_s, acc, u_out, st));
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;

@@ -49,8 +49,19 @@ void launch_dfma(int blocks, int iters, double* out, cudaStream_t s);
 struct RhsParams {
   double ko_sigma, eta, lambda_f0, lambda_f1, chi_floor;
 };
+// Fused patch-to-octant + RK4 stage in the RHS epilogue (s < 0: write rhs_oct).
+struct RkArgs {
+  int s;
+  double dt;
+  const double* u_n;
+  double* u_s;
+  double* acc;
+  double* u_out;
+  const int32_t* own;   // [n_owned * 343]: owned DOF this point is the zip owner of, or -1
+  int64_t stride;
+};
 void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const RhsParams& p,
-                cudaStream_t s);
+                const RkArgs* rk, cudaStream_t s);
 size_t rhs_smem_bytes();
 void upload_rhs_tables();
 

@@ -56,6 +56,14 @@ constexpr size_t SMEM_BYTES =
 // (global memory, not __constant__: every thread reads a different entry)
 __device__ int16_t g_perm[RT];
 
+// Items of the cooperative D1 pass: Tx on the cross-shaped region the mixed
+// stencils read (x interior; y all with z interior, or z all with y interior),
+// Ty on x, y interior with all z; each entry is the patch index c.  Tx items
+// run along rows (y + 13 z) at fixed x so a warp's addresses have distinct
+// residues mod 16 (13 is a unit mod 16); Ty items along z (169 is a unit).
+constexpr int N_TX = 7 * (13 * 7 + 7 * 6), N_TY = 7 * 7 * 13, N_TITEM = N_TX + N_TY;
+__device__ int16_t g_titem[N_TITEM];
+
 // field processing order
 __constant__ int c_order[NF] = {12, 13, 14, 15, 16, 17, 1, 0, 3, 4, 5, 6,
                                 7,  8,  2,  18, 19, 20, 21, 22, 23, 9, 10, 11};
@@ -197,7 +205,7 @@ __device__ __forceinline__ double trace6(const double* gi, const double* X) {
 
 __global__ void __launch_bounds__(RT, 1)
     k_rhs(DevMesh m, const double* __restrict__ patches, double* __restrict__ rhs_oct,
-          RhsParams prm) {
+          RhsParams prm, RkArgs rk) {
   extern __shared__ __align__(128) double smem[];
   double* slots = smem;                           // [NSLOT][NPP]
   double* stage = smem + NSLOT * NPP;             // [2][STAGE_DBL]
@@ -297,14 +305,12 @@ __global__ void __launch_bounds__(RT, 1)
       // item order keeps warps bank-conflict-free: Tx items run along rows
       // (y + 13 z) at fixed x (13 == -3 is a unit mod 16), Ty items along z at
       // fixed (x, y) (169 == 9 is a unit mod 16)
-      for (int k = tid; k < 1183 + 637; k += RT) {
-        if (k < 1183) {
-          const int c = 3 + (k / 169) + 13 * (k % 169);
+      for (int k = tid; k < N_TITEM; k += RT) {
+        const int c = __ldg(g_titem + k);          // patch index of the item (table)
+        if (k < N_TX) {
           Tx[c - TX_OFF] = (s[c + 1] - s[c - 1]) * 45.0 - (s[c + 2] - s[c - 2]) * 9.0 +
                            (s[c + 3] - s[c - 3]);
         } else {
-          const int k2 = k - 1183, xy = k2 / 13;
-          const int c = 3 + (xy % 7) + 13 * (3 + xy / 7) + 169 * (k2 % 13);
           Ty[c - TY_OFF] = (s[c + 13] - s[c - 13]) * 45.0 - (s[c + 26] - s[c - 26]) * 9.0 +
                            (s[c + 39] - s[c - 39]);
         }
@@ -601,8 +607,6 @@ __global__ void __launch_bounds__(RT, 1)
     }
 #pragma unroll
     for (int i = 0; i < 3; ++i) B[i] = __ldg(pbase + (9 + i) * fstride + c0);
-    double* out = rhs_oct + int64_t(e) * NPT + p;
-    const int64_t ostr = no * NPT;
     // At^k_j and At_ik At^k_j, At_ij At^ij
     double Am[3][3];
 #pragma unroll
@@ -616,27 +620,59 @@ __global__ void __launch_bounds__(RT, 1)
     for (int i = 0; i < 3; ++i)
 #pragma unroll
       for (int j = 0; j < 3; ++j) AA += Am[i][j] * Am[j][i];
-    out[0 * ostr] = rA - 2.0 * alpha * Kv;                                        // (1)
-    out[1 * ostr] = rC + (2.0 / 3.0) * chi * alpha * Kv;                          // (5)
-    out[2 * ostr] = rK + alpha * (AA + Kv * Kv * (1.0 / 3.0));                    // (7)
+    double r[NF];
+    r[0] = rA - 2.0 * alpha * Kv;                                                 // (1)
+    r[1] = rC + (2.0 / 3.0) * chi * alpha * Kv;                                   // (5)
+    r[2] = rK + alpha * (AA + Kv * Kv * (1.0 / 3.0));                             // (7)
     const double fa = prm.lambda_f0 + prm.lambda_f1 * alpha;
 #pragma unroll
     for (int i = 0; i < 3; ++i) {
       const double gbar = SL(A_GT + i);
-      out[(3 + i) * ostr] = gbar + SL(S0 + i);                                    // (8)
-      out[(6 + i) * ostr] = SL(A_BETA + i) + 0.75 * fa * B[i];                    // (2)
-      out[(9 + i) * ostr] = gbar - prm.eta * B[i] + SL(A_B + i);                  // (3)
+      r[3 + i] = gbar + SL(S0 + i);                                               // (8)
+      r[6 + i] = SL(A_BETA + i) + 0.75 * fa * B[i];                               // (2)
+      r[9 + i] = gbar - prm.eta * B[i] + SL(A_B + i);                             // (3)
     }
 #pragma unroll
     for (int i = 0; i < 3; ++i)
 #pragma unroll
       for (int j = i; j < 3; ++j) {
         const int q = sidx(i, j);
-        out[(12 + q) * ostr] = SL(A_GAM + q) - 2.0 * alpha * At[q];               // (4)
+        r[12 + q] = SL(A_GAM + q) - 2.0 * alpha * At[q];                          // (4)
         const double AAij = At[sidx(i, 0)] * Am[0][j] + At[sidx(i, 1)] * Am[1][j] +
                             At[sidx(i, 2)] * Am[2][j];
-        out[(18 + q) * ostr] = SL(A_AT + q) + alpha * (Kv * At[q] - 2.0 * AAij);  // (6)
+        r[18 + q] = SL(A_AT + q) + alpha * (Kv * At[q] - 2.0 * AAij);             // (6)
       }
+    if (rk.s < 0) {
+      double* out = rhs_oct + int64_t(e) * NPT + p;
+      const int64_t ostr = no * NPT;
+#pragma unroll
+      for (int f = 0; f < NF; ++f) out[f * ostr] = r[f];
+    } else {
+      // fused patch-to-octant + RK4 stage (same arithmetic as k_zip_rk4): only
+      // the zip owner of a DOF updates it
+      const int d = __ldg(rk.own + int64_t(e) * NPT + p);
+      if (d >= 0) {
+        const double dt = rk.dt;
+#pragma unroll
+        for (int f = 0; f < NF; ++f) {
+          const int64_t i = f * rk.stride + d;
+          const double k = r[f];
+          if (rk.s == 0) {
+            const double un = rk.u_n[i];
+            rk.acc[i] = un + (dt / 6.0) * k;
+            rk.u_s[i] = un + (dt / 2.0) * k;
+          } else if (rk.s == 1) {
+            rk.acc[i] += (dt / 3.0) * k;
+            rk.u_s[i] = rk.u_n[i] + (dt / 2.0) * k;
+          } else if (rk.s == 2) {
+            rk.acc[i] += (dt / 3.0) * k;
+            rk.u_s[i] = rk.u_n[i] + dt * k;
+          } else {
+            rk.u_out[i] = rk.acc[i] + (dt / 6.0) * k;
+          }
+        }
+      }
+    }
   }
   }  // octant loop
 #undef SL
@@ -659,10 +695,23 @@ void upload_rhs_tables() {
       if (next[r] < bucket[r].size()) perm[w * 32 + lane] = int16_t(bucket[r][next[r]++]);
     }
   cudaMemcpyToSymbol(g_perm, perm, sizeof(perm));
+  // cooperative-D1 item table
+  std::vector<int16_t> items;
+  for (int x = 3; x <= 9; ++x)
+    for (int row = 0; row < 169; ++row) {
+      const int y = row % 13, z = row / 13;
+      const bool yin = y >= 3 && y <= 9, zin = z >= 3 && z <= 9;
+      if (zin || yin) items.push_back(int16_t(x + 13 * row));
+    }
+  for (int x = 3; x <= 9; ++x)
+    for (int y = 3; y <= 9; ++y)
+      for (int z = 0; z < 13; ++z) items.push_back(int16_t(x + 13 * y + 169 * z));
+  if (int(items.size()) == N_TITEM)
+    cudaMemcpyToSymbol(g_titem, items.data(), items.size() * sizeof(int16_t));
 }
 
 void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const RhsParams& p,
-                cudaStream_t s) {
+                const RkArgs* rk, cudaStream_t s) {
   if (m.n_owned <= 0) return;
   static int n_sm = 0;
   if (!n_sm) {
@@ -674,7 +723,10 @@ void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const 
   }
   // persistent: one CTA per SM (225 KB of shared memory each)
   const int grid = m.n_owned < n_sm ? m.n_owned : n_sm;
-  k_rhs<<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p);
+  RkArgs a{};
+  a.s = -1;
+  if (rk) a = *rk;
+  k_rhs<<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a);
 }
 
 }  // namespace dgr

@@ -34,7 +34,8 @@ static dgr_status fail(dgr_status s, const std::string& msg) {
   do {                                                                                \
     cudaError_t _e = (x);                                                             \
     if (_e != cudaSuccess)                                                            \
-      return fail(DGR_ERR_CUDA, std::string(#x) + ": " + cudaGetErrorString(_e));   \
+      return fail(_e == cudaErrorMemoryAllocation ? DGR_ERR_OOM : DGR_ERR_CUDA,       \
+                  std::string(#x) + ": " + cudaGetErrorString(_e));                   \
   } while (0)
 
 // ---------------------------------------------------------------- NCCL (dlopen)

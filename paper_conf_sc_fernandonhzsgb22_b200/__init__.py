@@ -18,7 +18,7 @@ from dataclasses import dataclass
 import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "lib", "libdgr.so")
+LIB_PATH = os.environ.get("DGR_LIB") or os.path.join(HERE, "lib", "libdgr.so")
 
 NF = 24
 NPT = 343

@@ -54,31 +54,38 @@ def _run(cmd, verbose):
     return r
 
 
-def build(verbose: bool = False, ptxas_verbose: bool = False) -> str:
-    os.makedirs(OBJDIR, exist_ok=True)
+def build(verbose: bool = False, ptxas_verbose: bool = False, variant: str = "") -> str:
+    """variant="timing" builds lib/libdgr_timing.so with -DDGR_RHS_TIMING (per-stage
+    cycle counters in k_rhs, for tools/rhs_stage_profile.py); never the product."""
+    objdir = OBJDIR + (("_" + variant) if variant else "")
+    lib = LIB if not variant else os.path.join(LIBDIR, f"libdgr_{variant}.so")
+    defs = ["-DDGR_RHS_TIMING"] if variant == "timing" else []
+    os.makedirs(objdir, exist_ok=True)
     objs = []
     changed = False
     for s in SOURCES_CXX:
         src = os.path.join(CSRC, s)
-        obj = os.path.join(OBJDIR, s + ".o")
+        obj = os.path.join(objdir, s + ".o")
         objs.append(obj)
         if _stale(obj, src):
             _run([shutil.which("g++") or "g++"] + CXX_FLAGS + ["-c", src, "-o", obj], verbose)
             changed = True
     for s in SOURCES_CU:
         src = os.path.join(CSRC, s)
-        obj = os.path.join(OBJDIR, s + ".o")
+        obj = os.path.join(objdir, s + ".o")
         objs.append(obj)
         if _stale(obj, src):
             extra = ["-Xptxas", "-v"] if ptxas_verbose else []
-            _run([NVCC] + CU_FLAGS + extra + ["-c", src, "-o", obj], verbose or ptxas_verbose)
+            _run([NVCC] + CU_FLAGS + defs + extra + ["-c", src, "-o", obj],
+                 verbose or ptxas_verbose)
             changed = True
-    if changed or not os.path.exists(LIB):
-        _run([NVCC] + ARCH + ["-shared", "-o", LIB] + objs +
+    if changed or not os.path.exists(lib):
+        _run([NVCC] + ARCH + ["-shared", "-o", lib] + objs +
              ["-Xcompiler", "-fopenmp", "-lgomp", "-ldl"], verbose)
-    return LIB
+    return lib
 
 
 if __name__ == "__main__":
     v = "-v" in sys.argv
-    print(build(verbose=v, ptxas_verbose="--ptxas" in sys.argv))
+    var = sys.argv[sys.argv.index("--variant") + 1] if "--variant" in sys.argv else ""
+    print(build(verbose=v, ptxas_verbose="--ptxas" in sys.argv, variant=var))

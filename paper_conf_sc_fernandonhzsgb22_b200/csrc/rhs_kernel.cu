@@ -55,6 +55,9 @@ constexpr size_t SMEM_BYTES =
 // wavefronts, conflict-free); shifted stencil taps only rotate the residues.
 // (global memory, not __constant__: every thread reads a different entry)
 __device__ int16_t g_perm[RT];
+#ifdef DGR_RHS_TIMING
+__device__ long long g_stage_cycles[NF + 2];
+#endif
 
 // Items of the cooperative D1 pass: Tx on the cross-shaped region the mixed
 // stencils read (x interior; y all with z interior, or z all with y interior),
@@ -292,8 +295,19 @@ __global__ void __launch_bounds__(RT, 1)
   double rA = 0.0, rC = 0.0, rK = 0.0;   // accumulators of alpha, chi, K
   double dchi[3] = {0, 0, 0};
 
+#ifdef DGR_RHS_TIMING
+  long long t_last = clock64();
+#endif
   for (int st = 0; st < NF; ++st, ++g) {
     const int buf = g & 1;
+#ifdef DGR_RHS_TIMING
+    if (tid == 0) {   // per-stage cycle profile (experiment builds only)
+      const long long t = clock64();
+      atomicAdd(reinterpret_cast<unsigned long long*>(&g_stage_cycles[st]),
+                (unsigned long long)(t - t_last));
+      t_last = t;
+    }
+#endif
     mbar_wait(&bars[buf], (g >> 1) & 1);
     const double* s = stage + buf * STAGE_DBL;
     const int f = c_order[st];
@@ -531,22 +545,40 @@ __global__ void __launch_bounds__(RT, 1)
         for (int r = 0; r < 6; ++r) gi[r] = SL(G_INV + r);
 #pragma unroll
         for (int k = 0; k < 3; ++k) cal[k] = SL(A_B + k);
-        // Lie derivative pieces for T = gt and At:  T_i,kk d_j b + T_kk,j d_i b - 2/3 T_ij d_kk b
+        // Lie derivative terms of gt and At (eq 10, w = -2/3) need all of d_j beta^k:
+        // the first two beta stages park d_j beta^k in scratch slots S0+3.., the
+        // last one applies  T_ik d_j b^k + T_kj d_i b^k - 2/3 T_ij d_k b^k  once
+        if (kk < 2) {
 #pragma unroll
-        for (int t = 0; t < 2; ++t) {
-          const int vb = t == 0 ? V_GAM : V_AT;
-          const int ab = t == 0 ? A_GAM : A_AT;
-          double T[6];
+          for (int j = 0; j < 3; ++j) SL(S0 + 3 + 3 * kk + j) = db[j];
+        } else {
+          double DB[3][3];   // DB[k][j] = d_j beta^k
 #pragma unroll
-          for (int r = 0; r < 6; ++r) T[r] = SL(vb + r);
+          for (int k = 0; k < 2; ++k)
 #pragma unroll
-          for (int i = 0; i < 3; ++i)
+            for (int j = 0; j < 3; ++j) DB[k][j] = SL(S0 + 3 + 3 * k + j);
 #pragma unroll
-            for (int j = i; j < 3; ++j) {
-              const int q = sidx(i, j);
-              SL(ab + q) += T[sidx(i, kk)] * db[j] + T[sidx(kk, j)] * db[i] -
-                            (2.0 / 3.0) * T[q] * db[kk];
-            }
+          for (int j = 0; j < 3; ++j) DB[2][j] = db[j];
+          const double div = DB[0][0] + DB[1][1] + DB[2][2];
+#pragma unroll
+          for (int t = 0; t < 2; ++t) {
+            const int vb = t == 0 ? V_GAM : V_AT;
+            const int ab = t == 0 ? A_GAM : A_AT;
+            double T[6];
+#pragma unroll
+            for (int r = 0; r < 6; ++r) T[r] = SL(vb + r);
+#pragma unroll
+            for (int i = 0; i < 3; ++i)
+#pragma unroll
+              for (int j = i; j < 3; ++j) {
+                const int q = sidx(i, j);
+                double l = -(2.0 / 3.0) * T[q] * div;
+#pragma unroll
+                for (int k = 0; k < 3; ++k)
+                  l += T[sidx(i, k)] * DB[k][j] + T[sidx(k, j)] * DB[k][i];
+                SL(ab + q) += l;
+              }
+          }
         }
         rC += -(2.0 / 3.0) * chi * db[kk];
         // Gt^kk += gt^jl d_jl beta^kk - CalGt^j d_j beta^kk
@@ -597,6 +629,14 @@ __global__ void __launch_bounds__(RT, 1)
     }
   }
 
+#ifdef DGR_RHS_TIMING
+  if (tid == 0) {
+    const long long t = clock64();
+    atomicAdd(reinterpret_cast<unsigned long long*>(&g_stage_cycles[NF]),
+              (unsigned long long)(t - t_last));
+    t_last = t;
+  }
+#endif
   // ---- epilogue: undifferentiated terms, combine, store ----------------------
   if (active) {
     double gi[6], At[6], B[3];
@@ -679,6 +719,20 @@ __global__ void __launch_bounds__(RT, 1)
 }
 
 size_t rhs_smem_bytes() { return SMEM_BYTES; }
+
+#ifdef DGR_RHS_TIMING
+}  // namespace dgr
+// experiment builds only (tools/rhs_stage_profile.py): summed cycles of CTA
+// thread 0 per stage slot; out[NF + 1], reset after reading
+extern "C" int dgr_debug_rhs_stage_cycles(long long* out) {
+  cudaDeviceSynchronize();
+  cudaMemcpyFromSymbol(out, dgr::g_stage_cycles, sizeof(long long) * (dgr::NF + 1));
+  long long zero[dgr::NF + 2] = {0};
+  cudaMemcpyToSymbol(dgr::g_stage_cycles, zero, sizeof(zero));
+  return 0;
+}
+namespace dgr {
+#endif
 
 void upload_rhs_tables() {
   int16_t perm[RT];

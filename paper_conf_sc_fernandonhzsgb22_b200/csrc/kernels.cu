@@ -77,18 +77,52 @@ void launch_elements(const DevMesh& m, const double* u, double* E, int nf, cudaS
 
 // --------------------------------------------------------- hanging points
 // interp_hanging (Alg. 2 lines 4-5): E[e][node] = I_src(t2), rows of one level.
+// One thread per hanging row and a group of 4 fields: the stencil (which node
+// offsets, which weights) is decoded once and applied to 4 fields at a time.
+constexpr int HANG_FG = 4;
 __global__ void k_hanging(const int4* __restrict__ rows, int64_t count, double* __restrict__ E,
-                          int64_t nn) {
+                          int64_t nn, int nf) {
   __shared__ double W[91];
   for (int i = threadIdx.x; i < 91; i += blockDim.x) W[i] = c_W13[i];
   __syncthreads();
-  const int f = blockIdx.y;
-  double* Ef = E + f * nn;
+  const int f0 = blockIdx.y * HANG_FG;
   for (int64_t r = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; r < count;
        r += int64_t(gridDim.x) * blockDim.x) {
     const int4 row = rows[r];
     const int tx = row.w & 0xff, ty = (row.w >> 8) & 0xff, tz = (row.w >> 16) & 0xff;
-    Ef[int64_t(row.x) * NPT + row.y] = interp_point(Ef + int64_t(row.z) * NPT, tx, ty, tz, W);
+    const int nx = (tx & 1) ? 7 : 1, ny = (ty & 1) ? 7 : 1, nz = (tz & 1) ? 7 : 1;
+    const int x0 = (tx & 1) ? 0 : (tx >> 1), y0 = (ty & 1) ? 0 : (ty >> 1),
+              z0 = (tz & 1) ? 0 : (tz >> 1);
+    const double* Ec = E + int64_t(row.z) * NPT;
+    double acc[HANG_FG];
+#pragma unroll
+    for (int g = 0; g < HANG_FG; ++g) acc[g] = 0.0;
+    for (int c = 0; c < nz; ++c) {
+      const double wz = (tz & 1) ? W[tz * 7 + c] : 1.0;
+      double accy[HANG_FG];
+#pragma unroll
+      for (int g = 0; g < HANG_FG; ++g) accy[g] = 0.0;
+      for (int b = 0; b < ny; ++b) {
+        const double wy = (ty & 1) ? W[ty * 7 + b] : 1.0;
+        const int off = x0 + 7 * (y0 + b) + 49 * (z0 + c);
+        double accx[HANG_FG];
+#pragma unroll
+        for (int g = 0; g < HANG_FG; ++g) accx[g] = 0.0;
+        for (int a = 0; a < nx; ++a) {
+          const double wx = (tx & 1) ? W[tx * 7 + a] : 1.0;
+#pragma unroll
+          for (int g = 0; g < HANG_FG; ++g)
+            if (f0 + g < nf) accx[g] = fma(wx, __ldg(Ec + (f0 + g) * nn + off + a), accx[g]);
+        }
+#pragma unroll
+        for (int g = 0; g < HANG_FG; ++g) accy[g] = fma(wy, accx[g], accy[g]);
+      }
+#pragma unroll
+      for (int g = 0; g < HANG_FG; ++g) acc[g] = fma(wz, accy[g], acc[g]);
+    }
+#pragma unroll
+    for (int g = 0; g < HANG_FG; ++g)
+      if (f0 + g < nf) E[(f0 + g) * nn + int64_t(row.x) * NPT + row.y] = acc[g];
   }
 }
 
@@ -97,7 +131,8 @@ void launch_hanging(const DevMesh& m, const int4* rows, int64_t count, double* E
   if (count <= 0) return;
   int blocks = int((count + 127) / 128);
   if (blocks > 148 * 16) blocks = 148 * 16;
-  k_hanging<<<dim3(blocks, nf), 128, 0, s>>>(rows, count, E, int64_t(m.n_local) * NPT);
+  k_hanging<<<dim3(blocks, (nf + HANG_FG - 1) / HANG_FG), 128, 0, s>>>(
+      rows, count, E, int64_t(m.n_local) * NPT, nf);
 }
 
 // (octant-to-patch: unzip_kernel.cu)

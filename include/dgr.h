@@ -209,6 +209,15 @@ dgr_status dgr_rk4_step(dgr_mesh m, double dt, double* u, const dgr_params* prm,
 dgr_status dgr_constraints(dgr_mesh m, double* u, double* c, double* norms_host,
                            const dgr_params* prm, void* stream);
 
+/* Execution options of a mesh (host-side switch, takes effect at the next call):
+ *   DGR_OPT_FUSED_UNZIP (default 0): 1 = dgr_rhs / dgr_rk4_* gather every patch
+ *     inside the RHS kernel straight from the element values and interpolation
+ *     slots (no patch buffer); 0 = unzip into the 13^3 patch
+ *     buffer first (Alg. 2), then the RHS reads the patches.
+ *     Both give bit-identical results. */
+enum { DGR_OPT_FUSED_UNZIP = 1 };
+dgr_status dgr_set_option(dgr_mesh m, int option, int64_t value);
+
 /* Device-side timing helper for benchmarks: number of kernel launches the last
  * dgr_rk4_step / dgr_rhs enqueued. */
 int64_t dgr_last_launch_count(dgr_mesh m);
@@ -217,7 +226,8 @@ int64_t dgr_last_launch_count(dgr_mesh m);
  * CUDA events recorded on the launching stream.  dgr_profile_read synchronises
  * and returns, per kernel class, the summed milliseconds and launch counts
  * since the last reset (classes: 0 elements, 1 hanging, 2 unzip, 3 rhs,
- * 4 zip/zip+rk4, 5 ghost pack/exchange, 6 constraints, 7 other). */
+ * 4 zip/zip+rk4, 5 ghost pack/exchange, 6 constraints, 7 interp (coarse-neighbour
+ * padding values of the fused unzip)). */
 enum { DGR_PROF_CLASSES = 8 };
 dgr_status dgr_profile_enable(dgr_mesh m, int on);
 dgr_status dgr_profile_read(dgr_mesh m, double* ms, int64_t* counts, int reset);

@@ -27,6 +27,7 @@ NPATCH = 2197
 MAP_OCTANTS, MAP_O2N, MAP_HANGING, MAP_PAD_SRC, MAP_PAD_KIND, MAP_ZIP = 0, 1, 2, 3, 4, 5
 MAP_DOF_GID, MAP_DOF_XYZ, MAP_SEND, MAP_SEND_COUNTS, MAP_RECV_COUNTS = 6, 7, 8, 9, 10
 MAP_LOCAL_OCTS, MAP_O2N_LOCAL = 11, 12
+OPT_FUSED_UNZIP = 1
 
 
 class DgrError(RuntimeError):
@@ -75,9 +76,9 @@ EXPORTED = ["dgr_status_string", "dgr_last_error", "dgr_version", "dgr_octree_bu
             "dgr_mesh_create", "dgr_mesh_info_get", "dgr_mesh_export_maps", "dgr_mesh_destroy",
             "dgr_dof_coords", "dgr_unzip", "dgr_ghost_exchange", "dgr_rhs_patches", "dgr_rhs",
             "dgr_rk4_stage", "dgr_rk4_step", "dgr_constraints", "dgr_last_launch_count",
-            "dgr_profile_enable", "dgr_profile_read", "dgr_bench_dfma"]
+            "dgr_profile_enable", "dgr_profile_read", "dgr_bench_dfma", "dgr_set_option"]
 PROF_CLASSES = ["elements", "hanging", "unzip", "rhs", "zip_rk4", "exchange", "constraints",
-                "other"]
+                "interp"]
 
 
 def lib():
@@ -111,10 +112,11 @@ def lib():
         L.dgr_profile_enable.argtypes = [vp, i32]
         L.dgr_profile_read.argtypes = [vp, vp, vp, i32]
         L.dgr_bench_dfma.argtypes = [i32, i32, vp, C.POINTER(dp), C.POINTER(dp)]
+        L.dgr_set_option.argtypes = [vp, i32, i64]
         for f in ["dgr_octree_build", "dgr_mesh_create", "dgr_mesh_info_get",
                   "dgr_mesh_export_maps", "dgr_mesh_destroy", "dgr_dof_coords", "dgr_unzip",
                   "dgr_ghost_exchange", "dgr_rhs_patches", "dgr_rhs", "dgr_rk4_stage",
-                  "dgr_rk4_step", "dgr_constraints", "dgr_profile_enable", "dgr_profile_read",
+                  "dgr_rk4_step", "dgr_constraints", "dgr_profile_enable", "dgr_profile_read", "dgr_set_option",
                   "dgr_bench_dfma"]:
             getattr(L, f).restype = i32
         _lib = L
@@ -292,6 +294,11 @@ class Mesh:
 
     def last_launch_count(self):
         return int(lib().dgr_last_launch_count(self._h))
+
+    def set_fused(self, on=True):
+        """DGR_OPT_FUSED_UNZIP: gather patches inside the RHS kernel (1) or unzip into
+        the patch buffer first (0); bit-identical results."""
+        _check(lib().dgr_set_option(self._h, OPT_FUSED_UNZIP, int(bool(on))))
 
     def profile_enable(self, on=True):
         _check(lib().dgr_profile_enable(self._h, int(on)))

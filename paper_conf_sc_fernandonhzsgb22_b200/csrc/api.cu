@@ -99,8 +99,12 @@ struct dgr_mesh_s {
   int4* d_hang = nullptr;
   std::vector<int64_t> hang_level_off;  // row offsets per level group
   int64_t* d_dof_node = nullptr;
-  double* d_E = nullptr;        // [24][n_local][343]
-  double* d_patch = nullptr;    // [24][n_owned][PATCH_PITCH]
+  double* d_E = nullptr;        // [24][e_stride]: n_local*343 element values | n_interp slots
+  int32_t* d_gmap = nullptr;    // [n_owned][GM_PITCH] fused-unzip gather map
+  int4* d_iel = nullptr;        // interpolation work per coarse source element
+  uint16_t* d_ipt = nullptr;    // half-grid point of each interpolation slot
+  int64_t n_interp = 0;
+  double* d_patch = nullptr;    // [24][n_owned][PATCH_PITCH] (allocated on first dgr_unzip)
   double* d_rhs_oct = nullptr;  // [24][n_owned][343]
   double* d_us = nullptr;       // RK4 stage state [24][dof_stride]
   double* d_acc = nullptr;      // RK4 accumulator
@@ -111,6 +115,7 @@ struct dgr_mesh_s {
   double* d_sendbuf = nullptr;
   double* d_recvbuf = nullptr;
   int64_t launches = 0;
+  bool fused = false;           // DGR_OPT_FUSED_UNZIP (two-pass measured faster on C3)
   // profiling
   bool prof = false;
   struct Pend { int cls; cudaEvent_t a, b; };
@@ -276,19 +281,114 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
   }
   CUDA_TRY(m->alloc(&m->d_dof_node, node.size()));
   CUDA_TRY(cudaMemcpy(m->d_dof_node, node.data(), node.size() * 8, cudaMemcpyHostToDevice));
+  // patch gather map: patch point p of owned octant e reads
+  // SRC_f[gmap[e][p]] — the element value it copies/injects (same formula as
+  // the device setup of the former per-patch unzip), an interpolation slot, or
+  // -1 (extrapolated).  Interpolation slots are deduplicated: one per distinct
+  // (coarse source element, half-grid point t2), numbered element-major in
+  // ascending (element, t2z, t2y, t2x) order; k_interp fills them.
+  int64_t e_stride = 0;
+  {
+    const int64_t nle = nl * NPT;
+    std::vector<int32_t> cid(size_t(nl), -1);        // coarse source element -> need table
+    std::vector<std::vector<int32_t>> need;          // [t2x + 13 t2y + 169 t2z] -> slot (or -2)
+    std::vector<int32_t> celem;
+    auto each_interp = [&](auto&& fn) {
+      for (int64_t e = 0; e < no; ++e) {
+        const uint8_t* pm = h.pmap.data() + size_t(e) * PMAP_PITCH;
+        const NbrEntry* nb = h.nbr.data() + size_t(e) * NBR_MAX;
+        for (int p = 0; p < NPATCH; ++p) {
+          const int j = pm[p];
+          if (j == PM_SELF || j == PM_EXTRAP || nb[j].r != 1) continue;
+          const NbrEntry& t = nb[j];
+          const int ix = p % 13, iy = (p / 13) % 13, iz = p / 169;
+          const int tx = t.o[0] + ix, ty = t.o[1] + iy, tz = t.o[2] + iz;
+          if (tx < 0 || tx > 12 || ty < 0 || ty > 12 || tz < 0 || tz > 12) return false;
+          fn(e, p, t.src, tx + 13 * ty + 169 * tz);
+        }
+      }
+      return true;
+    };
+    bool ok = each_interp([&](int64_t, int, int32_t c, int q) {
+      if (cid[c] < 0) {
+        cid[c] = int32_t(need.size());
+        need.emplace_back(NPATCH, -1);
+        celem.push_back(c);
+      }
+      need[cid[c]][q] = -2;
+    });
+    if (!ok) return fail(DGR_ERR_TREE, "interpolation point outside its source element");
+    std::vector<int32_t> order(celem.size());
+    for (size_t i = 0; i < order.size(); ++i) order[i] = int32_t(i);
+    std::sort(order.begin(), order.end(), [&](int32_t a, int32_t b) { return celem[a] < celem[b]; });
+    std::vector<int4> iel;
+    std::vector<uint16_t> ipt;
+    int64_t slot = 0;
+    for (int32_t ci : order) {
+      int lo[3] = {12, 12, 12}, hi[3] = {0, 0, 0};
+      const int64_t first = slot;
+      for (int q = 0; q < NPATCH; ++q) {
+        if (need[ci][q] != -2) continue;
+        const int t[3] = {q % 13, (q / 13) % 13, q / 169};
+        for (int k = 0; k < 3; ++k) {
+          lo[k] = std::min(lo[k], t[k]);
+          hi[k] = std::max(hi[k], t[k]);
+        }
+        need[ci][q] = int32_t(slot++);
+        ipt.push_back(uint16_t(t[0] | (t[1] << 4) | (t[2] << 8)));
+      }
+      const int lohi = (lo[0] | (lo[1] << 4) | (lo[2] << 8)) | ((hi[0] | (hi[1] << 4) | (hi[2] << 8)) << 12);
+      iel.push_back(make_int4(celem[ci], int32_t(first), int32_t(slot - first), lohi));
+    }
+    if (nle + slot >= (int64_t(1) << 31)) return fail(DGR_ERR_ARG, "mesh too large for int32 gather map");
+    std::vector<int32_t> gm(size_t(no) * GM_PITCH, -1);
+    for (int64_t e = 0; e < no; ++e) {
+      const uint8_t* pm = h.pmap.data() + size_t(e) * PMAP_PITCH;
+      const NbrEntry* nb = h.nbr.data() + size_t(e) * NBR_MAX;
+      for (int p = 0; p < NPATCH; ++p) {
+        const int j = pm[p];
+        const int ix = p % 13, iy = (p / 13) % 13, iz = p / 169;
+        int64_t v = -1;
+        if (j == PM_SELF) {
+          v = e * NPT + (ix - 3) + 7 * (iy - 3) + 49 * (iz - 3);
+        } else if (j != PM_EXTRAP) {
+          const NbrEntry& t = nb[j];
+          if (t.r == 1) {
+            const int q = (t.o[0] + ix) + 13 * (t.o[1] + iy) + 169 * (t.o[2] + iz);
+            v = nle + need[cid[t.src]][q];
+          } else {
+            const int tx = (t.o[0] + t.r * ix) >> 1, ty = (t.o[1] + t.r * iy) >> 1,
+                      tz = (t.o[2] + t.r * iz) >> 1;
+            v = int64_t(t.src) * NPT + tx + 7 * ty + 49 * tz;
+          }
+        }
+        gm[size_t(e) * GM_PITCH + p] = int32_t(v);
+      }
+    }
+    m->n_interp = slot;
+    e_stride = ((nle + slot + 31) / 32) * 32;
+    CUDA_TRY(m->alloc(&m->d_gmap, gm.size()));
+    CUDA_TRY(cudaMemcpy(m->d_gmap, gm.data(), gm.size() * 4, cudaMemcpyHostToDevice));
+    CUDA_TRY(m->alloc(&m->d_iel, iel.size()));
+    if (!iel.empty())
+      CUDA_TRY(cudaMemcpy(m->d_iel, iel.data(), iel.size() * sizeof(int4), cudaMemcpyHostToDevice));
+    CUDA_TRY(m->alloc(&m->d_ipt, ipt.size()));
+    if (!ipt.empty())
+      CUDA_TRY(cudaMemcpy(m->d_ipt, ipt.data(), ipt.size() * 2, cudaMemcpyHostToDevice));
+    m->dm.n_iel = int32_t(iel.size());
+  }
   // workspace
-  CUDA_TRY(m->alloc(&m->d_E, size_t(NF) * nl * NPT));
-  CUDA_TRY(m->alloc(&m->d_patch, size_t(NF) * no * PATCH_PITCH));
+  CUDA_TRY(m->alloc(&m->d_E, size_t(NF) * e_stride));
   CUDA_TRY(m->alloc(&m->d_rhs_oct, size_t(NF) * no * NPT));
   CUDA_TRY(m->alloc(&m->d_us, size_t(NF) * stride));
   CUDA_TRY(m->alloc(&m->d_acc, size_t(NF) * stride));
-  CUDA_TRY(cudaMemset(m->d_patch, 0, size_t(NF) * no * PATCH_PITCH * 8));
+  CUDA_TRY(cudaMemset(m->d_E, 0, size_t(NF) * e_stride * 8));
   CUDA_TRY(cudaMemset(m->d_us, 0, size_t(NF) * stride * 8));
   CUDA_TRY(cudaMemset(m->d_acc, 0, size_t(NF) * stride * 8));
   double w13[91], wext[21];
   lagrange_tables(w13, wext);
   upload_tables(w13, wext);
-  upload_rhs_tables();
+  upload_rhs_tables(wext);
   CUDA_TRY(cudaGetLastError());
   DevMesh& dm = m->dm;
   dm.n_owned = int32_t(no);
@@ -304,6 +404,10 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
   dm.nbr = m->d_nbr;
   dm.zip = m->d_zip;
   dm.hang = m->d_hang;
+  dm.e_stride = e_stride;
+  dm.gmap = m->d_gmap;
+  dm.iel = m->d_iel;
+  dm.ipt = m->d_ipt;
   // multi-rank buffers
   if (h.nranks > 1) {
     CUDA_TRY(m->alloc(&m->d_send, h.send_list.size()));
@@ -513,13 +617,36 @@ static dgr_status exchange(dgr_mesh m, double* u, cudaStream_t st) {
   return DGR_OK;
 }
 
-static dgr_status do_unzip(dgr_mesh m, const double* u, int nf, cudaStream_t st) {
+// element reconstruction (Alg. 2 lines 2-5): E from u, hanging nodes level by level
+static dgr_status do_elements(dgr_mesh m, const double* u, int nf, cudaStream_t st) {
   PROF(m, 0, st, launch_elements(m->dm, u, m->d_E, nf, st));
   for (size_t g = 0; g + 1 < m->hang_level_off.size(); ++g) {
     const int64_t a = m->hang_level_off[g], b = m->hang_level_off[g + 1];
     PROF(m, 1, st, launch_hanging(m->dm, m->d_hang + a, b - a, m->d_E, nf, st));
   }
+  CUDA_TRY(cudaGetLastError());
+  return DGR_OK;
+}
+
+// explicit unzip into the patch buffer (dgr_unzip, constraints)
+static dgr_status do_unzip(dgr_mesh m, const double* u, int nf, cudaStream_t st) {
+  if (!m->d_patch) {
+    CUDA_TRY(m->alloc(&m->d_patch, size_t(NF) * m->dm.n_owned * PATCH_PITCH));
+    CUDA_TRY(cudaMemsetAsync(m->d_patch, 0, size_t(NF) * m->dm.n_owned * PATCH_PITCH * 8, st));
+  }
+  dgr_status s = do_elements(m, u, nf, st);
+  if (s) return s;
+  PROF(m, 7, st, launch_interp(m->dm, m->d_E, nf, st));
   PROF(m, 2, st, launch_unzip(m->dm, m->d_E, m->d_patch, nf, st));
+  CUDA_TRY(cudaGetLastError());
+  return DGR_OK;
+}
+
+// fused path: elements + coarse-neighbour interpolation slots; k_rhs<true> gathers the patches
+static dgr_status do_fused_sources(dgr_mesh m, const double* u, cudaStream_t st) {
+  dgr_status s = do_elements(m, u, NF, st);
+  if (s) return s;
+  PROF(m, 7, st, launch_interp(m->dm, m->d_E, NF, st));
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;
 }
@@ -528,6 +655,21 @@ static RhsParams to_rp(const dgr_params* p) {
   RhsParams r{0.4, 2.0, 1.0, 0.0, 1e-4};
   if (p) r = {p->ko_sigma, p->eta, p->lambda_f0, p->lambda_f1, p->chi_floor};
   return r;
+}
+
+// RHS of every owned octant's interior points into d_rhs_oct, by the fused
+// path (patches gathered inside k_rhs) or through the explicit patch buffer
+static dgr_status rhs_oct(dgr_mesh m, const double* u, const dgr_params* prm, cudaStream_t st) {
+  dgr_status s;
+  if (m->fused) {
+    if ((s = do_fused_sources(m, u, st))) return s;
+    PROF(m, 3, st, launch_rhs(m->dm, m->d_E, m->d_rhs_oct, to_rp(prm), nullptr, true, st));
+  } else {
+    if ((s = do_unzip(m, u, NF, st))) return s;
+    PROF(m, 3, st, launch_rhs(m->dm, m->d_patch, m->d_rhs_oct, to_rp(prm), nullptr, false, st));
+  }
+  CUDA_TRY(cudaGetLastError());
+  return DGR_OK;
 }
 
 extern "C" {
@@ -569,7 +711,7 @@ dgr_status dgr_rhs_patches(dgr_mesh m, const double* patches, double* rhs_oct,
   if (s) return s;
   if (!patches || !rhs_oct || !aligned16(patches)) return fail(DGR_ERR_ARG, "bad rhs args");
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  PROF(m, 3, st, launch_rhs(m->dm, patches, rhs_oct, to_rp(prm), nullptr, st));
+  PROF(m, 3, st, launch_rhs(m->dm, patches, rhs_oct, to_rp(prm), nullptr, false, st));
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;
 }
@@ -581,8 +723,7 @@ dgr_status dgr_rhs(dgr_mesh m, double* u, double* rhs, const dgr_params* prm, vo
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   m->launches = 0;
   if ((s = exchange(m, u, st))) return s;
-  if ((s = do_unzip(m, u, NF, st))) return s;
-  PROF(m, 3, st, launch_rhs(m->dm, m->d_patch, m->d_rhs_oct, to_rp(prm), nullptr, st));
+  if ((s = rhs_oct(m, u, prm, st))) return s;
   PROF(m, 4, st, launch_zip(m->dm, m->d_rhs_oct, rhs, NF, st));
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;
@@ -593,11 +734,10 @@ static dgr_status stage(dgr_mesh m, int s_, double dt, double* u_n, double* u_s,
   dgr_status s;
   double* cur = s_ == 0 ? u_n : u_s;
   if ((s = exchange(m, cur, st))) return s;
-  if ((s = do_unzip(m, cur, NF, st))) return s;
   // (k_rhs can also apply the zip + RK4 update in its epilogue (RkArgs); on C3
   // that measured 10.6 ms vs 7.5 + 0.8 ms for RHS + k_zip_rk4 — the scattered
   // state loads stall the single persistent CTA per SM — so it is not used)
-  PROF(m, 3, st, launch_rhs(m->dm, m->d_patch, m->d_rhs_oct, to_rp(prm), nullptr, st));
+  if ((s = rhs_oct(m, cur, prm, st))) return s;
   PROF(m, 4, st, launch_zip_rk4(m->dm, m->d_rhs_oct, s_, dt, u_n, u_s, acc, u_out, st));
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;
@@ -683,6 +823,14 @@ dgr_status dgr_constraints(dgr_mesh m, double* u, double* c, double* norms_host,
     }
   }
   return DGR_OK;
+}
+
+dgr_status dgr_set_option(dgr_mesh m, int option, int64_t value) {
+  if (!m) return fail(DGR_ERR_ARG, "null mesh");
+  switch (option) {
+    case DGR_OPT_FUSED_UNZIP: m->fused = value != 0; return DGR_OK;
+  }
+  return fail(DGR_ERR_ARG, "unknown option");
 }
 
 dgr_status dgr_profile_enable(dgr_mesh m, int on) {

@@ -57,10 +57,11 @@ __device__ __forceinline__ double interp_point(const double* __restrict__ Ec, in
 // E[f][e][n] = u[f][O2N[e][n]] for DOF nodes (Alg. 2 line 2); hanging nodes
 // are filled level by level by k_hanging.
 __global__ void k_elements(const double* __restrict__ u, int64_t stride,
-                           const int32_t* __restrict__ o2n, int64_t nn, double* __restrict__ E) {
+                           const int32_t* __restrict__ o2n, int64_t nn, int64_t es,
+                           double* __restrict__ E) {
   const int f = blockIdx.y;
   const double* uf = u + f * stride;
-  double* Ef = E + f * nn;
+  double* Ef = E + f * es;
   for (int64_t i = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; i < nn;
        i += int64_t(gridDim.x) * blockDim.x) {
     const int32_t id = __ldg(o2n + i);
@@ -72,7 +73,7 @@ void launch_elements(const DevMesh& m, const double* u, double* E, int nf, cudaS
   const int64_t nn = int64_t(m.n_local) * NPT;
   int blocks = int((nn + 255) / 256);
   if (blocks > 148 * 16) blocks = 148 * 16;
-  k_elements<<<dim3(blocks, nf), 256, 0, s>>>(u, m.dof_stride, m.o2n, nn, E);
+  k_elements<<<dim3(blocks, nf), 256, 0, s>>>(u, m.dof_stride, m.o2n, nn, m.e_stride, E);
 }
 
 // --------------------------------------------------------- hanging points
@@ -132,7 +133,7 @@ void launch_hanging(const DevMesh& m, const int4* rows, int64_t count, double* E
   int blocks = int((count + 127) / 128);
   if (blocks > 148 * 16) blocks = 148 * 16;
   k_hanging<<<dim3(blocks, (nf + HANG_FG - 1) / HANG_FG), 128, 0, s>>>(
-      rows, count, E, int64_t(m.n_local) * NPT, nf);
+      rows, count, E, m.e_stride, nf);
 }
 
 // (octant-to-patch: unzip_kernel.cu)

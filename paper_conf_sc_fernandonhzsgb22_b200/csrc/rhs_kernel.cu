@@ -46,8 +46,8 @@ constexpr int NSLOT = 57;
 // index c = x + 13y + 169z minus an offset so thread reads stay conflict-free
 constexpr int TX_OFF = 3, TX_N = 2191;    // x in 3..9, y, z in 0..12
 constexpr int TY_OFF = 42, TY_N = 2113;   // x, y in 3..9, z in 0..12
-constexpr size_t SMEM_BYTES =
-    size_t(NSLOT) * NPP * 8 + size_t(2) * STAGE_DBL * 8 + size_t(TX_N + TY_N) * 8 + 16;
+constexpr size_t SMEM_BYTES = size_t(NSLOT) * NPP * 8 + size_t(2) * STAGE_DBL * 8 +
+                              size_t(TX_N + TY_N) * 8 + 16 + size_t(2) * RT * 2;
 
 // thread -> interior point map (filled by upload_rhs_tables): every warp holds
 // at most two points per residue of their stage-buffer index mod 16, so its
@@ -61,11 +61,22 @@ __device__ long long g_stage_cycles[NF + 2];
 
 // Items of the cooperative D1 pass: Tx on the cross-shaped region the mixed
 // stencils read (x interior; y all with z interior, or z all with y interior),
-// Ty on x, y interior with all z; each entry is the patch index c.  Tx items
-// run along rows (y + 13 z) at fixed x so a warp's addresses have distinct
-// residues mod 16 (13 is a unit mod 16); Ty items along z (169 is a unit).
+// Ty on x, y interior with all z.  titem(k) is the patch index c of item k:
+// Tx items run along rows (y + 13 z) at fixed x so a warp's addresses have
+// distinct residues mod 16 (13 is a unit mod 16); Ty items along z (169 is a
+// unit).  (Computed, not tabulated: a table load misses L1 when the fused
+// gather streams through it.)
 constexpr int N_TX = 7 * (13 * 7 + 7 * 6), N_TY = 7 * 7 * 13, N_TITEM = N_TX + N_TY;
-__device__ int16_t g_titem[N_TITEM];
+__device__ __forceinline__ int titem(int k) {
+  if (k < N_TX) {
+    const int x = 3 + k / 133, r = k % 133;
+    if (r < 91) return x + 13 * (39 + r);            // z in 3..9, all y
+    const int r2 = r - 91, zz = r2 / 7;              // z in {0,1,2,10,11,12}, y in 3..9
+    return x + 13 * (3 + r2 % 7) + 169 * (zz < 3 ? zz : zz + 7);
+  }
+  const int k2 = k - N_TX, xy = k2 / 13;
+  return (3 + xy / 7) + 13 * (3 + xy % 7) + 169 * (k2 % 13);
+}
 
 // field processing order
 __constant__ int c_order[NF] = {12, 13, 14, 15, 16, 17, 1, 0, 3, 4, 5, 6,
@@ -96,6 +107,27 @@ __device__ __forceinline__ void bulk_load(double* dst, const double* src, uint32
       "l"(src), "r"(bytes), "r"(smem_u32(bar))
       : "memory");
 }
+
+// 8-byte asynchronous global->shared copy of src[idx] (the fused unzip's
+// gather); the address arithmetic stays inside the asm so the compiler cannot
+// rematerialise the field base per copy
+__device__ __forceinline__ void cp_async8(uint32_t dst, const double* src, int32_t idx) {
+  asm volatile(
+      "{\n .reg .u64 a;\n mad.wide.s32 a, %2, 8, %1;\n"
+      " cp.async.ca.shared.global [%0], [a], 8;\n}\n" ::"r"(dst),
+      "l"(src), "r"(idx)
+      : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() {
+  asm volatile("cp.async.commit_group;" ::: "memory");
+}
+__device__ __forceinline__ void cp_async_wait1() {
+  asm volatile("cp.async.wait_group 1;" ::: "memory");
+}
+
+// extrapolation rows l_m(-(t+1)), t = 0..2 (reading R12; host-computed, api.cu)
+__constant__ double c_rWEXT[3 * 7];
+constexpr int GJ = (NPATCH + RT - 1) / RT;   // gather points per thread (7)
 
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   uint32_t ok = 0;
@@ -206,6 +238,14 @@ __device__ __forceinline__ double trace6(const double* gi, const double* X) {
 
 }  // namespace
 
+// FUSED = false: `patches` is the 13^3 patch buffer [24][n_owned][PATCH_PITCH]
+// (bulk copies).  FUSED = true: `patches` is E (DevMesh::e_stride per field) and
+// every patch is gathered straight from it through m.gmap with 8-byte cp.async
+// (the unzip fused into the RHS): copy/injection points read
+// element values, coarse-neighbour points read the slots k_interp filled, and
+// points outside a non-periodic domain are extrapolated in shared memory with
+// the same arithmetic as k_unzip.
+template <bool FUSED>
 __global__ void __launch_bounds__(RT, 1)
     k_rhs(DevMesh m, const double* __restrict__ patches, double* __restrict__ rhs_oct,
           RhsParams prm, RkArgs rk) {
@@ -215,15 +255,37 @@ __global__ void __launch_bounds__(RT, 1)
   double* Tx = stage + 2 * STAGE_DBL;             // [TX_N]
   double* Ty = Tx + TX_N;                         // [TY_N]
   uint64_t* bars = reinterpret_cast<uint64_t*>(Ty + TY_N);
+  // this thread's point: patch index c0 (-1: no point) and interior index p, kept
+  // in shared memory and re-read where needed (cheaper than a register spill)
+  int16_t* tab_c0 = reinterpret_cast<int16_t*>(bars + 2);
+  int16_t* tab_p = tab_c0 + RT;
 
   const int tid = threadIdx.x;
-  const int pp = g_perm[tid];
-  const bool active = pp >= 0;
-  const int p = active ? pp : 0;
-  const int pi = p % 7, pj = (p / 7) % 7, pk = p / 49;
-  const int c0 = (pi + 3) + 13 * (pj + 3) + 169 * (pk + 3);
+  {
+    const int pp = g_perm[tid];
+    const int q = pp >= 0 ? pp : 0;
+    tab_c0[tid] = pp >= 0 ? int16_t((q % 7 + 3) + 13 * ((q / 7) % 7 + 3) + 169 * (q / 49 + 3)) : -1;
+    tab_p[tid] = int16_t(q);
+  }
   const int64_t no = m.n_owned;
-  const int64_t fstride = no * PATCH_PITCH;
+  const int64_t fstride = FUSED ? m.e_stride : no * PATCH_PITCH;
+  int gidx[GJ];   // FUSED: SRC index of patch points tid + RT*j of the current octant
+  auto load_gidx = [&](int oct) {
+    const int32_t* gm = m.gmap + int64_t(oct) * GM_PITCH;
+#pragma unroll
+    for (int j = 0; j < GJ; ++j) {
+      const int pt = tid + RT * j;
+      // (extrapolated points, -1, copy a dummy value and are overwritten later)
+      gidx[j] = pt < NPATCH ? max(__ldg(gm + pt), 0) : -1;
+    }
+  };
+  auto gather = [&](double* dst, const double* srcf) {
+    const uint32_t d0 = smem_u32(dst + tid);
+#pragma unroll
+    for (int j = 0; j < GJ - 1; ++j) cp_async8(d0 + 8 * RT * j, srcf, gidx[j]);
+    if (tid + RT * (GJ - 1) < NPATCH) cp_async8(d0 + 8 * RT * (GJ - 1), srcf, gidx[GJ - 1]);
+    cp_async_commit();
+  };
 #define SL(slot) slots[(slot) * NPP + tid]
   auto prefetch_l2 = [&](const double* src) {
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src),
@@ -242,7 +304,11 @@ __global__ void __launch_bounds__(RT, 1)
     mbar_init(&bars[1], 1);
   }
   __syncthreads();
-  if (tid == 0) {
+  if (FUSED) {
+    load_gidx(e);
+    gather(stage, patches + c_order[0] * fstride);
+    gather(stage + STAGE_DBL, patches + c_order[1] * fstride);
+  } else if (tid == 0) {
     const double* pb = patches + int64_t(e) * PATCH_PITCH;
     bulk_load(stage, pb + c_order[0] * fstride, STAGE_DBL * 8, &bars[0]);
     bulk_load(stage + STAGE_DBL, pb + c_order[1] * fstride, STAGE_DBL * 8, &bars[1]);
@@ -252,26 +318,52 @@ __global__ void __launch_bounds__(RT, 1)
   uint32_t g = 0;   // global stage counter of this CTA
   for (; e < no; e += gridDim.x) {
   const int en = e + gridDim.x;                    // next octant of this CTA
-  const double* pbase = patches + int64_t(e) * PATCH_PITCH;
+  const double* pbase = patches + int64_t(e) * (FUSED ? NPT : PATCH_PITCH);
+  const bool active = tab_c0[tid] >= 0;
+  const int cv = FUSED ? tab_p[tid] : tab_c0[tid];   // own value: element node p / patch index c0
 
   const int4 oi = m.oct[e];
+  // FUSED: which faces of this octant lie on a non-periodic domain boundary
+  // (bit a: low face along axis a outside the domain, bit 3 + a: high face)
+  int omask = 0;
+  if (FUSED && !m.periodic) {
+    const int nside = 1 << m.D, sd = 1 << (m.D - oi.w);
+    omask = (oi.x == 0) | ((oi.y == 0) << 1) | ((oi.z == 0) << 2) | ((oi.x + sd == nside) << 3) |
+            ((oi.y + sd == nside) << 4) | ((oi.z + sd == nside) << 5);
+  }
+  const bool bnd = omask != 0;
+  if (FUSED && en < no) {
+    if (tid == 32)   // next octant's gather map into L2
+      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(m.gmap + int64_t(en) * GM_PITCH),
+                   "r"(uint32_t(GM_PITCH * 4))
+                   : "memory");
+    else if (tid >= 64 && tid < 64 + NF) {
+      // ... and its own element values (read at its start and by its first gathers),
+      // 16-B aligned cover of the 343 doubles of field tid - 64
+      const uintptr_t a = reinterpret_cast<uintptr_t>(patches + (tid - 64) * fstride +
+                                                      int64_t(en) * NPT);
+      const uintptr_t a0 = a & ~uintptr_t(15), a1 = (a + NPT * 8 + 15) & ~uintptr_t(15);
+      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a0), "r"(uint32_t(a1 - a0))
+                   : "memory");
+    }
+  }
   const double ih = (6.0 * double(int64_t(1) << oi.w)) / m.width;   // 1/h
   const double ko_scale = prm.ko_sigma * ih * (1.0 / 64.0);
 
   // ---- values at the point (patch interior) -------------------------------
   double alpha = 0, chi = 0, Kv = 0, beta[3] = {0, 0, 0};
   if (active) {
-    alpha = __ldg(pbase + 0 * fstride + c0);
-    chi = __ldg(pbase + 1 * fstride + c0);
-    Kv = __ldg(pbase + 2 * fstride + c0);
+    alpha = __ldg(pbase + 0 * fstride + cv);
+    chi = __ldg(pbase + 1 * fstride + cv);
+    Kv = __ldg(pbase + 2 * fstride + cv);
 #pragma unroll
-    for (int i = 0; i < 3; ++i) beta[i] = __ldg(pbase + (6 + i) * fstride + c0);
+    for (int i = 0; i < 3; ++i) beta[i] = __ldg(pbase + (6 + i) * fstride + cv);
     double g[6];
 #pragma unroll
     for (int q = 0; q < 6; ++q) {
-      g[q] = __ldg(pbase + (12 + q) * fstride + c0);
+      g[q] = __ldg(pbase + (12 + q) * fstride + cv);
       SL(V_GAM + q) = g[q];
-      SL(V_AT + q) = __ldg(pbase + (18 + q) * fstride + c0);
+      SL(V_AT + q) = __ldg(pbase + (18 + q) * fstride + cv);
     }
     // inverse metric by adjugate / determinant
     const double a00 = g[3] * g[5] - g[4] * g[4];
@@ -308,7 +400,47 @@ __global__ void __launch_bounds__(RT, 1)
       t_last = t;
     }
 #endif
-    mbar_wait(&bars[buf], (g >> 1) & 1);
+    if (FUSED) {
+      cp_async_wait1();   // this thread's copies of stage st have landed
+      __syncthreads();    // ... and everyone else's
+      if (bnd) {
+        // outer-boundary extrapolation along x, then y, then z (reading R12),
+        // the arithmetic of k_unzip, in shared memory
+        double* sw = stage + buf * STAGE_DBL;
+        for (int a = 0; a < 3; ++a) {
+          const int sa = a == 0 ? 1 : (a == 1 ? 13 : 169);
+          const int sb = a == 0 ? 13 : 1, sc = a == 2 ? 13 : 169;
+          const int b_ax = a == 0 ? 1 : 0, c_ax = a == 2 ? 1 : 2;
+          for (int side = 0; side < 2; ++side) {
+            if (!((omask >> (a + 3 * side)) & 1)) continue;
+            for (int idx = tid; idx < 3 * 169; idx += RT) {
+              const int k3 = idx % 3, uv = idx / 3;
+              const int cb = uv % 13, cc = uv / 13;
+              if (b_ax > a && ((cb < 3 && ((omask >> b_ax) & 1)) || (cb > 9 && ((omask >> (3 + b_ax)) & 1))))
+                continue;
+              if (c_ax > a && ((cc < 3 && ((omask >> c_ax) & 1)) || (cc > 9 && ((omask >> (3 + c_ax)) & 1))))
+                continue;
+              const int ia = side == 0 ? k3 : 10 + k3;
+              const int base = cb * sb + cc * sc;
+              double acc = 0.0;
+              if (side == 0) {
+                const double* w = c_rWEXT + (2 - ia) * 7;
+#pragma unroll
+                for (int mm = 0; mm < 7; ++mm) acc = fma(w[mm], sw[base + (3 + mm) * sa], acc);
+              } else {
+                const double* w = c_rWEXT + (ia - 10) * 7;
+#pragma unroll
+                for (int mm = 0; mm < 7; ++mm) acc = fma(w[mm], sw[base + (9 - mm) * sa], acc);
+              }
+              sw[base + ia * sa] = acc;
+            }
+          }
+          __syncthreads();
+        }
+      }
+    } else {
+      mbar_wait(&bars[buf], (g >> 1) & 1);
+    }
     const double* s = stage + buf * STAGE_DBL;
     const int f = c_order[st];
     const bool second = f <= 1 || (f >= 6 && f <= 8) || (f >= 12 && f <= 17);
@@ -320,7 +452,7 @@ __global__ void __launch_bounds__(RT, 1)
       // (y + 13 z) at fixed x (13 == -3 is a unit mod 16), Ty items along z at
       // fixed (x, y) (169 == 9 is a unit mod 16)
       for (int k = tid; k < N_TITEM; k += RT) {
-        const int c = __ldg(g_titem + k);          // patch index of the item (table)
+        const int c = titem(k);                    // patch index of the item
         if (k < N_TX) {
           Tx[c - TX_OFF] = (s[c + 1] - s[c - 1]) * 45.0 - (s[c + 2] - s[c - 2]) * 9.0 +
                            (s[c + 3] - s[c - 3]);
@@ -331,7 +463,8 @@ __global__ void __launch_bounds__(RT, 1)
       }
       __syncthreads();
     }
-    if (active) {
+    const int c0 = tab_c0[tid];
+    if (c0 >= 0) {
       if (f >= 12 && f <= 17) {
         // ---------------- conformal metric gt_q: d gt, gt^lm d_lm gt, adv, KO
         const int q = f - 12;
@@ -613,6 +746,17 @@ __global__ void __launch_bounds__(RT, 1)
       }
     }
     __syncthreads();  // everyone is done with this stage buffer
+    if (FUSED) {
+      double* dst = stage + buf * STAGE_DBL;
+      if (st + 2 < NF) {
+        gather(dst, patches + c_order[st + 2] * fstride);
+      } else {
+        if (st + 2 == NF && en < no) load_gidx(en);   // the current octant's gathers are issued
+        if (en < no) gather(dst, patches + c_order[st + 2 - NF] * fstride);
+        else cp_async_commit();                        // (empty group keeps the count uniform)
+      }
+      continue;
+    }
     // L2 prefetch one octant ahead: the next octant's field of this stage
     // (measured faster than prefetching the current octant at its start,
     // although some prefetched lines are evicted and re-read)
@@ -638,15 +782,17 @@ __global__ void __launch_bounds__(RT, 1)
   }
 #endif
   // ---- epilogue: undifferentiated terms, combine, store ----------------------
-  if (active) {
+  const int p = tab_p[tid];
+  if (tab_c0[tid] >= 0) {
     double gi[6], At[6], B[3];
 #pragma unroll
     for (int r = 0; r < 6; ++r) {
       gi[r] = SL(G_INV + r);
       At[r] = SL(V_AT + r);
     }
+    const int cb = FUSED ? p : tab_c0[tid];
 #pragma unroll
-    for (int i = 0; i < 3; ++i) B[i] = __ldg(pbase + (9 + i) * fstride + c0);
+    for (int i = 0; i < 3; ++i) B[i] = __ldg(pbase + (9 + i) * fstride + cb);
     // At^k_j and At_ik At^k_j, At_ij At^ij
     double Am[3][3];
 #pragma unroll
@@ -734,7 +880,8 @@ extern "C" int dgr_debug_rhs_stage_cycles(long long* out) {
 namespace dgr {
 #endif
 
-void upload_rhs_tables() {
+void upload_rhs_tables(const double* wext) {
+  cudaMemcpyToSymbol(c_rWEXT, wext, sizeof(double) * 21);
   int16_t perm[RT];
   std::vector<int> bucket[16];
   for (int p = 0; p < NPT; ++p) {
@@ -749,27 +896,15 @@ void upload_rhs_tables() {
       if (next[r] < bucket[r].size()) perm[w * 32 + lane] = int16_t(bucket[r][next[r]++]);
     }
   cudaMemcpyToSymbol(g_perm, perm, sizeof(perm));
-  // cooperative-D1 item table
-  std::vector<int16_t> items;
-  for (int x = 3; x <= 9; ++x)
-    for (int row = 0; row < 169; ++row) {
-      const int y = row % 13, z = row / 13;
-      const bool yin = y >= 3 && y <= 9, zin = z >= 3 && z <= 9;
-      if (zin || yin) items.push_back(int16_t(x + 13 * row));
-    }
-  for (int x = 3; x <= 9; ++x)
-    for (int y = 3; y <= 9; ++y)
-      for (int z = 0; z < 13; ++z) items.push_back(int16_t(x + 13 * y + 169 * z));
-  if (int(items.size()) == N_TITEM)
-    cudaMemcpyToSymbol(g_titem, items.data(), items.size() * sizeof(int16_t));
 }
 
 void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const RhsParams& p,
-                const RkArgs* rk, cudaStream_t s) {
+                const RkArgs* rk, bool fused, cudaStream_t s) {
   if (m.n_owned <= 0) return;
   static int n_sm = 0;
   if (!n_sm) {
-    cudaFuncSetAttribute(k_rhs, cudaFuncAttributeMaxDynamicSharedMemorySize, int(SMEM_BYTES));
+    cudaFuncSetAttribute(k_rhs<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(SMEM_BYTES));
+    cudaFuncSetAttribute(k_rhs<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(SMEM_BYTES));
     int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&n_sm, cudaDevAttrMultiProcessorCount, dev);
@@ -780,7 +915,10 @@ void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const 
   RkArgs a{};
   a.s = -1;
   if (rk) a = *rk;
-  k_rhs<<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a);
+  if (fused)
+    k_rhs<true><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a);
+  else
+    k_rhs<false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a);
 }
 
 }  // namespace dgr

@@ -7,7 +7,9 @@ from synth import configs, initial
 name = sys.argv[1] if len(sys.argv) > 1 else "c3"
 steps = int(sys.argv[2]) if len(sys.argv) > 2 else 5
 cfg = configs.get(name)
-t = time.time(); m = dgr.Mesh(cfg); print("mesh", m.info, "%.1fs" % (time.time() - t), flush=True)
+fused = os.environ.get("DGR_FUSED", "0") != "0"
+t = time.time(); m = dgr.Mesh(cfg); m.set_fused(fused); print("fused", fused)
+print("mesh", m.info, "%.1fs" % (time.time() - t), flush=True)
 xyz = m.dof_xyz_host()
 u = torch.zeros((24, m.dof_stride), dtype=torch.float64, device="cuda")
 u[:, :xyz.shape[1]] = torch.from_numpy(initial.for_config(cfg, xyz))
@@ -26,4 +28,9 @@ e0.record()
 for _ in range(steps): m.rhs(u, out=r)
 e1.record(); torch.cuda.synchronize()
 print(f"{name}: rhs (unzip+rhs+zip) {e0.elapsed_time(e1)/steps:.3f} ms")
+m.profile_read(reset=True); m.profile_enable(True)
+for _ in range(2): m.rk4_step(u, dt)
+torch.cuda.synchronize(); m.profile_enable(False)
+for k, (t, n) in m.profile_read(reset=True).items():
+    print(f"  {k:12s} {t/n:8.3f} ms/launch  {n:4d} launches  {t/2:8.3f} ms/step")
 print("finite:", bool(torch.isfinite(u[:, :n]).all()))

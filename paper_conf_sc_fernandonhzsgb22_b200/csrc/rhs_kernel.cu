@@ -59,24 +59,9 @@ __device__ int16_t g_perm[RT];
 __device__ long long g_stage_cycles[NF + 2];
 #endif
 
-// Items of the cooperative D1 pass: Tx on the cross-shaped region the mixed
-// stencils read (x interior; y all with z interior, or z all with y interior),
-// Ty on x, y interior with all z.  titem(k) is the patch index c of item k:
-// Tx items run along rows (y + 13 z) at fixed x so a warp's addresses have
-// distinct residues mod 16 (13 is a unit mod 16); Ty items along z (169 is a
-// unit).  (Computed, not tabulated: a table load misses L1 when the fused
-// gather streams through it.)
-constexpr int N_TX = 7 * (13 * 7 + 7 * 6), N_TY = 7 * 7 * 13, N_TITEM = N_TX + N_TY;
-__device__ __forceinline__ int titem(int k) {
-  if (k < N_TX) {
-    const int x = 3 + k / 133, r = k % 133;
-    if (r < 91) return x + 13 * (39 + r);            // z in 3..9, all y
-    const int r2 = r - 91, zz = r2 / 7;              // z in {0,1,2,10,11,12}, y in 3..9
-    return x + 13 * (3 + r2 % 7) + 169 * (zz < 3 ? zz : zz + 7);
-  }
-  const int k2 = k - N_TX, xy = k2 / 13;
-  return (3 + xy / 7) + 13 * (3 + xy % 7) + 169 * (k2 % 13);
-}
+// Lines of the cooperative D1 pass (register pencils, see the stage loop)
+constexpr int N_TXL = 13 * 7 + 7 * 6, N_TYL = 7 * 13;
+static_assert(N_TXL + N_TYL <= RT, "one pencil per thread");
 
 // field processing order
 __constant__ int c_order[NF] = {12, 13, 14, 15, 16, 17, 1, 0, 3, 4, 5, 6,
@@ -446,20 +431,42 @@ __global__ void __launch_bounds__(RT, 1)
     const bool second = f <= 1 || (f >= 6 && f <= 8) || (f >= 12 && f <= 17);
     if (second) {
       // cooperative first derivatives along x (and y) of the staged field on
-      // the extended region the mixed stencils need (each value once, instead
-      // of 36 loads per mixed derivative per point)
-      // item order keeps warps bank-conflict-free: Tx items run along rows
-      // (y + 13 z) at fixed x (13 == -3 is a unit mod 16), Ty items along z at
-      // fixed (x, y) (169 == 9 is a unit mod 16)
-      for (int k = tid; k < N_TITEM; k += RT) {
-        const int c = titem(k);                    // patch index of the item
-        if (k < N_TX) {
-          Tx[c - TX_OFF] = (s[c + 1] - s[c - 1]) * 45.0 - (s[c + 2] - s[c - 2]) * 9.0 +
-                           (s[c + 3] - s[c - 3]);
+      // the extended region the mixed stencils need, by register pencils: each
+      // thread loads one 13-point line once and writes D1 at its 7 interior
+      // points (20 shared-memory accesses per 7 values instead of 49).
+      // Tx: lines along x at the 133 (y, z) rows of the cross-shaped region
+      // (z in 3..9 with all y, or y in 3..9 with z in {0,1,2,10,11,12});
+      // Ty: lines along y at x in 3..9, all z.  Consecutive lanes take rows
+      // 13 apart (Tx) or consecutive x (Ty), so loads and stores stay within
+      // two wavefronts per warp.
+      if (tid < N_TXL) {
+        int y, z;
+        if (tid < 91) {
+          z = 3 + tid / 13;
+          y = tid % 13;
         } else {
-          Ty[c - TY_OFF] = (s[c + 13] - s[c - 13]) * 45.0 - (s[c + 26] - s[c - 26]) * 9.0 +
-                           (s[c + 39] - s[c - 39]);
+          const int r2 = tid - 91, zz = r2 / 7;
+          z = zz < 3 ? zz : zz + 7;
+          y = 3 + r2 % 7;
         }
+        const int b = 13 * y + 169 * z;
+        double v[13];
+#pragma unroll
+        for (int k = 0; k < 13; ++k) v[k] = s[b + k];
+#pragma unroll
+        for (int x = 3; x <= 9; ++x)
+          Tx[b + x - TX_OFF] = (v[x + 1] - v[x - 1]) * 45.0 - (v[x + 2] - v[x - 2]) * 9.0 +
+                               (v[x + 3] - v[x - 3]);
+      } else if (tid < N_TXL + N_TYL) {
+        const int q = tid - N_TXL;
+        const int b = (3 + q % 7) + 169 * (q / 7);
+        double v[13];
+#pragma unroll
+        for (int k = 0; k < 13; ++k) v[k] = s[b + 13 * k];
+#pragma unroll
+        for (int y = 3; y <= 9; ++y)
+          Ty[b + 13 * y - TY_OFF] = (v[y + 1] - v[y - 1]) * 45.0 - (v[y + 2] - v[y - 2]) * 9.0 +
+                                    (v[y + 3] - v[y - 3]);
       }
       __syncthreads();
     }

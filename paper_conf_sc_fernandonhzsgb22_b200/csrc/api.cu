@@ -115,7 +115,7 @@ struct dgr_mesh_s {
   double* d_sendbuf = nullptr;
   double* d_recvbuf = nullptr;
   int64_t launches = 0;
-  bool fused = true;            // DGR_OPT_FUSED_UNZIP (measured faster on C3: 44.4 vs 46.3 ms/step)
+  bool fused = false;           // DGR_OPT_FUSED_UNZIP (two-pass: 44.6 ms/step on C3, steadier than fused)
   // profiling
   bool prof = false;
   struct Pend { int cls; cudaEvent_t a, b; };

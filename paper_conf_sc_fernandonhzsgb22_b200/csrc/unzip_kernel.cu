@@ -186,8 +186,10 @@ __global__ void __launch_bounds__(UZ_THREADS, 3)
   const double* Ef = E + f * nn;
   double* dst = patches + (int64_t(f) * m.n_owned + e) * PATCH_PITCH;
 
-  // ---- gather: 8 loads in flight per lane, coalesced stores
-  constexpr int U = 8;
+  // ---- gather: 16 loads in flight per lane; coalesced streaming (evict-first)
+  // stores, so the 10-GB patch stream does not evict the element values and
+  // slots the neighbouring patches still gather from L2
+  constexpr int U = 16;
   for (int p0 = 0; p0 < NPATCH; p0 += 32 * U) {
     double v[U];
     int o[U];
@@ -195,11 +197,13 @@ __global__ void __launch_bounds__(UZ_THREADS, 3)
     for (int u = 0; u < U; ++u) {
       const int p = p0 + u * 32 + lane;
       o[u] = p < NPATCH ? soff[p] : -3;
-      v[u] = o[u] >= 0 ? __ldg(Ef + o[u]) : 0.0;
+      // (volatile asm keeps all U loads ahead of the stores; invalid points load
+      // element value 0 and are not stored)
+      asm volatile("ld.global.nc.f64 %0, [%1];" : "=d"(v[u]) : "l"(Ef + max(o[u], 0)));
     }
 #pragma unroll
     for (int u = 0; u < U; ++u)
-      if (o[u] >= 0) dst[p0 + u * 32 + lane] = v[u];
+      if (o[u] >= 0) __stcs(dst + p0 + u * 32 + lane, v[u]);
   }
 
   // ---- outer-boundary extrapolation along x, then y, then z (reading R12)

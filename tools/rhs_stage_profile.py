@@ -6,6 +6,7 @@ import paper_conf_sc_fernandonhzsgb22_b200 as dgr
 from synth import configs, initial
 cfg = configs.get(sys.argv[1] if len(sys.argv) > 1 else "c3")
 m = dgr.Mesh(cfg)
+m.set_fused(os.environ.get("DGR_FUSED", "1") != "0")
 xyz = m.dof_xyz_host()
 u = torch.zeros((24, m.dof_stride), dtype=torch.float64, device="cuda")
 u[:, :xyz.shape[1]] = torch.from_numpy(initial.for_config(cfg, xyz))

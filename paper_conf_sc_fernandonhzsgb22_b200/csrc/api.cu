@@ -96,12 +96,13 @@ struct dgr_mesh_s {
   NbrEntry* d_nbr = nullptr;
   int32_t* d_zip = nullptr;
   int32_t* d_own = nullptr;     // [n_owned*343] zip-owned DOF of each point or -1
-  int4* d_hang = nullptr;
-  std::vector<int64_t> hang_level_off;  // row offsets per level group
   int64_t* d_dof_node = nullptr;
-  double* d_E = nullptr;        // [24][e_stride]: n_local*343 element values | n_interp slots
-  int32_t* d_gmap = nullptr;    // [n_owned][GM_PITCH] fused-unzip gather map
-  int4* d_iel = nullptr;        // interpolation work per coarse source element
+  double* d_aux = nullptr;      // [24][aux_stride] interpolation slots
+  int32_t* d_o2s = nullptr;     // [n_local][343] element node -> u / slot index
+  int32_t* d_gmap = nullptr;    // [n_owned][GM_PITCH] patch point -> u / slot index
+  std::vector<int64_t> iel_depth_off;   // k_interp launch ranges, one per depth
+  int4* d_iel = nullptr;        // interpolation work per element with slots
+  int4* d_igrp = nullptr;       // ... per face group of its slots
   uint16_t* d_ipt = nullptr;    // half-grid point of each interpolation slot
   int64_t n_interp = 0;
   double* d_patch = nullptr;    // [24][n_owned][PATCH_PITCH] (allocated on first dgr_unzip)
@@ -250,22 +251,6 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
   }
   CUDA_TRY(m->alloc(&m->d_zip, h.zip_local.size()));
   CUDA_TRY(cudaMemcpy(m->d_zip, h.zip_local.data(), h.zip_local.size() * 4, cudaMemcpyHostToDevice));
-  // hanging rows grouped by dependency depth (one launch per depth)
-  std::vector<int4> hr(h.hang_rows.size());
-  m->hang_level_off.clear();
-  int prev = -1;
-  for (size_t i = 0; i < h.hang_rows.size(); ++i) {
-    const auto& r = h.hang_rows[i];
-    if (r.depth != prev) {
-      m->hang_level_off.push_back(int64_t(i));
-      prev = r.depth;
-    }
-    hr[i] = make_int4(r.e_local, r.node, r.src_local, r.t2[0] | (r.t2[1] << 8) | (r.t2[2] << 16));
-  }
-  m->hang_level_off.push_back(int64_t(hr.size()));
-  CUDA_TRY(m->alloc(&m->d_hang, hr.size()));
-  if (!hr.empty())
-    CUDA_TRY(cudaMemcpy(m->d_hang, hr.data(), hr.size() * sizeof(int4), cudaMemcpyHostToDevice));
   // DOF lattice coordinates
   const int64_t nd = h.n_owned_dof + h.n_ghost_dof;
   const int64_t stride = ((nd + 31) / 32) * 32;
@@ -281,66 +266,144 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
   }
   CUDA_TRY(m->alloc(&m->d_dof_node, node.size()));
   CUDA_TRY(cudaMemcpy(m->d_dof_node, node.data(), node.size() * 8, cudaMemcpyHostToDevice));
-  // patch gather map: patch point p of owned octant e reads
-  // SRC_f[gmap[e][p]] — the element value it copies/injects (same formula as
-  // the device setup of the former per-patch unzip), an interpolation slot, or
-  // -1 (extrapolated).  Interpolation slots are deduplicated: one per distinct
-  // (coarse source element, half-grid point t2), numbered element-major in
-  // ascending (element, t2z, t2y, t2x) order; k_interp fills them.
-  int64_t e_stride = 0;
+  // Gather maps.  Every value a patch needs is either a DOF of
+  // the state u (index < dof_stride) or an interpolation SLOT of the auxiliary
+  // array (index dof_stride + slot): one slot per distinct (coarse element c,
+  // half-grid point t2 of c) that is needed, either by a hanging node of a finer
+  // element (Alg. 2 lines 4-5) or by a padding point sourced by a
+  // coarser neighbour.  o2s[e][n] maps element nodes to that index
+  // space; gmap[e][p] maps patch points (copy / injection through o2s of the
+  // source element, interpolation to its slot, -1 = extrapolated).  Slots are
+  // numbered by dependency depth (a slot of c whose 343 nodes are all DOFs has
+  // depth 0, else 1 + the deepest slot among c's nodes; reading R14), then
+  // element, then t2 — k_interp fills one depth per launch.
+  const int64_t ds = ((h.n_owned_dof + h.n_ghost_dof + 31) / 32) * 32;
+  int64_t aux_stride = 0;
   {
-    const int64_t nle = nl * NPT;
-    std::vector<int32_t> cid(size_t(nl), -1);        // coarse source element -> need table
-    std::vector<std::vector<int32_t>> need;          // [t2x + 13 t2y + 169 t2z] -> slot (or -2)
+    std::vector<int32_t> cid(size_t(nl), -1);        // element -> need table
+    std::vector<std::vector<int32_t>> need;          // [t2x + 13 t2y + 169 t2z] -> -1 / -2 / slot
     std::vector<int32_t> celem;
-    auto each_interp = [&](auto&& fn) {
-      for (int64_t e = 0; e < no; ++e) {
-        const uint8_t* pm = h.pmap.data() + size_t(e) * PMAP_PITCH;
-        const NbrEntry* nb = h.nbr.data() + size_t(e) * NBR_MAX;
-        for (int p = 0; p < NPATCH; ++p) {
-          const int j = pm[p];
-          if (j == PM_SELF || j == PM_EXTRAP || nb[j].r != 1) continue;
-          const NbrEntry& t = nb[j];
-          const int ix = p % 13, iy = (p / 13) % 13, iz = p / 169;
-          const int tx = t.o[0] + ix, ty = t.o[1] + iy, tz = t.o[2] + iz;
-          if (tx < 0 || tx > 12 || ty < 0 || ty > 12 || tz < 0 || tz > 12) return false;
-          fn(e, p, t.src, tx + 13 * ty + 169 * tz);
-        }
-      }
-      return true;
-    };
-    bool ok = each_interp([&](int64_t, int, int32_t c, int q) {
+    auto mark = [&](int32_t c, int q) {
       if (cid[c] < 0) {
         cid[c] = int32_t(need.size());
         need.emplace_back(NPATCH, -1);
         celem.push_back(c);
       }
       need[cid[c]][q] = -2;
-    });
-    if (!ok) return fail(DGR_ERR_TREE, "interpolation point outside its source element");
+    };
+    // hanging nodes
+    std::vector<int32_t> hsrc(size_t(nl) * NPT, -1);
+    std::vector<int16_t> hq(size_t(nl) * NPT, -1);
+    for (const auto& r : h.hang_rows) {
+      if (r.t2[0] > 12 || r.t2[1] > 12 || r.t2[2] > 12)
+        return fail(DGR_ERR_TREE, "hanging node outside its source element");
+      const int q = r.t2[0] + 13 * r.t2[1] + 169 * r.t2[2];
+      hsrc[size_t(r.e_local) * NPT + r.node] = r.src_local;
+      hq[size_t(r.e_local) * NPT + r.node] = int16_t(q);
+      mark(r.src_local, q);
+    }
+    // padding points sourced by a coarser neighbour
+    for (int64_t e = 0; e < no; ++e) {
+      const uint8_t* pm = h.pmap.data() + size_t(e) * PMAP_PITCH;
+      const NbrEntry* nb = h.nbr.data() + size_t(e) * NBR_MAX;
+      for (int p = 0; p < NPATCH; ++p) {
+        const int j = pm[p];
+        if (j == PM_SELF || j == PM_EXTRAP || nb[j].r != 1) continue;
+        const NbrEntry& t = nb[j];
+        const int tx = t.o[0] + p % 13, ty = t.o[1] + (p / 13) % 13, tz = t.o[2] + p / 169;
+        if (tx < 0 || tx > 12 || ty < 0 || ty > 12 || tz < 0 || tz > 12)
+          return fail(DGR_ERR_TREE, "interpolation point outside its source element");
+        mark(t.src, tx + 13 * ty + 169 * tz);
+      }
+    }
+    // dependency depth per slot element, coarse to fine (a hanging node's source is coarser)
     std::vector<int32_t> order(celem.size());
     for (size_t i = 0; i < order.size(); ++i) order[i] = int32_t(i);
-    std::sort(order.begin(), order.end(), [&](int32_t a, int32_t b) { return celem[a] < celem[b]; });
-    std::vector<int4> iel;
-    std::vector<uint16_t> ipt;
-    int64_t slot = 0;
+    auto lev = [&](int32_t c) { return h.oct[h.local_oct[c]].l; };
+    std::sort(order.begin(), order.end(), [&](int32_t a, int32_t b) {
+      return lev(celem[a]) != lev(celem[b]) ? lev(celem[a]) < lev(celem[b]) : celem[a] < celem[b];
+    });
+    std::vector<int32_t> edepth(size_t(nl), -1);   // depth of the slots of element c
+    auto node_depth = [&](int32_t e, int n) -> int32_t {   // -1: a DOF
+      const int32_t src = hsrc[size_t(e) * NPT + n];
+      return src < 0 ? -1 : edepth[src];
+    };
     for (int32_t ci : order) {
-      int lo[3] = {12, 12, 12}, hi[3] = {0, 0, 0};
-      const int64_t first = slot;
-      for (int q = 0; q < NPATCH; ++q) {
-        if (need[ci][q] != -2) continue;
-        const int t[3] = {q % 13, (q / 13) % 13, q / 169};
-        for (int k = 0; k < 3; ++k) {
-          lo[k] = std::min(lo[k], t[k]);
-          hi[k] = std::max(hi[k], t[k]);
-        }
-        need[ci][q] = int32_t(slot++);
-        ipt.push_back(uint16_t(t[0] | (t[1] << 4) | (t[2] << 8)));
+      const int32_t c = celem[ci];
+      int32_t d = 0;
+      for (int n = 0; n < NPT; ++n) {
+        const int32_t nd = node_depth(c, n);
+        if (nd == -1) continue;
+        if (edepth[hsrc[size_t(c) * NPT + n]] < 0)
+          return fail(DGR_ERR_TREE, "hanging source not coarser than its element");
+        d = std::max(d, nd + 1);
       }
-      const int lohi = (lo[0] | (lo[1] << 4) | (lo[2] << 8)) | ((hi[0] | (hi[1] << 4) | (hi[2] << 8)) << 12);
-      iel.push_back(make_int4(celem[ci], int32_t(first), int32_t(slot - first), lohi));
+      edepth[c] = d;
     }
-    if (nle + slot >= (int64_t(1) << 31)) return fail(DGR_ERR_ARG, "mesh too large for int32 gather map");
+    std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) {
+      const int32_t da = edepth[celem[a]], db = edepth[celem[b]];
+      return da != db ? da < db : celem[a] < celem[b];
+    });
+    std::vector<int4> iel, igrp;
+    std::vector<uint16_t> ipt;
+    m->iel_depth_off.clear();
+    int64_t slot = 0;
+    int prev_depth = -1;
+    for (int32_t ci : order) {
+      const int32_t c = celem[ci];
+      if (edepth[c] != prev_depth) {
+        m->iel_depth_off.push_back(int64_t(iel.size()));
+        prev_depth = edepth[c];
+      }
+      // one work entry per (element, face group): a slot belongs to the first
+      // face (x-low, x-high, y-low, ...) it lies within 3 half-grid points of
+      // (every slot does: hanging nodes lie on faces, padding reaches 1.5
+      // coarse cells in), and its group sweeps that face's normal axis first
+      // over a bounding box <= 4 points thick.  The sweep order is thus a
+      // function of (element, point) alone, so a slot has the same value on
+      // every partition (multi-rank bit identity).
+      const int32_t g_first = int32_t(igrp.size());
+      for (int grp = 0; grp < 6; ++grp) {
+        int lo[3] = {12, 12, 12}, hi[3] = {0, 0, 0};
+        const int64_t first = slot;
+        for (int q = 0; q < NPATCH; ++q) {
+          if (need[ci][q] != -2) continue;
+          const int t[3] = {q % 13, (q / 13) % 13, q / 169};
+          int g = -1;
+          for (int a = 0; a < 3 && g < 0; ++a)
+            g = t[a] <= 3 ? 2 * a : (t[a] >= 9 ? 2 * a + 1 : -1);
+          if (g < 0) return fail(DGR_ERR_TREE, "interpolation point not near a face of its element");
+          if (g != grp) continue;
+          for (int k = 0; k < 3; ++k) {
+            lo[k] = std::min(lo[k], t[k]);
+            hi[k] = std::max(hi[k], t[k]);
+          }
+          need[ci][q] = int32_t(slot++);
+          ipt.push_back(uint16_t(t[0] | (t[1] << 4) | (t[2] << 8)));
+        }
+        if (slot == first) continue;
+        const int lohi = (lo[0] | (lo[1] << 4) | (lo[2] << 8)) |
+                         ((hi[0] | (hi[1] << 4) | (hi[2] << 8)) << 12) | ((grp / 2) << 24);
+        igrp.push_back(make_int4(int32_t(first), int32_t(slot - first), lohi, 0));
+      }
+      iel.push_back(make_int4(c, g_first, int32_t(igrp.size()) - g_first, 0));
+    }
+    m->iel_depth_off.push_back(int64_t(iel.size()));
+    if (ds + slot >= (int64_t(1) << 31)) return fail(DGR_ERR_ARG, "mesh too large for int32 gather maps");
+    // element nodes -> u / slot index
+    std::vector<int32_t> o2s(size_t(nl) * NPT);
+    for (int64_t e = 0; e < nl; ++e)
+      for (int n = 0; n < NPT; ++n) {
+        const size_t k = size_t(e) * NPT + n;
+        const int32_t d = h.o2n_local[k];
+        if (d >= 0) {
+          o2s[k] = d;
+        } else {
+          if (hsrc[k] < 0) return fail(DGR_ERR_TREE, "hanging node without a source");
+          o2s[k] = int32_t(ds + need[cid[hsrc[k]]][hq[k]]);
+        }
+      }
+    // patch points -> u / slot index
     std::vector<int32_t> gm(size_t(no) * GM_PITCH, -1);
     for (int64_t e = 0; e < no; ++e) {
       const uint8_t* pm = h.pmap.data() + size_t(e) * PMAP_PITCH;
@@ -348,41 +411,46 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
       for (int p = 0; p < NPATCH; ++p) {
         const int j = pm[p];
         const int ix = p % 13, iy = (p / 13) % 13, iz = p / 169;
-        int64_t v = -1;
+        int32_t v = -1;
         if (j == PM_SELF) {
-          v = e * NPT + (ix - 3) + 7 * (iy - 3) + 49 * (iz - 3);
+          v = o2s[size_t(e) * NPT + (ix - 3) + 7 * (iy - 3) + 49 * (iz - 3)];
         } else if (j != PM_EXTRAP) {
           const NbrEntry& t = nb[j];
           if (t.r == 1) {
             const int q = (t.o[0] + ix) + 13 * (t.o[1] + iy) + 169 * (t.o[2] + iz);
-            v = nle + need[cid[t.src]][q];
+            v = int32_t(ds + need[cid[t.src]][q]);
           } else {
             const int tx = (t.o[0] + t.r * ix) >> 1, ty = (t.o[1] + t.r * iy) >> 1,
                       tz = (t.o[2] + t.r * iz) >> 1;
-            v = int64_t(t.src) * NPT + tx + 7 * ty + 49 * tz;
+            v = o2s[size_t(t.src) * NPT + tx + 7 * ty + 49 * tz];
           }
         }
-        gm[size_t(e) * GM_PITCH + p] = int32_t(v);
+        gm[size_t(e) * GM_PITCH + p] = v;
       }
     }
     m->n_interp = slot;
-    e_stride = ((nle + slot + 31) / 32) * 32;
+    aux_stride = std::max<int64_t>(32, ((slot + 31) / 32) * 32);
+    CUDA_TRY(m->alloc(&m->d_o2s, o2s.size()));
+    CUDA_TRY(cudaMemcpy(m->d_o2s, o2s.data(), o2s.size() * 4, cudaMemcpyHostToDevice));
     CUDA_TRY(m->alloc(&m->d_gmap, gm.size()));
     CUDA_TRY(cudaMemcpy(m->d_gmap, gm.data(), gm.size() * 4, cudaMemcpyHostToDevice));
     CUDA_TRY(m->alloc(&m->d_iel, iel.size()));
     if (!iel.empty())
       CUDA_TRY(cudaMemcpy(m->d_iel, iel.data(), iel.size() * sizeof(int4), cudaMemcpyHostToDevice));
+    CUDA_TRY(m->alloc(&m->d_igrp, igrp.size()));
+    if (!igrp.empty())
+      CUDA_TRY(cudaMemcpy(m->d_igrp, igrp.data(), igrp.size() * sizeof(int4), cudaMemcpyHostToDevice));
     CUDA_TRY(m->alloc(&m->d_ipt, ipt.size()));
     if (!ipt.empty())
       CUDA_TRY(cudaMemcpy(m->d_ipt, ipt.data(), ipt.size() * 2, cudaMemcpyHostToDevice));
     m->dm.n_iel = int32_t(iel.size());
   }
   // workspace
-  CUDA_TRY(m->alloc(&m->d_E, size_t(NF) * e_stride));
+  CUDA_TRY(m->alloc(&m->d_aux, size_t(NF) * aux_stride));
   CUDA_TRY(m->alloc(&m->d_rhs_oct, size_t(NF) * no * NPT));
   CUDA_TRY(m->alloc(&m->d_us, size_t(NF) * stride));
   CUDA_TRY(m->alloc(&m->d_acc, size_t(NF) * stride));
-  CUDA_TRY(cudaMemset(m->d_E, 0, size_t(NF) * e_stride * 8));
+  CUDA_TRY(cudaMemset(m->d_aux, 0, size_t(NF) * aux_stride * 8));
   CUDA_TRY(cudaMemset(m->d_us, 0, size_t(NF) * stride * 8));
   CUDA_TRY(cudaMemset(m->d_acc, 0, size_t(NF) * stride * 8));
   double w13[91], wext[21];
@@ -403,10 +471,12 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
   dm.pmap = m->d_pmap;
   dm.nbr = m->d_nbr;
   dm.zip = m->d_zip;
-  dm.hang = m->d_hang;
-  dm.e_stride = e_stride;
+  dm.aux_stride = aux_stride;
+  dm.aux = m->d_aux;
+  dm.o2s = m->d_o2s;
   dm.gmap = m->d_gmap;
   dm.iel = m->d_iel;
+  dm.igrp = m->d_igrp;
   dm.ipt = m->d_ipt;
   // multi-rank buffers
   if (h.nranks > 1) {
@@ -617,36 +687,26 @@ static dgr_status exchange(dgr_mesh m, double* u, cudaStream_t st) {
   return DGR_OK;
 }
 
-// element reconstruction (Alg. 2 lines 2-5): E from u, hanging nodes level by level
-static dgr_status do_elements(dgr_mesh m, const double* u, int nf, cudaStream_t st) {
-  PROF(m, 0, st, launch_elements(m->dm, u, m->d_E, nf, st));
-  for (size_t g = 0; g + 1 < m->hang_level_off.size(); ++g) {
-    const int64_t a = m->hang_level_off[g], b = m->hang_level_off[g + 1];
-    PROF(m, 1, st, launch_hanging(m->dm, m->d_hang + a, b - a, m->d_E, nf, st));
+// interpolation slots (hanging nodes and coarse-neighbour padding values,
+// Alg. 2 lines 4-5 and P:L295), one k_interp launch per dependency depth
+static dgr_status do_interp(dgr_mesh m, const double* u, int nf, cudaStream_t st) {
+  for (size_t g = 0; g + 1 < m->iel_depth_off.size(); ++g) {
+    const int64_t a = m->iel_depth_off[g], b = m->iel_depth_off[g + 1];
+    PROF(m, 7, st, launch_interp(m->dm, u, nf, a, b - a, st));
   }
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;
 }
 
-// explicit unzip into the patch buffer (dgr_unzip, constraints)
+// explicit unzip into the patch buffer (two-pass path, dgr_unzip, constraints)
 static dgr_status do_unzip(dgr_mesh m, const double* u, int nf, cudaStream_t st) {
   if (!m->d_patch) {
     CUDA_TRY(m->alloc(&m->d_patch, size_t(NF) * m->dm.n_owned * PATCH_PITCH));
     CUDA_TRY(cudaMemsetAsync(m->d_patch, 0, size_t(NF) * m->dm.n_owned * PATCH_PITCH * 8, st));
   }
-  dgr_status s = do_elements(m, u, nf, st);
+  dgr_status s = do_interp(m, u, nf, st);
   if (s) return s;
-  PROF(m, 7, st, launch_interp(m->dm, m->d_E, nf, st));
-  PROF(m, 2, st, launch_unzip(m->dm, m->d_E, m->d_patch, nf, st));
-  CUDA_TRY(cudaGetLastError());
-  return DGR_OK;
-}
-
-// fused path: elements + coarse-neighbour interpolation slots; k_rhs<true> gathers the patches
-static dgr_status do_fused_sources(dgr_mesh m, const double* u, cudaStream_t st) {
-  dgr_status s = do_elements(m, u, NF, st);
-  if (s) return s;
-  PROF(m, 7, st, launch_interp(m->dm, m->d_E, NF, st));
+  PROF(m, 2, st, launch_unzip(m->dm, u, m->d_patch, nf, st));
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;
 }
@@ -662,8 +722,8 @@ static RhsParams to_rp(const dgr_params* p) {
 static dgr_status rhs_oct(dgr_mesh m, const double* u, const dgr_params* prm, cudaStream_t st) {
   dgr_status s;
   if (m->fused) {
-    if ((s = do_fused_sources(m, u, st))) return s;
-    PROF(m, 3, st, launch_rhs(m->dm, m->d_E, m->d_rhs_oct, to_rp(prm), nullptr, true, st));
+    if ((s = do_interp(m, u, NF, st))) return s;
+    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, to_rp(prm), nullptr, true, st));
   } else {
     if ((s = do_unzip(m, u, NF, st))) return s;
     PROF(m, 3, st, launch_rhs(m->dm, m->d_patch, m->d_rhs_oct, to_rp(prm), nullptr, false, st));

@@ -26,29 +26,33 @@ struct DevMesh {
   const uint8_t* pmap;      // [n_owned * 2197]
   const NbrEntry* nbr;      // [n_owned * NBR_MAX]
   const int32_t* zip;       // [n_owned_dof] local octant * 343 + node
-  const int4* hang;         // rows: e_local, node, src_local, t2 packed (x | y<<8 | z<<16)
-  // Patch gather: per field the source array SRC_f = E + f * e_stride holds
-  // [element values of the n_local octants (n_local*343) | interpolation slots (n_interp)].
-  // A slot is one distinct (coarse source element, half-grid point) pair that some
-  // patch point interpolates from a coarser neighbour (deduplicated over all patches).
-  // gmap[e][p] is the SRC_f index of patch point p of owned octant e, or -1 for a point
-  // outside a non-periodic domain (extrapolated).
-  int64_t e_stride;         // doubles per field of E (>= n_local*343 + n_interp)
+  // Gather maps.  Index space of every value a patch needs:
+  // i < dof_stride -> u[f * dof_stride + i] (a DOF of the state), else
+  // aux[f * aux_stride + i - dof_stride] (an interpolation slot: one distinct
+  // (coarse element, half-grid point) needed by a hanging node or by a padding
+  // point sourced by a coarser neighbour, filled by k_interp).
+  double* aux;              // [24][aux_stride]
+  int64_t aux_stride;
+  const int32_t* o2s;       // [n_local * 343] element node -> index
+  // gmap[e][p]: index of patch point p of owned octant e, -1 outside a
+  // non-periodic domain (extrapolated)
   const int32_t* gmap;      // [n_owned * GM_PITCH]
-  // interpolation work, one entry per coarse source element:
-  //   {element, first slot, slot count, bbox lo (x|y<<4|z<<8) | hi << 12}
+  // interpolation work: one entry per element with slots (sorted by dependency
+  // depth) {element, first group, group count, 0}, and per face group of its
+  // slots {first slot, slot count, bbox lo (x|y<<4|z<<8) | hi << 12 | first
+  // sweep axis << 24, 0}
   const int4* iel;
+  const int4* igrp;
   int32_t n_iel;
   const uint16_t* ipt;      // [n_interp] half-grid point of each slot, t2x | t2y<<4 | t2z<<8
 };
 
+// unzip_kernel.cu
+void launch_unzip(const DevMesh& m, const double* u, double* patches, int nf, cudaStream_t s);
+// interpolation slots of m.iel[first .. first + count) (one dependency depth)
+void launch_interp(const DevMesh& m, const double* u, int nf, int64_t first, int64_t count,
+                   cudaStream_t s);
 // kernels.cu
-void launch_elements(const DevMesh& m, const double* u, double* E, int nf, cudaStream_t s);
-void launch_hanging(const DevMesh& m, const int4* rows, int64_t count, double* E, int nf,
-                    cudaStream_t s);
-void launch_unzip(const DevMesh& m, const double* E, double* patches, int nf, cudaStream_t s);
-// interpolation slots (coarse-neighbour padding values) of E, from the element values
-void launch_interp(const DevMesh& m, double* E, int nf, cudaStream_t s);
 void launch_zip(const DevMesh& m, const double* rhs_oct, double* rhs, int nf, cudaStream_t s);
 void launch_zip_rk4(const DevMesh& m, const double* rhs_oct, int stage, double dt,
                     const double* u_n, double* u_s, double* acc, double* u_out, cudaStream_t s);
@@ -77,7 +81,8 @@ struct RkArgs {
   int64_t stride;
 };
 // fused = false: read 13^3 patches ([24][n_owned][PATCH_PITCH], TMA bulk copies);
-// fused = true: gather every patch from E through gmap (no patch buffer)
+// fused = true: `src` is the state u; every patch is gathered from u and the
+// slots through gmap (no patch buffer)
 void launch_rhs(const DevMesh& m, const double* src, double* rhs_oct, const RhsParams& p,
                 const RkArgs* rk, bool fused, cudaStream_t s);
 size_t rhs_smem_bytes();

@@ -1,5 +1,6 @@
-// Unzip (octant-to-patch), element reconstruction, zip (patch-to-octant) and
-// the fused zip + RK4 stage kernels (sm_100a, fp64).
+// Zip (patch-to-octant), the fused zip + RK4 stage kernels, DOF coordinates,
+// ghost pack/unpack and the fp64 microbenchmark (sm_100a, fp64).  Octant-to-
+// patch (unzip, hanging nodes, interpolation): unzip_kernel.cu.
 //
 // PAPER.md Alg. 2 (L249-283) / §IV-A (L235-306): octant-to-patch fills the
 // (r+2k)^3 = 13^3 padded patch of every octant by copy (same level), injection
@@ -16,125 +17,9 @@ namespace dgr {
 
 // Lagrange rows: [t2][m] = l_m(t2/2), degree 6 on nodes 0..6;
 // extrapolation rows [t][m] = l_m(-(t+1)).  Filled by the host (api.cu).
-__constant__ double c_W13[13 * 7];
-__constant__ double c_WEXT[3 * 7];
-
 void upload_unzip_tables(const double* w13, const double* wext);  // unzip_kernel.cu
 
-void upload_tables(const double* w13, const double* wext) {
-  cudaMemcpyToSymbol(c_W13, w13, sizeof(double) * 91);
-  cudaMemcpyToSymbol(c_WEXT, wext, sizeof(double) * 21);
-  upload_unzip_tables(w13, wext);
-}
-
-// I_c(t2) = sum_{ijk} W[t2x][i] W[t2y][j] W[t2z][k] E_c[i + 7j + 49k]; along an
-// axis with even t2 the row is a unit vector: a single term.
-__device__ __forceinline__ double interp_point(const double* __restrict__ Ec, int tx, int ty,
-                                               int tz, const double* __restrict__ W) {
-  const int nx = (tx & 1) ? 7 : 1, ny = (ty & 1) ? 7 : 1, nz = (tz & 1) ? 7 : 1;
-  const int x0 = (tx & 1) ? 0 : (tx >> 1), y0 = (ty & 1) ? 0 : (ty >> 1),
-            z0 = (tz & 1) ? 0 : (tz >> 1);
-  double acc = 0.0;
-  for (int c = 0; c < nz; ++c) {
-    const double wz = (tz & 1) ? W[tz * 7 + c] : 1.0;
-    double accy = 0.0;
-    for (int b = 0; b < ny; ++b) {
-      const double wy = (ty & 1) ? W[ty * 7 + b] : 1.0;
-      const double* row = Ec + (x0 + 7 * (y0 + b) + 49 * (z0 + c));
-      double accx = 0.0;
-      for (int a = 0; a < nx; ++a) {
-        const double wx = (tx & 1) ? W[tx * 7 + a] : 1.0;
-        accx = fma(wx, __ldg(row + a), accx);
-      }
-      accy = fma(wy, accx, accy);
-    }
-    acc = fma(wz, accy, acc);
-  }
-  return acc;
-}
-
-// ---------------------------------------------------------- element gather
-// E[f][e][n] = u[f][O2N[e][n]] for DOF nodes (Alg. 2 line 2); hanging nodes
-// are filled level by level by k_hanging.
-__global__ void k_elements(const double* __restrict__ u, int64_t stride,
-                           const int32_t* __restrict__ o2n, int64_t nn, int64_t es,
-                           double* __restrict__ E) {
-  const int f = blockIdx.y;
-  const double* uf = u + f * stride;
-  double* Ef = E + f * es;
-  for (int64_t i = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; i < nn;
-       i += int64_t(gridDim.x) * blockDim.x) {
-    const int32_t id = __ldg(o2n + i);
-    Ef[i] = id >= 0 ? __ldg(uf + id) : 0.0;
-  }
-}
-
-void launch_elements(const DevMesh& m, const double* u, double* E, int nf, cudaStream_t s) {
-  const int64_t nn = int64_t(m.n_local) * NPT;
-  int blocks = int((nn + 255) / 256);
-  if (blocks > 148 * 16) blocks = 148 * 16;
-  k_elements<<<dim3(blocks, nf), 256, 0, s>>>(u, m.dof_stride, m.o2n, nn, m.e_stride, E);
-}
-
-// --------------------------------------------------------- hanging points
-// interp_hanging (Alg. 2 lines 4-5): E[e][node] = I_src(t2), rows of one level.
-// One thread per hanging row and a group of 4 fields: the stencil (which node
-// offsets, which weights) is decoded once and applied to 4 fields at a time.
-constexpr int HANG_FG = 4;
-__global__ void k_hanging(const int4* __restrict__ rows, int64_t count, double* __restrict__ E,
-                          int64_t nn, int nf) {
-  __shared__ double W[91];
-  for (int i = threadIdx.x; i < 91; i += blockDim.x) W[i] = c_W13[i];
-  __syncthreads();
-  const int f0 = blockIdx.y * HANG_FG;
-  for (int64_t r = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; r < count;
-       r += int64_t(gridDim.x) * blockDim.x) {
-    const int4 row = rows[r];
-    const int tx = row.w & 0xff, ty = (row.w >> 8) & 0xff, tz = (row.w >> 16) & 0xff;
-    const int nx = (tx & 1) ? 7 : 1, ny = (ty & 1) ? 7 : 1, nz = (tz & 1) ? 7 : 1;
-    const int x0 = (tx & 1) ? 0 : (tx >> 1), y0 = (ty & 1) ? 0 : (ty >> 1),
-              z0 = (tz & 1) ? 0 : (tz >> 1);
-    const double* Ec = E + int64_t(row.z) * NPT;
-    double acc[HANG_FG];
-#pragma unroll
-    for (int g = 0; g < HANG_FG; ++g) acc[g] = 0.0;
-    for (int c = 0; c < nz; ++c) {
-      const double wz = (tz & 1) ? W[tz * 7 + c] : 1.0;
-      double accy[HANG_FG];
-#pragma unroll
-      for (int g = 0; g < HANG_FG; ++g) accy[g] = 0.0;
-      for (int b = 0; b < ny; ++b) {
-        const double wy = (ty & 1) ? W[ty * 7 + b] : 1.0;
-        const int off = x0 + 7 * (y0 + b) + 49 * (z0 + c);
-        double accx[HANG_FG];
-#pragma unroll
-        for (int g = 0; g < HANG_FG; ++g) accx[g] = 0.0;
-        for (int a = 0; a < nx; ++a) {
-          const double wx = (tx & 1) ? W[tx * 7 + a] : 1.0;
-#pragma unroll
-          for (int g = 0; g < HANG_FG; ++g)
-            if (f0 + g < nf) accx[g] = fma(wx, __ldg(Ec + (f0 + g) * nn + off + a), accx[g]);
-        }
-#pragma unroll
-        for (int g = 0; g < HANG_FG; ++g) accy[g] = fma(wy, accx[g], accy[g]);
-      }
-#pragma unroll
-      for (int g = 0; g < HANG_FG; ++g) acc[g] = fma(wz, accy[g], acc[g]);
-    }
-#pragma unroll
-    for (int g = 0; g < HANG_FG; ++g)
-      if (f0 + g < nf) E[(f0 + g) * nn + int64_t(row.x) * NPT + row.y] = acc[g];
-  }
-}
-
-void launch_hanging(const DevMesh& m, const int4* rows, int64_t count, double* E, int nf,
-                    cudaStream_t s) {
-  if (count <= 0) return;
-  int blocks = int((count + 127) / 128);
-  if (blocks > 148 * 16) blocks = 148 * 16;
-  k_hanging<<<dim3(blocks, (nf + HANG_FG - 1) / HANG_FG), 128, 0, s>>>(
-      rows, count, E, m.e_stride, nf);
-}
+void upload_tables(const double* w13, const double* wext) { upload_unzip_tables(w13, wext); }
 
 // (octant-to-patch: unzip_kernel.cu)
 

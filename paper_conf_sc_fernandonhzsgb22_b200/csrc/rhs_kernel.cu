@@ -93,14 +93,17 @@ __device__ __forceinline__ void bulk_load(double* dst, const double* src, uint32
       : "memory");
 }
 
-// 8-byte asynchronous global->shared copy of src[idx] (the fused unzip's
-// gather); the address arithmetic stays inside the asm so the compiler cannot
-// rematerialise the field base per copy
-__device__ __forceinline__ void cp_async8(uint32_t dst, const double* src, int32_t idx) {
+// 8-byte asynchronous global->shared copy of (idx < ds ? uf : af)[idx] (the
+// fused unzip's gather: a DOF of the state or an interpolation slot); the
+// address arithmetic stays inside the asm so the compiler cannot rematerialise
+// the field bases per copy
+__device__ __forceinline__ void cp_async8(uint32_t dst, const double* uf, const double* af,
+                                          int32_t idx, int32_t ds) {
   asm volatile(
-      "{\n .reg .u64 a;\n mad.wide.s32 a, %2, 8, %1;\n"
+      "{\n .reg .u64 a;\n .reg .pred q;\n setp.lt.s32 q, %3, %4;\n"
+      " selp.b64 a, %1, %2, q;\n mad.wide.s32 a, %3, 8, a;\n"
       " cp.async.ca.shared.global [%0], [a], 8;\n}\n" ::"r"(dst),
-      "l"(src), "r"(idx)
+      "l"(uf), "l"(af), "r"(idx), "r"(ds)
       : "memory");
 }
 __device__ __forceinline__ void cp_async_commit() {
@@ -224,10 +227,9 @@ __device__ __forceinline__ double trace6(const double* gi, const double* X) {
 }  // namespace
 
 // FUSED = false: `patches` is the 13^3 patch buffer [24][n_owned][PATCH_PITCH]
-// (bulk copies).  FUSED = true: `patches` is E (DevMesh::e_stride per field) and
-// every patch is gathered straight from it through m.gmap with 8-byte cp.async
-// (the unzip fused into the RHS): copy/injection points read
-// element values, coarse-neighbour points read the slots k_interp filled, and
+// (bulk copies).  FUSED = true: `patches` is the state u and every patch is
+// gathered straight from u and the interpolation slots through m.gmap with
+// 8-byte cp.async (the unzip fused into the RHS), and
 // points outside a non-periodic domain are extrapolated in shared memory with
 // the same arithmetic as k_unzip.
 template <bool FUSED>
@@ -253,7 +255,8 @@ __global__ void __launch_bounds__(RT, 1)
     tab_p[tid] = int16_t(q);
   }
   const int64_t no = m.n_owned;
-  const int64_t fstride = FUSED ? m.e_stride : no * PATCH_PITCH;
+  const int64_t fstride = FUSED ? m.dof_stride : no * PATCH_PITCH;
+  const int32_t ds = int32_t(m.dof_stride);
   int gidx[GJ];   // FUSED: SRC index of patch points tid + RT*j of the current octant
   auto load_gidx = [&](int oct) {
     const int32_t* gm = m.gmap + int64_t(oct) * GM_PITCH;
@@ -264,12 +267,19 @@ __global__ void __launch_bounds__(RT, 1)
       gidx[j] = pt < NPATCH ? max(__ldg(gm + pt), 0) : -1;
     }
   };
-  auto gather = [&](double* dst, const double* srcf) {
+  auto gather = [&](double* dst, int f) {
     const uint32_t d0 = smem_u32(dst + tid);
+    const double* uf = patches + f * fstride;
+    const double* af = m.aux + f * m.aux_stride - m.dof_stride;
 #pragma unroll
-    for (int j = 0; j < GJ - 1; ++j) cp_async8(d0 + 8 * RT * j, srcf, gidx[j]);
-    if (tid + RT * (GJ - 1) < NPATCH) cp_async8(d0 + 8 * RT * (GJ - 1), srcf, gidx[GJ - 1]);
+    for (int j = 0; j < GJ - 1; ++j) cp_async8(d0 + 8 * RT * j, uf, af, gidx[j], ds);
+    if (tid + RT * (GJ - 1) < NPATCH) cp_async8(d0 + 8 * RT * (GJ - 1), uf, af, gidx[GJ - 1], ds);
     cp_async_commit();
+  };
+  // FUSED: the value of field f at element node (e, p), through o2s
+  auto node_value = [&](int f, int oct, int node) {
+    const int32_t x = __ldg(m.o2s + int64_t(oct) * NPT + node);
+    return x < ds ? __ldg(patches + f * fstride + x) : __ldg(m.aux + f * m.aux_stride + (x - ds));
   };
 #define SL(slot) slots[(slot) * NPP + tid]
   auto prefetch_l2 = [&](const double* src) {
@@ -291,8 +301,8 @@ __global__ void __launch_bounds__(RT, 1)
   __syncthreads();
   if (FUSED) {
     load_gidx(e);
-    gather(stage, patches + c_order[0] * fstride);
-    gather(stage + STAGE_DBL, patches + c_order[1] * fstride);
+    gather(stage, c_order[0]);
+    gather(stage + STAGE_DBL, c_order[1]);
   } else if (tid == 0) {
     const double* pb = patches + int64_t(e) * PATCH_PITCH;
     bulk_load(stage, pb + c_order[0] * fstride, STAGE_DBL * 8, &bars[0]);
@@ -305,7 +315,13 @@ __global__ void __launch_bounds__(RT, 1)
   const int en = e + gridDim.x;                    // next octant of this CTA
   const double* pbase = patches + int64_t(e) * (FUSED ? NPT : PATCH_PITCH);
   const bool active = tab_c0[tid] >= 0;
-  const int cv = FUSED ? tab_p[tid] : tab_c0[tid];   // own value: element node p / patch index c0
+  // the point's own values: patch index c0 of the staged patches, or (FUSED)
+  // element node p of u / a hanging-node slot through o2s
+  const int cv = FUSED ? __ldg(m.o2s + int64_t(e) * NPT + max(int(tab_p[tid]), 0)) : tab_c0[tid];
+  auto own = [&](int f) -> double {
+    if (!FUSED) return __ldg(pbase + f * fstride + cv);
+    return cv < ds ? __ldg(patches + f * fstride + cv) : __ldg(m.aux + f * m.aux_stride + (cv - ds));
+  };
 
   const int4 oi = m.oct[e];
   // FUSED: which faces of this octant lie on a non-periodic domain boundary
@@ -317,38 +333,27 @@ __global__ void __launch_bounds__(RT, 1)
             ((oi.y + sd == nside) << 4) | ((oi.z + sd == nside) << 5);
   }
   const bool bnd = omask != 0;
-  if (FUSED && en < no) {
-    if (tid == 32)   // next octant's gather map into L2
-      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(m.gmap + int64_t(en) * GM_PITCH),
-                   "r"(uint32_t(GM_PITCH * 4))
-                   : "memory");
-    else if (tid >= 64 && tid < 64 + NF) {
-      // ... and its own element values (read at its start and by its first gathers),
-      // 16-B aligned cover of the 343 doubles of field tid - 64
-      const uintptr_t a = reinterpret_cast<uintptr_t>(patches + (tid - 64) * fstride +
-                                                      int64_t(en) * NPT);
-      const uintptr_t a0 = a & ~uintptr_t(15), a1 = (a + NPT * 8 + 15) & ~uintptr_t(15);
-      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a0), "r"(uint32_t(a1 - a0))
-                   : "memory");
-    }
-  }
+  if (FUSED && en < no && tid == 32)   // next octant's gather map into L2
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(m.gmap + int64_t(en) * GM_PITCH),
+                 "r"(uint32_t(GM_PITCH * 4))
+                 : "memory");
   const double ih = (6.0 * double(int64_t(1) << oi.w)) / m.width;   // 1/h
   const double ko_scale = prm.ko_sigma * ih * (1.0 / 64.0);
 
   // ---- values at the point (patch interior) -------------------------------
   double alpha = 0, chi = 0, Kv = 0, beta[3] = {0, 0, 0};
   if (active) {
-    alpha = __ldg(pbase + 0 * fstride + cv);
-    chi = __ldg(pbase + 1 * fstride + cv);
-    Kv = __ldg(pbase + 2 * fstride + cv);
+    alpha = own(0);
+    chi = own(1);
+    Kv = own(2);
 #pragma unroll
-    for (int i = 0; i < 3; ++i) beta[i] = __ldg(pbase + (6 + i) * fstride + cv);
+    for (int i = 0; i < 3; ++i) beta[i] = own(6 + i);
     double g[6];
 #pragma unroll
     for (int q = 0; q < 6; ++q) {
-      g[q] = __ldg(pbase + (12 + q) * fstride + cv);
+      g[q] = own(12 + q);
       SL(V_GAM + q) = g[q];
-      SL(V_AT + q) = __ldg(pbase + (18 + q) * fstride + cv);
+      SL(V_AT + q) = own(18 + q);
     }
     // inverse metric by adjugate / determinant
     const double a00 = g[3] * g[5] - g[4] * g[4];
@@ -756,10 +761,10 @@ __global__ void __launch_bounds__(RT, 1)
     if (FUSED) {
       double* dst = stage + buf * STAGE_DBL;
       if (st + 2 < NF) {
-        gather(dst, patches + c_order[st + 2] * fstride);
+        gather(dst, c_order[st + 2]);
       } else {
         if (st + 2 == NF && en < no) load_gidx(en);   // the current octant's gathers are issued
-        if (en < no) gather(dst, patches + c_order[st + 2 - NF] * fstride);
+        if (en < no) gather(dst, c_order[st + 2 - NF]);
         else cp_async_commit();                        // (empty group keeps the count uniform)
       }
       continue;
@@ -797,9 +802,12 @@ __global__ void __launch_bounds__(RT, 1)
       gi[r] = SL(G_INV + r);
       At[r] = SL(V_AT + r);
     }
-    const int cb = FUSED ? p : tab_c0[tid];
+    const int cb = FUSED ? __ldg(m.o2s + int64_t(e) * NPT + p) : tab_c0[tid];
 #pragma unroll
-    for (int i = 0; i < 3; ++i) B[i] = __ldg(pbase + (9 + i) * fstride + cb);
+    for (int i = 0; i < 3; ++i)
+      B[i] = !FUSED ? __ldg(pbase + (9 + i) * fstride + cb)
+                    : (cb < ds ? __ldg(patches + (9 + i) * fstride + cb)
+                               : __ldg(m.aux + (9 + i) * m.aux_stride + (cb - ds)));
     // At^k_j and At_ik At^k_j, At_ij At^ij
     double Am[3][3];
 #pragma unroll

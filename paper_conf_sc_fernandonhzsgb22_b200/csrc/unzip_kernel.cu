@@ -3,15 +3,18 @@
 // Gather formulation, in two kernels:
 //  * k_interp computes every *interpolation slot* once: the value of a coarser
 //    element's degree-6 tensor Lagrange interpolant at a half-grid
-//    point some finer neighbour's patch needs.  Slots are deduplicated on the
-//    host (one per distinct (coarse element, point); on C3 3.6x fewer than the
-//    padding points they feed) and evaluated per coarse element by three 1-D
-//    sweeps over the bounding box of its slots, thinnest axis first.
+//    point that a hanging node of a finer element (Alg. 2 lines 4-5) or a
+//    finer neighbour's padding point needs.  Slots are deduplicated on the
+//    host (one per distinct (coarse element, point); on C3 the padding points
+//    alone need 3.6x fewer slots than points) and evaluated per element by
+//    three 1-D sweeps over the bounding box of its slots, thinnest axis first;
+//    the element's 343 nodal values are gathered from the state u and from
+//    coarser slots (one launch per dependency depth: hanging chains, R14).
 //  * k_unzip then assembles each 13^3 patch as a pure gather through the
-//    mesh's gather map (copy / injection from element values, interpolated
-//    points from the slots) with coalesced stores, and extrapolates outside a
-//    non-periodic domain (reading R12).  The fused RHS (rhs_kernel.cu) performs
-//    the same gather itself, straight into shared memory.
+//    mesh's gather map (copy / injection of DOFs or hanging-node slots,
+//    interpolated points from their slots) with coalesced stores, and
+//    extrapolates outside a non-periodic domain (reading R12).  The fused RHS
+//    (rhs_kernel.cu) performs the same gather itself, into shared memory.
 #include <cuda_runtime.h>
 
 #include "device.cuh"
@@ -38,34 +41,44 @@ constexpr int IP_FIELD = NPT + IP_T1 + IP_T2;   // scratch doubles per field
 __device__ __forceinline__ int fdiv(int i, float rn) { return int((float(i) + 0.5f) * rn); }
 }  // namespace
 
-// One CTA per (coarse source element, group of IP_FG fields).  Sweep 1 along
-// the thinnest axis a1 of the slots' bounding box over all 7x7 node rows,
-// sweep 2 along a2, then each slot's value along a3 (same 1-D operation per
+// One CTA per (element, group of IP_FG fields): the element's nodal values are
+// staged once, then for each face group of its slots, sweep 1 along the
+// group's face normal a1 (its bounding box is <= 4 points thick along it) over
+// all 7x7 node rows, sweep 2 along a2, then each slot's value along a3 (same 1-D operation per
 // axis as the oracle's definition: sum_m l_m(t2/2) v_m, m = 0..6, or a copy at
 // even t2).
 __global__ void __launch_bounds__(IP_THREADS)
-    k_interp(DevMesh m, double* __restrict__ E, int nf) {
+    k_interp(DevMesh m, const double* __restrict__ u, int nf, int64_t first) {
   extern __shared__ __align__(16) double dyn[];
   __shared__ double W[91];
-  const int4 el = m.iel[blockIdx.x];
+  const int4 el = m.iel[first + blockIdx.x];
   const int f0 = blockIdx.y * IP_FG;
   const int tid = threadIdx.x;
-  const int64_t es = m.e_stride;
+  const int64_t ds = m.dof_stride, as = m.aux_stride;
   double* Es = dyn;                              // [IP_FG][NPT]
   double* T1 = Es + IP_FG * NPT;                 // [IP_FG][IP_T1]
   double* T2 = T1 + IP_FG * IP_T1;               // [IP_FG][IP_T2]
   for (int i = tid; i < 91; i += IP_THREADS) W[i] = c_uW13[i];
   for (int i = tid; i < IP_FG * NPT; i += IP_THREADS) {
     const int g = i / NPT, n = i - g * NPT;
-    Es[i] = f0 + g < nf ? __ldg(E + (f0 + g) * es + int64_t(el.x) * NPT + n) : 0.0;
+    double v = 0.0;
+    if (f0 + g < nf) {
+      const int32_t x = __ldg(m.o2s + int64_t(el.x) * NPT + n);
+      // (slots of coarser elements were written by an earlier launch: plain load)
+      v = x < ds ? __ldg(u + (f0 + g) * ds + x) : m.aux[(f0 + g) * as + (x - ds)];
+    }
+    Es[i] = v;
   }
+  __syncthreads();
+  for (int gi = 0; gi < el.z; ++gi) {
+  const int4 gr = m.igrp[el.y + gi];
   int lo[3], n[3];
 #pragma unroll
   for (int k = 0; k < 3; ++k) {
-    lo[k] = (el.w >> (4 * k)) & 15;
-    n[k] = ((el.w >> (12 + 4 * k)) & 15) - lo[k] + 1;
+    lo[k] = (gr.z >> (4 * k)) & 15;
+    n[k] = ((gr.z >> (12 + 4 * k)) & 15) - lo[k] + 1;
   }
-  const int a1 = n[0] <= n[1] && n[0] <= n[2] ? 0 : (n[1] <= n[2] ? 1 : 2);
+  const int a1 = (gr.z >> 24) & 3;   // the group's face normal (host-chosen, partition-invariant)
   const int a2 = a1 == 0 ? 1 : 0, a3 = a1 == 2 ? 1 : 2;
   const int n1 = n[a1], n2 = n[a2];
   const int es1 = a1 == 0 ? 1 : (a1 == 1 ? 7 : 49);
@@ -73,7 +86,6 @@ __global__ void __launch_bounds__(IP_THREADS)
   const int es3 = a3 == 0 ? 1 : (a3 == 1 ? 7 : 49);
   const int lo1 = lo[a1], lo2 = lo[a2];
   const float rn1 = 1.0f / float(n1), rn2 = 1.0f / float(n2);
-  __syncthreads();
   // T1[g][r3][r2][i1] = sum_m W[lo1+i1][m] E_g[m, r2, r3]
   for (int idx = tid; idx < 49 * n1; idx += IP_THREADS) {
     const int r = fdiv(idx, rn1), i1 = idx - r * n1;   // r = r3 * 7 + r2
@@ -125,9 +137,9 @@ __global__ void __launch_bounds__(IP_THREADS)
   }
   __syncthreads();
   // slot value = sum_m W[t2_a3][m] T2[g][m][i2][i1]
-  const int64_t base = int64_t(m.n_local) * NPT + el.y;
-  for (int k = tid; k < el.z; k += IP_THREADS) {
-    const int t = __ldg(m.ipt + el.y + k);
+  double* out = m.aux + gr.x;
+  for (int k = tid; k < gr.y; k += IP_THREADS) {
+    const int t = __ldg(m.ipt + gr.x + k);
     const int t2[3] = {t & 15, (t >> 4) & 15, (t >> 8) & 15};
     const int i1 = t2[a1] - lo1, i2 = t2[a2] - lo2, tt = t2[a3];
     const int col = i2 * n1 + i1, st = n2 * n1;
@@ -148,19 +160,23 @@ __global__ void __launch_bounds__(IP_THREADS)
     }
 #pragma unroll
     for (int g = 0; g < IP_FG; ++g)
-      if (f0 + g < nf) E[(f0 + g) * es + base + k] = v[g];
+      if (f0 + g < nf) out[(f0 + g) * as + k] = v[g];
   }
+  __syncthreads();   // T1/T2 reused by the next group
+  }  // face groups
 }
 
-void launch_interp(const DevMesh& m, double* E, int nf, cudaStream_t s) {
-  if (m.n_iel <= 0) return;
+void launch_interp(const DevMesh& m, const double* u, int nf, int64_t first, int64_t count,
+                   cudaStream_t s) {
+  if (count <= 0) return;
   const size_t dyn = size_t(IP_FG) * IP_FIELD * sizeof(double);
   static bool attr = false;
   if (!attr) {
     cudaFuncSetAttribute(k_interp, cudaFuncAttributeMaxDynamicSharedMemorySize, int(dyn));
     attr = true;
   }
-  k_interp<<<dim3(m.n_iel, (nf + IP_FG - 1) / IP_FG), IP_THREADS, dyn, s>>>(m, E, nf);
+  k_interp<<<dim3(unsigned(count), (nf + IP_FG - 1) / IP_FG), IP_THREADS, dyn, s>>>(m, u, nf,
+                                                                                    first);
 }
 
 // One CTA per patch, ONE WARP PER FIELD (warp w builds fields w, w+8, w+16):
@@ -168,7 +184,7 @@ void launch_interp(const DevMesh& m, double* E, int nf, cudaStream_t s) {
 // outer-boundary extrapolation along x, y, z (boundary octants only) in three
 // warp-synchronous passes over the patch just written.
 __global__ void __launch_bounds__(UZ_THREADS, 3)
-    k_unzip(DevMesh m, const double* __restrict__ E, double* __restrict__ patches, int nf) {
+    k_unzip(DevMesh m, const double* __restrict__ u, double* __restrict__ patches, int nf) {
   __shared__ int32_t soff[NPATCH];
   __shared__ double WX[21];
   const int e = blockIdx.x;
@@ -181,9 +197,10 @@ __global__ void __launch_bounds__(UZ_THREADS, 3)
   }
   __syncthreads();
 
-  const int64_t nn = m.e_stride;
+  const int64_t ds = m.dof_stride;
   for (int f = warp; f < nf; f += UZ_WARPS) {
-  const double* Ef = E + f * nn;
+  const double* uf = u + f * ds;
+  const double* af = m.aux + f * m.aux_stride - ds;   // slot i - ds
   double* dst = patches + (int64_t(f) * m.n_owned + e) * PATCH_PITCH;
 
   // ---- gather: 16 loads in flight per lane; coalesced streaming (evict-first)
@@ -199,7 +216,8 @@ __global__ void __launch_bounds__(UZ_THREADS, 3)
       o[u] = p < NPATCH ? soff[p] : -3;
       // (volatile asm keeps all U loads ahead of the stores; invalid points load
       // element value 0 and are not stored)
-      asm volatile("ld.global.nc.f64 %0, [%1];" : "=d"(v[u]) : "l"(Ef + max(o[u], 0)));
+      const int x = max(o[u], 0);
+      asm volatile("ld.global.nc.f64 %0, [%1];" : "=d"(v[u]) : "l"((x < ds ? uf : af) + x));
     }
 #pragma unroll
     for (int u = 0; u < U; ++u)
@@ -249,9 +267,9 @@ __global__ void __launch_bounds__(UZ_THREADS, 3)
   }  // field loop
 }
 
-void launch_unzip(const DevMesh& m, const double* E, double* patches, int nf, cudaStream_t s) {
+void launch_unzip(const DevMesh& m, const double* u, double* patches, int nf, cudaStream_t s) {
   if (m.n_owned <= 0) return;
-  k_unzip<<<m.n_owned, UZ_THREADS, 0, s>>>(m, E, patches, nf);
+  k_unzip<<<m.n_owned, UZ_THREADS, 0, s>>>(m, u, patches, nf);
 }
 
 }  // namespace dgr

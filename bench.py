@@ -36,17 +36,20 @@ UNIT = "grid-pts/s"
 # Algorithmic work per unit:
 UNZIP_BYTES_PER_OCT = 24 * (2197 + 216) * 8       # write every patch point, read every DOF once
 ZIP_BYTES_PER_DOF_STAGE = 24 * 34                 # avg over the 4 stages of read k,u_n,acc / write acc,u_s
-ELEM_BYTES_PER_OCT = 24 * 343 * (8 + 8) + 343 * 4  # E write + u gather + O2N read
+INTERP_BYTES_PER_SLOT = 24 * 8                     # write every slot once
+INTERP_BYTES_PER_ELEM = 24 * 343 * 8 + 343 * 4    # read the element's nodal values once (+ o2s)
 RHS_BYTES_PER_OCT = 24 * (2197 + 343) * 8         # patch read + rhs write (eq 21a denominator)
 PAPER_FLOPS_PER_POINT = 5502 + 3998               # eq (21a) numerator per point, O_A from Q_L = 6.68
 # executed fp64 FLOPs per interior point of k_rhs (2 per DFMA + DADD + DMUL), from
-# ncu sm__sass_thread_inst_executed_op_d{fma,add,mul}_pred_on (profiles/)
-# (profiles/r1_ncu_flops.txt: 4.491e10 FLOP per C3 launch / 8,329,412 points = 5,392)
-RHS_EXEC_FLOPS_PER_POINT = float(os.environ.get("DGR_RHS_FLOPS_PER_POINT", "5392"))
+# ncu sm__sass_thread_inst_executed_op_d{fma,add,mul}_pred_on on C3 (profiles/r1c_ncu_flops.csv):
+# fused 2 x 12.991e9 + 11.129e9 + 6.736e9 = 43.85e9 FLOP / 8,329,412 points = 5,265
+# (the in-kernel extrapolation adds ~12 FLOP/pt); two-pass 43.75e9 / 8,329,412 = 5,253
+RHS_EXEC_FLOPS_PER_POINT = {"fused": 5265.0, "two-pass": 5253.0}
 # DRAM bytes per launch (dram__bytes_read.sum + dram__bytes_write.sum) from one
-# ncu --set full capture of the C3 workload on 1 GPU (profiles/r1_ncu_full_c3_kernels.txt)
-NCU_TRAFFIC_C3 = {"rhs": 18.723e9 + 3.207e9, "unzip": 3.261e9 + 10.850e9,
-                  "elements": 1.819e9 + 1.561e9}
+# ncu --set full capture of the C3 workload on 1 GPU, per path
+# (profiles/ncu_traffic_c3.json, written by tools/ncu_traffic.py)
+_TRAFFIC_JSON = os.path.join(ROOT, "profiles", "ncu_traffic_c3.json")
+NCU_TRAFFIC_C3 = json.load(open(_TRAFFIC_JSON)) if os.path.exists(_TRAFFIC_JSON) else {}
 
 
 def _peaks():
@@ -174,6 +177,8 @@ def main():
     ap.add_argument("--impl", default="dgr", choices=["dgr", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=None)
+    ap.add_argument("--path", default="fused", choices=["fused", "two-pass"],
+                    help="fused: patches gathered inside the RHS kernel; two-pass: unzip first")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -200,6 +205,7 @@ def main():
 
     octs = dgr.octree_build(cfg)
     mesh = dgr.Mesh(cfg, octs, rank=rank, nranks=world, nccl_id=nccl_id)
+    mesh.set_fused(args.path == "fused")
     info = mesh.info
     xyz = mesh.dof_xyz_host()
     u = torch.zeros((24, mesh.dof_stride), dtype=torch.float64, device="cuda")
@@ -292,7 +298,8 @@ def main():
         k.update({"bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s",
                   "frac": ach / hbm_peak, "algorithmic_bytes_per_launch": bytes_per_launch})
     hbm("unzip", UNZIP_BYTES_PER_OCT * no)
-    hbm("elements", ELEM_BYTES_PER_OCT * nl)
+    hbm("interp", INTERP_BYTES_PER_SLOT * info["n_interp_slots"] +
+        INTERP_BYTES_PER_ELEM * info["n_interp_elems"])
     hbm("zip_rk4", ZIP_BYTES_PER_DOF_STAGE * info["n_dof_owned"])
     if "rhs" in kern:
         k = kern["rhs"]
@@ -302,7 +309,7 @@ def main():
         k["paper_nominal_tflops"] = nominal
         k["hbm_GBps_algorithmic"] = RHS_BYTES_PER_OCT * no / sec / 1e9
         if RHS_EXEC_FLOPS_PER_POINT:
-            ach = pts * RHS_EXEC_FLOPS_PER_POINT / sec / 1e12
+            ach = pts * RHS_EXEC_FLOPS_PER_POINT[args.path] / sec / 1e12
             k.update({"bound": "alu", "achieved": ach, "peak": fp64_peak, "unit": "TFLOP/s",
                       "frac": ach / fp64_peak, "peak_measured_dfma": dfma_tflops})
         else:
@@ -315,8 +322,8 @@ def main():
         k = kern[dom]
         roof = {"kernel": dom, "bound": k["bound"], "achieved": k["achieved"], "peak": k["peak"],
                 "unit": k["unit"], "frac": k["frac"],
-                "traffic": (NCU_TRAFFIC_C3.get(dom) if cfg.name == "c3" and world == 1
-                            else None),
+                "traffic": (NCU_TRAFFIC_C3.get(args.path, {}).get(dom)
+                            if cfg.name == "c3" and world == 1 else None),
                 "traffic_unit": "bytes per launch (ncu dram read+write)",
                 "peak_source": (f"MEASURED_PEAKS.json ({peak_kind})" if k["bound"] == "hbm" else
                                 "148 SM x 64 DFMA/clk x 2 x sm_max_mhz (derived)")}
@@ -336,7 +343,10 @@ def main():
         "config": {"workload": f"{cfg.name}: {cfg.description}", "octants": info["n_oct_global"],
                    "dofs": n_dof, "unknowns": 24 * n_dof, "levels": [info["level_min"],
                                                                     info["level_max"]],
-                   "dt": dt, "l2": "inputs larger than L2 (10 GB patch buffer per stage)",
+                   "dt": dt, "path": args.path,
+                   "l2": ("inputs larger than L2 (state 0.97 GB + gather maps 0.2 GB + slots "
+                          "streamed every stage"
+                          + (", 10 GB patch buffer per stage)" if args.path == "two-pass" else ")")),
                    "parallelism": f"morton-partition x{world}"},
         "rhs_gflops": (kern.get("rhs", {}).get("achieved", 0) * 1e3) or None,
         "roofline": roof,

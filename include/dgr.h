@@ -125,6 +125,9 @@ typedef struct {
   int64_t n_hanging;     /* hanging (octant, node) pairs over local+ghost    */
   double h_min;          /* finest grid spacing width / (6 * 2^level_max)    */
   int32_t level_min, level_max;
+  int64_t n_interp_slots;  /* interpolation slots (hanging nodes + coarse-neighbour
+                              padding values, deduplicated; device meshes only) */
+  int64_t n_interp_elems;  /* elements whose slots k_interp evaluates          */
 } dgr_mesh_info;
 
 typedef struct dgr_mesh_s* dgr_mesh;
@@ -210,7 +213,7 @@ dgr_status dgr_constraints(dgr_mesh m, double* u, double* c, double* norms_host,
                            const dgr_params* prm, void* stream);
 
 /* Execution options of a mesh (host-side switch, takes effect at the next call):
- *   DGR_OPT_FUSED_UNZIP (default 0): 1 = dgr_rhs / dgr_rk4_* gather every patch
+ *   DGR_OPT_FUSED_UNZIP (default 1): 1 = dgr_rhs / dgr_rk4_* gather every patch
  *     inside the RHS kernel straight from the element values and interpolation
  *     slots (no patch buffer); 0 = unzip into the 13^3 patch
  *     buffer first (Alg. 2), then the RHS reads the patches.

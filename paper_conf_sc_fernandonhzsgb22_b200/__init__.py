@@ -68,7 +68,8 @@ class _Info(C.Structure):
                 ("n_dof_global", C.c_int64), ("n_dof_owned", C.c_int64),
                 ("n_dof_ghost", C.c_int64), ("dof_stride", C.c_int64),
                 ("patch_pitch", C.c_int64), ("n_hanging", C.c_int64), ("h_min", C.c_double),
-                ("level_min", C.c_int32), ("level_max", C.c_int32)]
+                ("level_min", C.c_int32), ("level_max", C.c_int32),
+                ("n_interp_slots", C.c_int64), ("n_interp_elems", C.c_int64)]
 
 
 _lib = None

@@ -7,7 +7,7 @@ from synth import configs, initial
 name = sys.argv[1] if len(sys.argv) > 1 else "c3"
 steps = int(sys.argv[2]) if len(sys.argv) > 2 else 5
 cfg = configs.get(name)
-fused = os.environ.get("DGR_FUSED", "0") != "0"
+fused = os.environ.get("DGR_FUSED", "1") != "0"
 t = time.time(); m = dgr.Mesh(cfg); m.set_fused(fused); print("fused", fused)
 print("mesh", m.info, "%.1fs" % (time.time() - t), flush=True)
 xyz = m.dof_xyz_host()

@@ -59,15 +59,30 @@ __global__ void __launch_bounds__(IP_THREADS)
   double* T1 = Es + IP_FG * NPT;                 // [IP_FG][IP_T1]
   double* T2 = T1 + IP_FG * IP_T1;               // [IP_FG][IP_T2]
   for (int i = tid; i < 91; i += IP_THREADS) W[i] = c_uW13[i];
-  for (int i = tid; i < IP_FG * NPT; i += IP_THREADS) {
-    const int g = i / NPT, n = i - g * NPT;
-    double v = 0.0;
-    if (f0 + g < nf) {
-      const int32_t x = __ldg(m.o2s + int64_t(el.x) * NPT + n);
-      // (slots of coarser elements were written by an earlier launch: plain load)
-      v = x < ds ? __ldg(u + (f0 + g) * ds + x) : m.aux[(f0 + g) * as + (x - ds)];
+  {
+    // all index loads, then all value loads in flight (two memory round trips)
+    constexpr int NIT = (IP_FG * NPT + IP_THREADS - 1) / IP_THREADS;
+    int32_t xs[NIT];
+#pragma unroll
+    for (int it = 0; it < NIT; ++it) {
+      const int i = tid + it * IP_THREADS;
+      const int g = i / NPT, n = i - g * NPT;
+      xs[it] = (i < IP_FG * NPT && f0 + g < nf) ? __ldg(m.o2s + int64_t(el.x) * NPT + n) : -1;
     }
-    Es[i] = v;
+    double v[NIT];
+#pragma unroll
+    for (int it = 0; it < NIT; ++it) {
+      const int i = tid + it * IP_THREADS;
+      const int g = i / NPT;
+      const int32_t x = xs[it];
+      // (slots of coarser elements were written by an earlier launch: plain load)
+      v[it] = x < 0 ? 0.0 : (x < ds ? __ldg(u + (f0 + g) * ds + x) : m.aux[(f0 + g) * as + (x - ds)]);
+    }
+#pragma unroll
+    for (int it = 0; it < NIT; ++it) {
+      const int i = tid + it * IP_THREADS;
+      if (i < IP_FG * NPT) Es[i] = v[it];
+    }
   }
   __syncthreads();
   for (int gi = 0; gi < el.z; ++gi) {

@@ -128,6 +128,9 @@ typedef struct {
   int64_t n_interp_slots;  /* interpolation slots (hanging nodes + coarse-neighbour
                               padding values, deduplicated; device meshes only) */
   int64_t n_interp_elems;  /* elements whose slots k_interp evaluates          */
+  int64_t n_oct_interior;  /* owned octants whose patches need no ghost value
+                              (computed while the ghost exchange is in flight,
+                              SURVEY.md §8e; = n_oct_local on one rank)        */
 } dgr_mesh_info;
 
 typedef struct dgr_mesh_s* dgr_mesh;
@@ -150,7 +153,9 @@ enum {
   DGR_MAP_SEND_COUNTS = 9, /* int64 [nranks]: DOFs sent to each peer               */
   DGR_MAP_RECV_COUNTS = 10, /* int64 [nranks]: ghost DOFs received from each peer  */
   DGR_MAP_LOCAL_OCTS = 11,  /* int32 [n_oct_local + n_oct_ghost]: global octant ids */
-  DGR_MAP_O2N_LOCAL = 12    /* int32 [n_oct_local + n_oct_ghost][343]: local DOF id or -1 */
+  DGR_MAP_O2N_LOCAL = 12,   /* int32 [n_oct_local + n_oct_ghost][343]: local DOF id or -1 */
+  DGR_MAP_RHS_ORDER = 13    /* int32 [n_oct_local]: owned octants (local ids) in RHS order,
+                               the first n_oct_interior need no ghost value (device meshes) */
 };
 
 const char* dgr_status_string(dgr_status s);
@@ -218,7 +223,12 @@ dgr_status dgr_constraints(dgr_mesh m, double* u, double* c, double* norms_host,
  *     slots (no patch buffer); 0 = unzip into the 13^3 patch
  *     buffer first (Alg. 2), then the RHS reads the patches.
  *     Both give bit-identical results. */
-enum { DGR_OPT_FUSED_UNZIP = 1 };
+/*   DGR_OPT_PHASES (default 0): how the fused path orders the owned octants.
+ *     0 = interior octants overlap the ghost exchange when there is a
+ *     communicator, else one pass; 1 = always run the interior octants (and the
+ *     slots they need) first, then the rest; 2 = interior octants only (test
+ *     hook: boundary octants' RHS is not computed). */
+enum { DGR_OPT_FUSED_UNZIP = 1, DGR_OPT_PHASES = 2 };
 dgr_status dgr_set_option(dgr_mesh m, int option, int64_t value);
 
 /* Device-side timing helper for benchmarks: number of kernel launches the last

@@ -26,8 +26,8 @@ NPATCH = 2197
 
 MAP_OCTANTS, MAP_O2N, MAP_HANGING, MAP_PAD_SRC, MAP_PAD_KIND, MAP_ZIP = 0, 1, 2, 3, 4, 5
 MAP_DOF_GID, MAP_DOF_XYZ, MAP_SEND, MAP_SEND_COUNTS, MAP_RECV_COUNTS = 6, 7, 8, 9, 10
-MAP_LOCAL_OCTS, MAP_O2N_LOCAL = 11, 12
-OPT_FUSED_UNZIP = 1
+MAP_LOCAL_OCTS, MAP_O2N_LOCAL, MAP_RHS_ORDER = 11, 12, 13
+OPT_FUSED_UNZIP, OPT_PHASES = 1, 2
 
 
 class DgrError(RuntimeError):
@@ -69,7 +69,8 @@ class _Info(C.Structure):
                 ("n_dof_ghost", C.c_int64), ("dof_stride", C.c_int64),
                 ("patch_pitch", C.c_int64), ("n_hanging", C.c_int64), ("h_min", C.c_double),
                 ("level_min", C.c_int32), ("level_max", C.c_int32),
-                ("n_interp_slots", C.c_int64), ("n_interp_elems", C.c_int64)]
+                ("n_interp_slots", C.c_int64), ("n_interp_elems", C.c_int64),
+                ("n_oct_interior", C.c_int64)]
 
 
 _lib = None
@@ -300,6 +301,17 @@ class Mesh:
         """DGR_OPT_FUSED_UNZIP: gather patches inside the RHS kernel (1) or unzip into
         the patch buffer first (0); bit-identical results."""
         _check(lib().dgr_set_option(self._h, OPT_FUSED_UNZIP, int(bool(on))))
+
+    def set_phases(self, mode=0):
+        """DGR_OPT_PHASES: 0 = overlap interior octants with the ghost exchange when
+        there is a communicator; 1 = interior octants first, then the rest;
+        2 = interior octants only (test hook)."""
+        _check(lib().dgr_set_option(self._h, OPT_PHASES, int(mode)))
+
+    def rhs_order(self):
+        """Owned octants (local ids) in RHS order; the first info['n_oct_interior']
+        need no ghost value."""
+        return self.export(MAP_RHS_ORDER, np.int32)
 
     def profile_enable(self, on=True):
         _check(lib().dgr_profile_enable(self._h, int(on)))

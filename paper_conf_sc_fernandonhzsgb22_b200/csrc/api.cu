@@ -100,7 +100,18 @@ struct dgr_mesh_s {
   double* d_aux = nullptr;      // [24][aux_stride] interpolation slots
   int32_t* d_o2s = nullptr;     // [n_local][343] element node -> u / slot index
   int32_t* d_gmap = nullptr;    // [n_owned][GM_PITCH] patch point -> u / slot index
-  std::vector<int64_t> iel_depth_off;   // k_interp launch ranges, one per depth
+  // k_interp launch ranges, one per dependency depth, per phase: phase 0 =
+  // slot elements whose values depend on owned DOFs only, phase 1 = the rest
+  // (they wait for the ghost exchange; empty on one rank)
+  std::vector<int64_t> iel_depth_off[2];
+  // RHS octant order: olist[0, n_interior) need no ghost value (they run while
+  // the ghost exchange is in flight), olist[n_interior, n_owned) the rest
+  int32_t* d_olist = nullptr;
+  int64_t n_interior = 0;
+  cudaStream_t xstream = nullptr;   // ghost exchange stream (N > 1)
+  int xsm = 8;                      // SMs k_rhs leaves to NCCL while overlapping
+  int phases = 0;                   // DGR_OPT_PHASES
+  cudaEvent_t ev_ready = nullptr, ev_xdone = nullptr;
   int4* d_iel = nullptr;        // interpolation work per element with slots
   int4* d_igrp = nullptr;       // ... per face group of its slots
   uint16_t* d_ipt = nullptr;    // half-grid point of each interpolation slot
@@ -146,6 +157,9 @@ struct dgr_mesh_s {
     for (auto e : pool) cudaEventDestroy(e);
     for (void* q : allocs) cudaFree(q);
     if (comm && g_nccl.CommDestroy) g_nccl.CommDestroy(comm);
+    if (ev_ready) cudaEventDestroy(ev_ready);
+    if (ev_xdone) cudaEventDestroy(ev_xdone);
+    if (xstream) cudaStreamDestroy(xstream);
   }
 };
 
@@ -340,19 +354,41 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
       }
       edepth[c] = d;
     }
+    // remote dependency: a slot element needs a ghost value if one of its
+    // nodes is a ghost DOF or a slot of such an element (coarse to fine)
+    std::vector<uint8_t> erdep(size_t(nl), 0);
+    for (int32_t ci : order) {
+      const int32_t c = celem[ci];
+      uint8_t r = 0;
+      for (int n = 0; n < NPT && !r; ++n) {
+        const size_t k = size_t(c) * NPT + n;
+        const int32_t d = h.o2n_local[k];
+        r = d >= 0 ? uint8_t(d >= h.n_owned_dof) : erdep[hsrc[k]];
+      }
+      erdep[c] = r;
+    }
     std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) {
+      const int32_t pa = erdep[celem[a]], pb = erdep[celem[b]];
+      if (pa != pb) return pa < pb;
       const int32_t da = edepth[celem[a]], db = edepth[celem[b]];
       return da != db ? da < db : celem[a] < celem[b];
     });
     std::vector<int4> iel, igrp;
     std::vector<uint16_t> ipt;
-    m->iel_depth_off.clear();
+    m->iel_depth_off[0].clear();
+    m->iel_depth_off[1].clear();
+    std::vector<uint8_t> slot_rdep;
     int64_t slot = 0;
-    int prev_depth = -1;
+    int prev_depth = -1, prev_phase = 0;
     for (int32_t ci : order) {
       const int32_t c = celem[ci];
+      if (erdep[c] != prev_phase) {   // phase 0 -> 1
+        m->iel_depth_off[0].push_back(int64_t(iel.size()));
+        prev_phase = erdep[c];
+        prev_depth = -1;
+      }
       if (edepth[c] != prev_depth) {
-        m->iel_depth_off.push_back(int64_t(iel.size()));
+        m->iel_depth_off[prev_phase].push_back(int64_t(iel.size()));
         prev_depth = edepth[c];
       }
       // one work entry per (element, face group): a slot belongs to the first
@@ -387,8 +423,9 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
         igrp.push_back(make_int4(int32_t(first), int32_t(slot - first), lohi, 0));
       }
       iel.push_back(make_int4(c, g_first, int32_t(igrp.size()) - g_first, 0));
+      slot_rdep.resize(size_t(slot), erdep[c]);
     }
-    m->iel_depth_off.push_back(int64_t(iel.size()));
+    m->iel_depth_off[prev_phase].push_back(int64_t(iel.size()));
     if (ds + slot >= (int64_t(1) << 31)) return fail(DGR_ERR_ARG, "mesh too large for int32 gather maps");
     // element nodes -> u / slot index
     std::vector<int32_t> o2s(size_t(nl) * NPT);
@@ -427,6 +464,27 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
         }
         gm[size_t(e) * GM_PITCH + p] = v;
       }
+    }
+    // interior octants first (no gather source depends on a ghost value)
+    {
+      std::vector<int32_t> olist;
+      olist.reserve(size_t(no));
+      std::vector<int32_t> bnd;
+      for (int64_t e = 0; e < no; ++e) {
+        bool remote = false;
+        const int32_t* row = gm.data() + size_t(e) * GM_PITCH;
+        for (int p = 0; p < NPATCH && !remote; ++p) {
+          const int32_t v = row[p];
+          if (v < 0) continue;
+          remote = v < ds ? v >= h.n_owned_dof : slot_rdep[size_t(v - ds)] != 0;
+        }
+        (remote ? bnd : olist).push_back(int32_t(e));
+      }
+      m->n_interior = int64_t(olist.size());
+      olist.insert(olist.end(), bnd.begin(), bnd.end());
+      CUDA_TRY(m->alloc(&m->d_olist, olist.size()));
+      if (!olist.empty())
+        CUDA_TRY(cudaMemcpy(m->d_olist, olist.data(), olist.size() * 4, cudaMemcpyHostToDevice));
     }
     m->n_interp = slot;
     aux_stride = std::max<int64_t>(32, ((slot + 31) / 32) * 32);
@@ -475,6 +533,7 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
   dm.aux = m->d_aux;
   dm.o2s = m->d_o2s;
   dm.gmap = m->d_gmap;
+  dm.olist = m->d_olist;
   dm.iel = m->d_iel;
   dm.igrp = m->d_igrp;
   dm.ipt = m->d_ipt;
@@ -547,6 +606,7 @@ dgr_status dgr_mesh_info_get(dgr_mesh m, dgr_mesh_info* info) {
   info->h_min = h.width / (6.0 * std::ldexp(1.0, h.level_max));
   info->n_interp_slots = m->n_interp;
   info->n_interp_elems = m->dm.n_iel;
+  info->n_oct_interior = m->device ? m->n_interior : h.n_owned_oct;
   return DGR_OK;
 }
 
@@ -625,6 +685,15 @@ dgr_status dgr_mesh_export_maps(dgr_mesh m, int which, void* host_buf, size_t* n
       return put(h.local_oct.data(), h.local_oct.size() * 4);
     case DGR_MAP_O2N_LOCAL:
       return put(h.o2n_local.data(), h.o2n_local.size() * 4);
+    case DGR_MAP_RHS_ORDER: {
+      if (!m->device) return fail(DGR_ERR_STATE, "RHS order exists on device meshes only");
+      std::vector<int32_t> v(static_cast<size_t>(no));
+      if (no) {
+        cudaError_t e = cudaMemcpy(v.data(), m->d_olist, size_t(no) * 4, cudaMemcpyDeviceToHost);
+        if (e != cudaSuccess) return fail(DGR_ERR_CUDA, cudaGetErrorString(e));
+      }
+      return put(v.data(), v.size() * 4);
+    }
   }
   return fail(DGR_ERR_ARG, "unknown map id");
 }
@@ -691,10 +760,13 @@ static dgr_status exchange(dgr_mesh m, double* u, cudaStream_t st) {
 
 // interpolation slots (hanging nodes and coarse-neighbour padding values,
 // Alg. 2 lines 4-5 and P:L295), one k_interp launch per dependency depth
-static dgr_status do_interp(dgr_mesh m, const double* u, int nf, cudaStream_t st) {
-  for (size_t g = 0; g + 1 < m->iel_depth_off.size(); ++g) {
-    const int64_t a = m->iel_depth_off[g], b = m->iel_depth_off[g + 1];
-    PROF(m, 7, st, launch_interp(m->dm, u, nf, a, b - a, st));
+// (phase 0: slot elements that need owned DOFs only; 1: the rest; -1: both)
+static dgr_status do_interp(dgr_mesh m, const double* u, int nf, cudaStream_t st, int phase = -1) {
+  for (int ph = 0; ph < 2; ++ph) {
+    if (phase >= 0 && ph != phase) continue;
+    const std::vector<int64_t>& off = m->iel_depth_off[ph];
+    for (size_t g = 0; g + 1 < off.size(); ++g)
+      if (off[g + 1] > off[g]) PROF(m, 7, st, launch_interp(m->dm, u, nf, off[g], off[g + 1] - off[g], st));
   }
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;
@@ -719,16 +791,55 @@ static RhsParams to_rp(const dgr_params* p) {
   return r;
 }
 
-// RHS of every owned octant's interior points into d_rhs_oct, by the fused
-// path (patches gathered inside k_rhs) or through the explicit patch buffer
-static dgr_status rhs_oct(dgr_mesh m, const double* u, const dgr_params* prm, cudaStream_t st) {
+// Ghost exchange + RHS of every owned octant's interior points into d_rhs_oct,
+// by the fused path (patches gathered inside k_rhs) or through the explicit
+// patch buffer.  With a communicator (N > 1) the fused path overlaps the
+// exchange with the interior octants: the pack + NCCL group runs
+// on its own stream while k_interp (phase 0) and k_rhs work through the
+// octants whose patches need no ghost value — k_rhs then leaves a few SMs
+// free, since it otherwise holds every SM and the NCCL kernels could not
+// start — and the boundary octants follow once the ghosts have landed.
+static dgr_status rhs_oct(dgr_mesh m, double* u, const dgr_params* prm, cudaStream_t st) {
   dgr_status s;
-  if (m->fused) {
-    if ((s = do_interp(m, u, NF, st))) return s;
-    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, to_rp(prm), nullptr, true, st));
-  } else {
+  const int64_t no = m->dm.n_owned, ni = m->n_interior;
+  const RhsParams rp = to_rp(prm);
+  if (!m->fused) {
+    if ((s = exchange(m, u, st))) return s;
     if ((s = do_unzip(m, u, NF, st))) return s;
-    PROF(m, 3, st, launch_rhs(m->dm, m->d_patch, m->d_rhs_oct, to_rp(prm), nullptr, false, st));
+    PROF(m, 3, st, launch_rhs(m->dm, m->d_patch, m->d_rhs_oct, rp, false, 0, no, 0, st));
+    CUDA_TRY(cudaGetLastError());
+    return DGR_OK;
+  }
+  const bool overlap = m->host.nranks > 1 && m->comm && ni > 0 && ni < no && m->phases == 0;
+  if (m->phases > 0) {
+    // interior octants and the slots they need first, then (unless the test
+    // hook stops here) the rest — no stream overlap
+    if ((s = exchange(m, u, st))) return s;
+    if ((s = do_interp(m, u, NF, st, 0))) return s;
+    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, ni, 0, st));
+    if (m->phases == 1) {
+      if ((s = do_interp(m, u, NF, st, 1))) return s;
+      PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, ni, no - ni, 0, st));
+    }
+  } else if (overlap) {
+    if (!m->xstream) {
+      CUDA_TRY(cudaStreamCreateWithFlags(&m->xstream, cudaStreamNonBlocking));
+      CUDA_TRY(cudaEventCreateWithFlags(&m->ev_ready, cudaEventDisableTiming));
+      CUDA_TRY(cudaEventCreateWithFlags(&m->ev_xdone, cudaEventDisableTiming));
+    }
+    CUDA_TRY(cudaEventRecord(m->ev_ready, st));
+    CUDA_TRY(cudaStreamWaitEvent(m->xstream, m->ev_ready, 0));
+    if ((s = exchange(m, u, m->xstream))) return s;
+    CUDA_TRY(cudaEventRecord(m->ev_xdone, m->xstream));
+    if ((s = do_interp(m, u, NF, st, 0))) return s;
+    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, ni, m->xsm, st));
+    CUDA_TRY(cudaStreamWaitEvent(st, m->ev_xdone, 0));
+    if ((s = do_interp(m, u, NF, st, 1))) return s;
+    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, ni, no - ni, 0, st));
+  } else {
+    if ((s = exchange(m, u, st))) return s;
+    if ((s = do_interp(m, u, NF, st))) return s;
+    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, no, 0, st));
   }
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;
@@ -773,7 +884,7 @@ dgr_status dgr_rhs_patches(dgr_mesh m, const double* patches, double* rhs_oct,
   if (s) return s;
   if (!patches || !rhs_oct || !aligned16(patches)) return fail(DGR_ERR_ARG, "bad rhs args");
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  PROF(m, 3, st, launch_rhs(m->dm, patches, rhs_oct, to_rp(prm), nullptr, false, st));
+  PROF(m, 3, st, launch_rhs(m->dm, patches, rhs_oct, to_rp(prm), false, 0, m->dm.n_owned, 0, st));
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;
 }
@@ -784,7 +895,6 @@ dgr_status dgr_rhs(dgr_mesh m, double* u, double* rhs, const dgr_params* prm, vo
   if (!u || !rhs) return fail(DGR_ERR_ARG, "null state");
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   m->launches = 0;
-  if ((s = exchange(m, u, st))) return s;
   if ((s = rhs_oct(m, u, prm, st))) return s;
   PROF(m, 4, st, launch_zip(m->dm, m->d_rhs_oct, rhs, NF, st));
   CUDA_TRY(cudaGetLastError());
@@ -795,10 +905,9 @@ static dgr_status stage(dgr_mesh m, int s_, double dt, double* u_n, double* u_s,
                         double* u_out, const dgr_params* prm, cudaStream_t st) {
   dgr_status s;
   double* cur = s_ == 0 ? u_n : u_s;
-  if ((s = exchange(m, cur, st))) return s;
-  // (k_rhs can also apply the zip + RK4 update in its epilogue (RkArgs); on C3
-  // that measured 10.6 ms vs 7.5 + 0.8 ms for RHS + k_zip_rk4 — the scattered
-  // state loads stall the single persistent CTA per SM — so it is not used)
+  // (applying the zip + RK4 update inside k_rhs measured 10.6 ms vs 7.5 + 0.8 ms
+  // for RHS + k_zip_rk4 on C3 — the scattered state loads stall the single
+  // persistent CTA per SM — so the update is a separate kernel)
   if ((s = rhs_oct(m, cur, prm, st))) return s;
   PROF(m, 4, st, launch_zip_rk4(m->dm, m->d_rhs_oct, s_, dt, u_n, u_s, acc, u_out, st));
   CUDA_TRY(cudaGetLastError());
@@ -891,6 +1000,10 @@ dgr_status dgr_set_option(dgr_mesh m, int option, int64_t value) {
   if (!m) return fail(DGR_ERR_ARG, "null mesh");
   switch (option) {
     case DGR_OPT_FUSED_UNZIP: m->fused = value != 0; return DGR_OK;
+    case DGR_OPT_PHASES:
+      if (value < 0 || value > 2) return fail(DGR_ERR_ARG, "DGR_OPT_PHASES is 0, 1 or 2");
+      m->phases = int(value);
+      return DGR_OK;
   }
   return fail(DGR_ERR_ARG, "unknown option");
 }

@@ -37,6 +37,9 @@ struct DevMesh {
   // gmap[e][p]: index of patch point p of owned octant e, -1 outside a
   // non-periodic domain (extrapolated)
   const int32_t* gmap;      // [n_owned * GM_PITCH]
+  // RHS octant order: interior octants (no ghost-dependent gather source)
+  // first, then the boundary octants (api.cu, overlap of the ghost exchange)
+  const int32_t* olist;     // [n_owned]
   // interpolation work: one entry per element with slots (sorted by dependency
   // depth) {element, first group, group count, 0}, and per face group of its
   // slots {first slot, slot count, bbox lo (x|y<<4|z<<8) | hi << 12 | first
@@ -69,22 +72,13 @@ void launch_dfma(int blocks, int iters, double* out, cudaStream_t s);
 struct RhsParams {
   double ko_sigma, eta, lambda_f0, lambda_f1, chi_floor;
 };
-// Fused patch-to-octant + RK4 stage in the RHS epilogue (s < 0: write rhs_oct).
-struct RkArgs {
-  int s;
-  double dt;
-  const double* u_n;
-  double* u_s;
-  double* acc;
-  double* u_out;
-  const int32_t* own;   // [n_owned * 343]: owned DOF this point is the zip owner of, or -1
-  int64_t stride;
-};
 // fused = false: read 13^3 patches ([24][n_owned][PATCH_PITCH], TMA bulk copies);
 // fused = true: `src` is the state u; every patch is gathered from u and the
 // slots through gmap (no patch buffer)
+// RHS of the owned octants m.olist[first, first + count); at most
+// n_SM - leave_sm persistent CTAs
 void launch_rhs(const DevMesh& m, const double* src, double* rhs_oct, const RhsParams& p,
-                const RkArgs* rk, bool fused, cudaStream_t s);
+                bool fused, int64_t first, int64_t count, int leave_sm, cudaStream_t s);
 size_t rhs_smem_bytes();
 void upload_rhs_tables(const double* wext);
 

@@ -235,7 +235,7 @@ __device__ __forceinline__ double trace6(const double* gi, const double* X) {
 template <bool FUSED>
 __global__ void __launch_bounds__(RT, 1)
     k_rhs(DevMesh m, const double* __restrict__ patches, double* __restrict__ rhs_oct,
-          RhsParams prm, RkArgs rk) {
+          RhsParams prm, int first, int count) {
   extern __shared__ __align__(128) double smem[];
   double* slots = smem;                           // [NSLOT][NPP]
   double* stage = smem + NSLOT * NPP;             // [2][STAGE_DBL]
@@ -292,8 +292,12 @@ __global__ void __launch_bounds__(RT, 1)
   // (double-buffered bulk copies, mbarrier phase = global stage count) runs
   // on across octant boundaries, and the next octant's 24 field patches are
   // prefetched into L2 one octant ahead.
-  int e = blockIdx.x;
-  if (e >= no) return;
+  // (octant list m.olist[first, first + count): interior octants before the
+  // ones that wait for ghost values, api.cu)
+  const int32_t* ol = m.olist + first;
+  int li = blockIdx.x;
+  if (li >= count) return;
+  int e = ol[li];
   if (tid == 0) {
     mbar_init(&bars[0], 1);
     mbar_init(&bars[1], 1);
@@ -311,8 +315,9 @@ __global__ void __launch_bounds__(RT, 1)
     prefetch_l2(patches + int64_t(e) * PATCH_PITCH + c_order[tid + 1] * fstride);
   }
   uint32_t g = 0;   // global stage counter of this CTA
-  for (; e < no; e += gridDim.x) {
-  const int en = e + gridDim.x;                    // next octant of this CTA
+  for (; li < count; li += gridDim.x) {
+  e = ol[li];
+  const int en = li + int(gridDim.x) < count ? ol[li + gridDim.x] : -1;   // next octant of this CTA
   const double* pbase = patches + int64_t(e) * (FUSED ? NPT : PATCH_PITCH);
   const bool active = tab_c0[tid] >= 0;
   // the point's own values: patch index c0 of the staged patches, or (FUSED)
@@ -333,7 +338,7 @@ __global__ void __launch_bounds__(RT, 1)
             ((oi.y + sd == nside) << 4) | ((oi.z + sd == nside) << 5);
   }
   const bool bnd = omask != 0;
-  if (FUSED && en < no && tid == 32)   // next octant's gather map into L2
+  if (FUSED && en >= 0 && tid == 32)   // next octant's gather map into L2
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(m.gmap + int64_t(en) * GM_PITCH),
                  "r"(uint32_t(GM_PITCH * 4))
                  : "memory");
@@ -763,8 +768,8 @@ __global__ void __launch_bounds__(RT, 1)
       if (st + 2 < NF) {
         gather(dst, c_order[st + 2]);
       } else {
-        if (st + 2 == NF && en < no) load_gidx(en);   // the current octant's gathers are issued
-        if (en < no) gather(dst, c_order[st + 2 - NF]);
+        if (st + 2 == NF && en >= 0) load_gidx(en);   // the current octant's gathers are issued
+        if (en >= 0) gather(dst, c_order[st + 2 - NF]);
         else cp_async_commit();                        // (empty group keeps the count uniform)
       }
       continue;
@@ -772,13 +777,13 @@ __global__ void __launch_bounds__(RT, 1)
     // L2 prefetch one octant ahead: the next octant's field of this stage
     // (measured faster than prefetching the current octant at its start,
     // although some prefetched lines are evicted and re-read)
-    if (tid == 32 && en < no)
+    if (tid == 32 && en >= 0)
       prefetch_l2(patches + int64_t(en) * PATCH_PITCH + c_order[st] * fstride);
     if (tid == 0) {
       if (st + 2 < NF)
         bulk_load(stage + buf * STAGE_DBL, pbase + c_order[st + 2] * fstride, STAGE_DBL * 8,
                   &bars[buf]);
-      else if (en < no)   // the stream continues with the next octant's first fields
+      else if (en >= 0)   // the stream continues with the next octant's first fields
         bulk_load(stage + buf * STAGE_DBL,
                   patches + int64_t(en) * PATCH_PITCH + c_order[st + 2 - NF] * fstride,
                   STAGE_DBL * 8, &bars[buf]);
@@ -843,37 +848,10 @@ __global__ void __launch_bounds__(RT, 1)
                             At[sidx(i, 2)] * Am[2][j];
         r[18 + q] = SL(A_AT + q) + alpha * (Kv * At[q] - 2.0 * AAij);             // (6)
       }
-    if (rk.s < 0) {
-      double* out = rhs_oct + int64_t(e) * NPT + p;
-      const int64_t ostr = no * NPT;
+    double* out = rhs_oct + int64_t(e) * NPT + p;
+    const int64_t ostr = no * NPT;
 #pragma unroll
-      for (int f = 0; f < NF; ++f) out[f * ostr] = r[f];
-    } else {
-      // fused patch-to-octant + RK4 stage (same arithmetic as k_zip_rk4): only
-      // the zip owner of a DOF updates it
-      const int d = __ldg(rk.own + int64_t(e) * NPT + p);
-      if (d >= 0) {
-        const double dt = rk.dt;
-#pragma unroll
-        for (int f = 0; f < NF; ++f) {
-          const int64_t i = f * rk.stride + d;
-          const double k = r[f];
-          if (rk.s == 0) {
-            const double un = rk.u_n[i];
-            rk.acc[i] = un + (dt / 6.0) * k;
-            rk.u_s[i] = un + (dt / 2.0) * k;
-          } else if (rk.s == 1) {
-            rk.acc[i] += (dt / 3.0) * k;
-            rk.u_s[i] = rk.u_n[i] + (dt / 2.0) * k;
-          } else if (rk.s == 2) {
-            rk.acc[i] += (dt / 3.0) * k;
-            rk.u_s[i] = rk.u_n[i] + dt * k;
-          } else {
-            rk.u_out[i] = rk.acc[i] + (dt / 6.0) * k;
-          }
-        }
-      }
-    }
+    for (int f = 0; f < NF; ++f) out[f * ostr] = r[f];
   }
   }  // octant loop
 #undef SL
@@ -914,8 +892,8 @@ void upload_rhs_tables(const double* wext) {
 }
 
 void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const RhsParams& p,
-                const RkArgs* rk, bool fused, cudaStream_t s) {
-  if (m.n_owned <= 0) return;
+                bool fused, int64_t first, int64_t count, int leave_sm, cudaStream_t s) {
+  if (count <= 0) return;
   static int n_sm = 0;
   if (!n_sm) {
     cudaFuncSetAttribute(k_rhs<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(SMEM_BYTES));
@@ -926,14 +904,12 @@ void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const 
     if (n_sm <= 0) n_sm = 148;
   }
   // persistent: one CTA per SM (225 KB of shared memory each)
-  const int grid = m.n_owned < n_sm ? m.n_owned : n_sm;
-  RkArgs a{};
-  a.s = -1;
-  if (rk) a = *rk;
+  const int64_t cap = leave_sm > 0 && n_sm - leave_sm > 0 ? n_sm - leave_sm : n_sm;
+  const int grid = int(count < cap ? count : cap);
   if (fused)
-    k_rhs<true><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a);
+    k_rhs<true><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, int(first), int(count));
   else
-    k_rhs<false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a);
+    k_rhs<false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, int(first), int(count));
 }
 
 }  // namespace dgr

@@ -41,8 +41,8 @@ def _exchange(meshes, states, lists):
             states[peer][:, goff:goff + n] = states[r][:, ids]
 
 
-@pytest.mark.parametrize("world", [2, 3])
-def test_multirank_bit_identical(world):
+@pytest.mark.parametrize("world,phases", [(2, 0), (3, 0), (2, 1)])
+def test_multirank_bit_identical(world, phases):
     need_gpu()
     cfg = configs.small_bbh(lmax=6, rho=0.5)
     om = OracleMesh(cfg)
@@ -54,6 +54,7 @@ def test_multirank_bit_identical(world):
     meshes, states, lists, gids = [], [], [], []
     for r in range(world):
         m = dgr.Mesh(cfg, rank=r, nranks=world)
+        m.set_phases(phases)   # 1: interior octants first, then the boundary ones
         gid = m.export(dgr.MAP_DOF_GID, np.int64)
         st = torch.zeros((NF, m.dof_stride), dtype=torch.float64, device="cuda")
         st[:, :len(gid)] = torch.from_numpy(u[:, gid])
@@ -84,3 +85,38 @@ def test_multirank_bit_identical(world):
         no = meshes[r].info["n_dof_owned"]
         got = states[r][:, :no].cpu().numpy()
         assert np.array_equal(got, full[:, gids[r][:no]]), f"rank {r} differs"
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_interior_octants_need_no_ghost_values(world):
+    """The octants the fused path runs while the ghost exchange is in flight
+    (SURVEY §8e overlap) must not read any ghost value: with every ghost DOF set
+    to NaN and only the interior phase executed (DGR_OPT_PHASES = 2), the RHS at
+    every DOF whose zip owner is an interior octant is finite and bit-identical
+    to the single-rank RHS."""
+    need_gpu()
+    cfg = configs.small_bbh(lmax=6, rho=0.5)
+    om = OracleMesh(cfg)
+    om.build_dofs()
+    u = initial.for_config(cfg, om.dof_coords())
+    ref = dgr.Mesh(cfg)
+    rfull = ref.rhs(to_dev(u, ref.dof_stride))[:, :om.n_dof].cpu().numpy()
+    for r in range(world):
+        m = dgr.Mesh(cfg, rank=r, nranks=world)
+        no_oct, ni = m.info["n_oct_local"], m.info["n_oct_interior"]
+        order = m.rhs_order()
+        assert sorted(order.tolist()) == list(range(no_oct))
+        assert 0 < ni < no_oct, (ni, no_oct)
+        gid = m.export(dgr.MAP_DOF_GID, np.int64)
+        n_own = m.info["n_dof_owned"]
+        st = torch.full((NF, m.dof_stride), float("nan"), dtype=torch.float64, device="cuda")
+        st[:, :n_own] = torch.from_numpy(u[:, gid[:n_own]])
+        m.set_phases(2)
+        got = m.rhs(st)[:, :n_own].cpu().numpy()
+        # zip owner (global leaf) of each owned DOF -> local octant id
+        g2l = {g: l for l, g in enumerate(m.export(dgr.MAP_LOCAL_OCTS, np.int32).tolist())}
+        owner = np.array([g2l[g] for g in m.export(dgr.MAP_ZIP, np.int32).reshape(-1, 2)[:, 0]])
+        sel = np.isin(owner, order[:ni])
+        assert sel.sum() > 0
+        assert np.isfinite(got[:, sel]).all(), f"rank {r}: an interior octant read a ghost value"
+        assert np.array_equal(got[:, sel], rfull[:, gid[:n_own]][:, sel]), f"rank {r} differs"

@@ -103,13 +103,17 @@ typedef struct {
                              itself (DGR_MAP_SEND / _COUNTS) before each stage */
 } dgr_mesh_desc;
 
-/* Parameters of the RHS (readings R6, R8, R13). */
+/* Parameters of the RHS (readings R6, R8, R13, R29). */
 typedef struct {
   double ko_sigma;   /* Kreiss-Oliger strength sigma (0.4)                  */
   double eta;        /* Gamma-driver damping eta (2.0), eq (3)              */
   double lambda_f0;  /* f(alpha) = lambda_f0 + lambda_f1 alpha, eq (2) (1,0) */
   double lambda_f1;
   double chi_floor;  /* chi in every division is max(chi, chi_floor) (1e-4) */
+  int32_t sommerfeld; /* 1: radiative outer boundary at the DOFs on the faces of a
+                         non-periodic domain, d_t f = -(x^i/r) d_i f - (f - f_inf)/r
+                         (reading R29; PAPER.md is silent); 0: none (default) */
+  int32_t reserved;   /* 0 */
 } dgr_params;
 
 typedef struct {

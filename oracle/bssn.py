@@ -37,6 +37,7 @@ class Params:
     lambda_f0: float = 1.0
     lambda_f1: float = 0.0
     chi_floor: float = 1e-4
+    sommerfeld: int = 0        # 1: radiative outer boundary (oracle/boundary.py, R29)
 
 
 def sym_to_full(v):

@@ -16,6 +16,7 @@ import os
 
 import numpy as np
 
+from .boundary import apply_sommerfeld
 from .bssn import NF, Params, rhs_patches
 from .maps import OracleMesh
 from .unzip import elements, padding_sources_cached, unzip, unzip_from_elements, zip_rhs
@@ -39,6 +40,8 @@ def rhs_dofs(mesh: OracleMesh, u: np.ndarray, prm: Params, workers=None) -> np.n
     if workers <= 1 or mesh.n_oct < 4 * workers:
         P = unzip(mesh, u)
         r = rhs_patches(P, octant_h(mesh), prm)
+        if prm.sommerfeld:
+            r = apply_sommerfeld(mesh, np.arange(mesh.n_oct), P, r)
         return zip_rhs(mesh, r.reshape(NF, mesh.n_oct, 343))
     E = elements(mesh, u)
     padding_sources_cached(mesh, np.arange(1))          # fill the cache before forking
@@ -66,6 +69,8 @@ def _chunk_rhs(ab):
     with threadpool_limits(limits=1):
         P = unzip_from_elements(mesh, E, octs)
         r = rhs_patches(P, octant_h(mesh)[octs], prm)
+        if prm.sommerfeld:
+            r = apply_sommerfeld(mesh, octs, P, r)
     return a, r.reshape(NF, len(octs), 343)
 
 

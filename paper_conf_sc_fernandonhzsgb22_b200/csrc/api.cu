@@ -524,6 +524,7 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
   dm.D = h.D;
   dm.periodic = h.periodic ? 1 : 0;
   dm.width = h.width;
+  for (int a = 0; a < 3; ++a) dm.xmin[a] = h.xmin[a];
   dm.oct = m->d_oct;
   dm.o2n = m->d_o2n;
   dm.pmap = m->d_pmap;
@@ -786,8 +787,8 @@ static dgr_status do_unzip(dgr_mesh m, const double* u, int nf, cudaStream_t st)
 }
 
 static RhsParams to_rp(const dgr_params* p) {
-  RhsParams r{0.4, 2.0, 1.0, 0.0, 1e-4};
-  if (p) r = {p->ko_sigma, p->eta, p->lambda_f0, p->lambda_f1, p->chi_floor};
+  RhsParams r{0.4, 2.0, 1.0, 0.0, 1e-4, 0};
+  if (p) r = {p->ko_sigma, p->eta, p->lambda_f0, p->lambda_f1, p->chi_floor, p->sommerfeld != 0};
   return r;
 }
 

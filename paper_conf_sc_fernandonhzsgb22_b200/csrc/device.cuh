@@ -21,6 +21,7 @@ struct DevMesh {
   int32_t D;
   int32_t periodic;
   double width;
+  double xmin[3];           // physical coordinates of the domain corner
   const int4* oct;          // [n_local] anchor x,y,z, level
   const int32_t* o2n;       // [n_local * 343] local DOF id or -1
   const uint8_t* pmap;      // [n_owned * 2197]
@@ -71,6 +72,7 @@ void launch_dfma(int blocks, int iters, double* out, cudaStream_t s);
 // rhs_kernel.cu
 struct RhsParams {
   double ko_sigma, eta, lambda_f0, lambda_f1, chi_floor;
+  int sommerfeld;   // radiative outer boundary (reading R29)
 };
 // fused = false: read 13^3 patches ([24][n_owned][PATCH_PITCH], TMA bulk copies);
 // fused = true: `src` is the state u; every patch is gathered from u and the

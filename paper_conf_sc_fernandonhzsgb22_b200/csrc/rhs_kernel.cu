@@ -232,7 +232,9 @@ __device__ __forceinline__ double trace6(const double* gi, const double* X) {
 // 8-byte cp.async (the unzip fused into the RHS), and
 // points outside a non-periodic domain are extrapolated in shared memory with
 // the same arithmetic as k_unzip.
-template <bool FUSED>
+// SOMM: radiative outer boundary (reading R29) compiled in (a separate
+// instantiation, so the default path carries none of its registers).
+template <bool FUSED, bool SOMM>
 __global__ void __launch_bounds__(RT, 1)
     k_rhs(DevMesh m, const double* __restrict__ patches, double* __restrict__ rhs_oct,
           RhsParams prm, int first, int count) {
@@ -344,6 +346,15 @@ __global__ void __launch_bounds__(RT, 1)
                  : "memory");
   const double ih = (6.0 * double(int64_t(1) << oi.w)) / m.width;   // 1/h
   const double ko_scale = prm.ko_sigma * ih * (1.0 / 64.0);
+  // Sommerfeld (reading R29): this point is a node on a face of the domain
+  bool bpt = false;
+  if (SOMM && tab_c0[tid] >= 0) {
+    const int q = tab_p[tid], nx = q % 7, ny = (q / 7) % 7, nz = q / 49;
+    const int nside = 1 << m.D, sd = 1 << (m.D - oi.w);
+    bpt = (nx == 0 && oi.x == 0) || (ny == 0 && oi.y == 0) || (nz == 0 && oi.z == 0) ||
+          (nx == 6 && oi.x + sd == nside) || (ny == 6 && oi.y + sd == nside) ||
+          (nz == 6 && oi.z + sd == nside);
+  }
 
   // ---- values at the point (patch interior) -------------------------------
   double alpha = 0, chi = 0, Kv = 0, beta[3] = {0, 0, 0};
@@ -481,6 +492,27 @@ __global__ void __launch_bounds__(RT, 1)
       __syncthreads();
     }
     const int c0 = tab_c0[tid];
+    if (SOMM && bpt) {
+      // radiative condition d_t f = -(x^i/r) d_i f - (f - f_inf)/r replaces the
+      // whole right-hand side of field f here (the epilogue skips this point)
+      const int q = tab_p[tid];
+      const int sd = 1 << (m.D - oi.w);
+      const double unit = m.width / (6.0 * double(int64_t(1) << m.D));
+      const int nd[3] = {q % 7, (q / 7) % 7, q / 49}, an[3] = {oi.x, oi.y, oi.z};
+      double xr = 0.0, r2 = 0.0;
+#pragma unroll
+      for (int a = 0; a < 3; ++a) {
+        const int st = a == 0 ? 1 : (a == 1 ? 13 : 169);
+        const double x = m.xmin[a] + double(6 * int64_t(an[a]) + int64_t(nd[a]) * sd) * unit;
+        const double g = ((s[c0 + st] - s[c0 - st]) * 45.0 - (s[c0 + 2 * st] - s[c0 - 2 * st]) * 9.0 +
+                          (s[c0 + 3 * st] - s[c0 - 3 * st])) * (ih * (1.0 / 60.0));
+        xr += x * g;
+        r2 += x * x;
+      }
+      const double finf = (f <= 1 || f == 12 || f == 15 || f == 17) ? 1.0 : 0.0;
+      const double ir = 1.0 / sqrt(r2);
+      rhs_oct[int64_t(f) * no * NPT + int64_t(e) * NPT + q] = -xr * ir - (s[c0] - finf) * ir;
+    }
     if (c0 >= 0) {
       if (f >= 12 && f <= 17) {
         // ---------------- conformal metric gt_q: d gt, gt^lm d_lm gt, adv, KO
@@ -850,8 +882,10 @@ __global__ void __launch_bounds__(RT, 1)
       }
     double* out = rhs_oct + int64_t(e) * NPT + p;
     const int64_t ostr = no * NPT;
+    if (!SOMM || !bpt) {
 #pragma unroll
-    for (int f = 0; f < NF; ++f) out[f * ostr] = r[f];
+      for (int f = 0; f < NF; ++f) out[f * ostr] = r[f];
+    }
   }
   }  // octant loop
 #undef SL
@@ -896,8 +930,10 @@ void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const 
   if (count <= 0) return;
   static int n_sm = 0;
   if (!n_sm) {
-    cudaFuncSetAttribute(k_rhs<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(SMEM_BYTES));
-    cudaFuncSetAttribute(k_rhs<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(SMEM_BYTES));
+    cudaFuncSetAttribute(k_rhs<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(SMEM_BYTES));
+    cudaFuncSetAttribute(k_rhs<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(SMEM_BYTES));
+    cudaFuncSetAttribute(k_rhs<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(SMEM_BYTES));
+    cudaFuncSetAttribute(k_rhs<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(SMEM_BYTES));
     int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&n_sm, cudaDevAttrMultiProcessorCount, dev);
@@ -906,10 +942,15 @@ void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const 
   // persistent: one CTA per SM (225 KB of shared memory each)
   const int64_t cap = leave_sm > 0 && n_sm - leave_sm > 0 ? n_sm - leave_sm : n_sm;
   const int grid = int(count < cap ? count : cap);
-  if (fused)
-    k_rhs<true><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, int(first), int(count));
+  const bool somm = p.sommerfeld && !m.periodic;
+  if (fused && !somm)
+    k_rhs<true, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, int(first), int(count));
+  else if (fused)
+    k_rhs<true, true><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, int(first), int(count));
+  else if (!somm)
+    k_rhs<false, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, int(first), int(count));
   else
-    k_rhs<false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, int(first), int(count));
+    k_rhs<false, true><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, int(first), int(count));
 }
 
 }  // namespace dgr

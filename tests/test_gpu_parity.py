@@ -207,3 +207,45 @@ def test_100_steps_parity(name):
     got = ud[:, :om.n_dof].cpu().numpy()
     assert np.max(np.abs(v - u)) > 1e-3            # the state really evolved
     assert_parity(got, v, 1e-8, f"100 steps {name}")
+
+
+@pytest.mark.parametrize("kind", ["bl", "random"])
+def test_rhs_sommerfeld_parity(kind):
+    """Radiative outer boundary (reading R29): the CUDA RHS
+    with dgr_params.sommerfeld = 1 matches the oracle's on a non-periodic mesh
+    with hanging chains, on both the fused and the two-pass path, and differs
+    from the extrapolating boundary exactly at the DOFs on the domain faces."""
+    need_gpu()
+    cfg = configs.small_bbh(lmax=6, rho=0.5)
+    om = OracleMesh(cfg)
+    om.build_dofs()
+    x = om.dof_coords()
+    u = initial.for_config(cfg, x, kind=kind, seed=5)
+    m = dgr.Mesh(cfg)
+    ud = to_dev(u, m.dof_stride)
+    r = m.rhs(ud, prm=dgr.Params(sommerfeld=1))[:, :om.n_dof]
+    ro = ork4.rhs_dofs(om, u, obssn.Params(sommerfeld=1))
+    assert_parity(r.cpu().numpy(), ro, TOL, f"rhs sommerfeld {kind}")
+    m.set_fused(False)
+    r2 = m.rhs(ud, prm=dgr.Params(sommerfeld=1))[:, :om.n_dof]
+    m.set_fused(True)
+    assert torch.equal(r, r2)
+    r0 = m.rhs(ud)[:, :om.n_dof].cpu().numpy()
+    lo = np.asarray(cfg.xmin)[:, None]
+    face = np.any((x == lo) | (x == lo + cfg.width), axis=0)
+    changed = np.any(r.cpu().numpy() != r0, axis=0)
+    assert np.array_equal(changed, face)
+
+
+def test_rk4_step_sommerfeld_parity():
+    need_gpu()
+    cfg = configs.small_adaptive(lmax=5, rho=0.5)
+    om = OracleMesh(cfg)
+    om.build_dofs()
+    u = initial.for_config(cfg, om.dof_coords(), kind="bl", seed=0)
+    m = dgr.Mesh(cfg)
+    dt = ork4.dt_courant(om)
+    ud = to_dev(u, m.dof_stride)
+    m.rk4_step(ud, dt, prm=dgr.Params(sommerfeld=1))
+    uo = ork4.rk4_step(om, u, dt, obssn.Params(sommerfeld=1))
+    assert_parity(ud[:, :om.n_dof].cpu().numpy(), uo, TOL, "rk4 sommerfeld")

@@ -1,0 +1,55 @@
+"""Long single-puncture evolution on the GPU: C2
+(Schwarzschild m = 1, [-32, 32]^3, levels 3..8) with the extrapolating outer
+boundary (R12) and with the radiative condition (R29), constraint norms
+(dgr_constraints: Hamiltonian H, momentum M^i, Gamma constraint G^i) and the
+lapse minimum sampled along the run.
+
+    python tools/long_run.py [t_end=100] [samples=20]
+"""
+import os
+import sys
+import time
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np
+import torch
+
+import paper_conf_sc_fernandonhzsgb22_b200 as dgr
+from synth import configs, initial
+
+t_end = float(sys.argv[1]) if len(sys.argv) > 1 else 100.0
+samples = int(sys.argv[2]) if len(sys.argv) > 2 else 20
+cfg = configs.c2_schwarzschild()
+m = dgr.Mesh(cfg)
+xyz = m.dof_xyz_host()
+n = xyz.shape[1]
+u0 = initial.for_config(cfg, xyz, kind="bl")
+dt = 0.25 * m.info["h_min"]
+steps = int(round(t_end / dt))
+every = max(1, steps // samples)
+r = np.sqrt((xyz ** 2).sum(axis=0))
+far = torch.from_numpy(r > 24.0).cuda()           # outer region (boundary at 32)
+print(f"C2: {m.info['n_oct_global']} octants, {n} DOFs, dt = {dt:.5f}, {steps} steps to t = {t_end}")
+for somm in (0, 1):
+    prm = dgr.Params(sommerfeld=somm)
+    u = torch.zeros((24, m.dof_stride), dtype=torch.float64, device="cuda")
+    u[:, :n] = torch.from_numpy(u0)
+    print(f"--- outer boundary: {'Sommerfeld (R29)' if somm else 'extrapolation (R12)'}")
+    print(f"{'t':>7s} {'H_L2':>10s} {'H_max':>10s} {'M_L2':>10s} {'G_L2':>10s} "
+          f"{'H_max(r>24)':>12s} {'alpha_min':>10s} {'finite':>6s}")
+    t0 = time.time()
+    for k in range(steps + 1):
+        if k % every == 0 or k == steps:
+            c, nm = m.constraints(u, prm=prm)
+            fin = bool(torch.isfinite(u[:, :n]).all())
+            hfar = float(c[0, :n][far].abs().max())
+            mL2 = float(np.sqrt((nm[1:4, 0] ** 2).sum()))
+            gL2 = float(np.sqrt((nm[4:7, 0] ** 2).sum()))
+            print(f"{k * dt:7.2f} {nm[0, 0]:10.3e} {nm[0, 1]:10.3e} {mL2:10.3e} {gL2:10.3e} "
+                  f"{hfar:12.3e} {float(u[0, :n].min()):10.5f} {str(fin):>6s}", flush=True)
+            if not fin:
+                break
+        if k < steps:
+            m.rk4_step(u, dt, prm=prm)
+    torch.cuda.synchronize()
+    print(f"    wall {time.time() - t0:.1f} s")

@@ -418,6 +418,8 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
           ipt.push_back(uint16_t(t[0] | (t[1] << 4) | (t[2] << 8)));
         }
         if (slot == first) continue;
+        if (hi[grp / 2] - lo[grp / 2] + 1 > 4)   // k_interp's scratch bound (IP_N1)
+          return fail(DGR_ERR_TREE, "interpolation face group thicker than 4 points");
         const int lohi = (lo[0] | (lo[1] << 4) | (lo[2] << 8)) |
                          ((hi[0] | (hi[1] << 4) | (hi[2] << 8)) << 12) | ((grp / 2) << 24);
         igrp.push_back(make_int4(int32_t(first), int32_t(slot - first), lohi, 0));

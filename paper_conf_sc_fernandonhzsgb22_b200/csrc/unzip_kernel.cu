@@ -34,7 +34,11 @@ constexpr int UZ_WARPS = 8;                 // = fields per CTA
 constexpr int UZ_THREADS = 32 * UZ_WARPS;
 constexpr int IP_FG = 4;                    // fields per k_interp CTA
 constexpr int IP_THREADS = 256;
-constexpr int IP_T1 = 49 * 13, IP_T2 = 7 * 13 * 13;
+// sweep scratch per field: a face group's box is at most IP_N1 = 4 points thick
+// along its first sweep axis (host-checked in api.cu), so T1 = 49 x n1 and
+// T2 = 7 x n2 x n1 <= 7 x 13 x 4 (29 KB per 4-field CTA: 6 CTAs per SM)
+constexpr int IP_N1 = 4;
+constexpr int IP_T1 = 49 * IP_N1, IP_T2 = 7 * 13 * IP_N1;
 constexpr int IP_FIELD = NPT + IP_T1 + IP_T2;   // scratch doubles per field
 
 // q = floor(i / n) for 0 <= i < 2^16, 1 <= n <= 13 (float reciprocal, exact here)

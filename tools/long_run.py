@@ -5,6 +5,8 @@ boundary (R12) and with the radiative condition (R29), constraint norms
 lapse minimum sampled along the run.
 
     python tools/long_run.py [t_end=100] [samples=20]
+Environment: DGR_SIGMA (KO strength, 0.4), DGR_ETA (2.0), DGR_CFL (0.25),
+DGR_BC ("both" | "somm" | "extrap").
 """
 import os
 import sys
@@ -24,14 +26,18 @@ m = dgr.Mesh(cfg)
 xyz = m.dof_xyz_host()
 n = xyz.shape[1]
 u0 = initial.for_config(cfg, xyz, kind="bl")
-dt = 0.25 * m.info["h_min"]
+sigma = float(os.environ.get("DGR_SIGMA", "0.4"))
+eta = float(os.environ.get("DGR_ETA", "2.0"))
+dt = float(os.environ.get("DGR_CFL", "0.25")) * m.info["h_min"]
+bcs = {"both": (0, 1), "somm": (1,), "extrap": (0,)}[os.environ.get("DGR_BC", "both")]
 steps = int(round(t_end / dt))
 every = max(1, steps // samples)
 r = np.sqrt((xyz ** 2).sum(axis=0))
 far = torch.from_numpy(r > 24.0).cuda()           # outer region (boundary at 32)
-print(f"C2: {m.info['n_oct_global']} octants, {n} DOFs, dt = {dt:.5f}, {steps} steps to t = {t_end}")
-for somm in (0, 1):
-    prm = dgr.Params(sommerfeld=somm)
+print(f"C2: {m.info['n_oct_global']} octants, {n} DOFs, dt = {dt:.5f}, {steps} steps to t = {t_end}, "
+      f"KO sigma {sigma}, eta {eta}")
+for somm in bcs:
+    prm = dgr.Params(sommerfeld=somm, ko_sigma=sigma, eta=eta)
     u = torch.zeros((24, m.dof_stride), dtype=torch.float64, device="cuda")
     u[:, :n] = torch.from_numpy(u0)
     print(f"--- outer boundary: {'Sommerfeld (R29)' if somm else 'extrapolation (R12)'}")

@@ -6,7 +6,8 @@ lapse minimum sampled along the run.
 
     python tools/long_run.py [t_end=100] [samples=20]
 Environment: DGR_SIGMA (KO strength, 0.4), DGR_ETA (2.0), DGR_CFL (0.25),
-DGR_BC ("both" | "somm" | "extrap").
+DGR_BC ("both" | "somm" | "extrap"), DGR_LMAX (finest level, 8),
+DGR_PUNCT ("c2": offset h/4 in z as in synth.configs; "cell": at a cell centre).
 """
 import os
 import sys
@@ -21,7 +22,13 @@ from synth import configs, initial
 
 t_end = float(sys.argv[1]) if len(sys.argv) > 1 else 100.0
 samples = int(sys.argv[2]) if len(sys.argv) > 2 else 20
-cfg = configs.c2_schwarzschild()
+import dataclasses
+from synth.configs import Puncture
+lmax = int(os.environ.get("DGR_LMAX", "8"))
+cfg = configs.c2_schwarzschild(lmax=lmax)
+if os.environ.get("DGR_PUNCT", "c2") == "cell":
+    hh = cfg.width / (6.0 * (1 << lmax))
+    cfg = dataclasses.replace(cfg, punctures=(Puncture(hh / 2, hh / 2, hh / 2, 1.0, lmax),))
 m = dgr.Mesh(cfg)
 xyz = m.dof_xyz_host()
 n = xyz.shape[1]

@@ -250,6 +250,25 @@ def main():
     value = n_dof / (ms_max * 1e-3)
     finite = bool(torch.isfinite(u[:, :info["n_dof_owned"]]).all())
 
+    # ---- a7: constraint diagnostics (not part of the RK4 step)
+    cons = None
+    if world == 1:
+        mesh.constraints(u)                                   # allocates the patch buffer
+        torch.cuda.synchronize()
+        mesh.profile_read(reset=True)
+        mesh.profile_enable(True)
+        c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        c0.record()
+        for _ in range(3):
+            _, norms = mesh.constraints(u)
+        c1.record()
+        torch.cuda.synchronize()
+        mesh.profile_enable(False)
+        cp = mesh.profile_read(reset=True)
+        cons = {"ms_per_call": c0.elapsed_time(c1) / 3,
+                "kernels_ms_per_call": {k: v[0] / 3 for k, v in cp.items()},
+                "H_L2": float(norms[0, 0]), "H_max": float(norms[0, 1])}
+
     # ---- end to end through the public API with host buffers
     n_loc = info["n_dof_owned"] + info["n_dof_ghost"]
     host_in = torch.empty((24, mesh.dof_stride), dtype=torch.float64, pin_memory=True)
@@ -355,6 +374,7 @@ def main():
         "cpu_baseline": cpu,
         "e2e": {"value": n_dof / (ms_e2e * 1e-3), "unit": UNIT, "h2d_bytes_per_step": bytes_io,
                 "d2h_bytes_per_step": bytes_io, "ms_per_step": ms_e2e},
+        "constraints": cons,
         "gpu_launches": launches_per_step * args.steps,
         "clocks": clk.summary(),
         "finite": finite,

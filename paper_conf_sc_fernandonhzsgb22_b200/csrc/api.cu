@@ -549,7 +549,7 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
     CUDA_TRY(m->alloc(&m->d_sendbuf, size_t(NF) * h.send_list.size()));
     CUDA_TRY(m->alloc(&m->d_recvbuf, size_t(NF) * h.n_ghost_dof));
   }
-  CUDA_TRY(m->alloc(&m->d_cnorm, 64));
+  CUDA_TRY(m->alloc(&m->d_cnorm, 16 + size_t(7) * 2 * CN_BLOCKS));   // [16] result + partials
   CUDA_TRY(cudaStreamSynchronize(st));
   return DGR_OK;
 }
@@ -954,21 +954,13 @@ dgr_status dgr_constraints(dgr_mesh m, double* u, double* c, double* norms_host,
   PROF(m, 4, st, launch_zip(dm, m->d_rhs_oct, c, 7, st));
   CUDA_TRY(cudaGetLastError());
   if (norms_host) {
+    // norms on the device (deterministic two-pass reduction), 14 doubles to the host
     const int64_t n = m->host.n_owned_dof;
-    std::vector<double> hc(size_t(7) * stride);
-    CUDA_TRY(cudaMemcpyAsync(hc.data(), c, hc.size() * 8, cudaMemcpyDeviceToHost, st));
-    CUDA_TRY(cudaStreamSynchronize(st));
+    PROF(m, 6, st, launch_cnorms(c, stride, n, 7, m->d_cnorm + 16, m->d_cnorm, st));
+    CUDA_TRY(cudaGetLastError());
     double part[14];
-    for (int q = 0; q < 7; ++q) {
-      double ss = 0, mx = 0;
-      for (int64_t d = 0; d < n; ++d) {
-        const double v = hc[q * stride + d];
-        ss += v * v;
-        mx = std::max(mx, std::fabs(v));
-      }
-      part[2 * q] = ss;
-      part[2 * q + 1] = mx;
-    }
+    CUDA_TRY(cudaMemcpyAsync(part, m->d_cnorm, sizeof(part), cudaMemcpyDeviceToHost, st));
+    CUDA_TRY(cudaStreamSynchronize(st));
     double ntot = double(n);
     if (m->host.nranks > 1 && m->comm) {   // (external-exchange mode: rank-local norms)
       double* d = m->d_cnorm;

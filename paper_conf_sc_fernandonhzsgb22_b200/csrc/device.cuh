@@ -58,6 +58,11 @@ void launch_interp(const DevMesh& m, const double* u, int nf, int64_t first, int
                    cudaStream_t s);
 // kernels.cu
 void launch_zip(const DevMesh& m, const double* rhs_oct, double* rhs, int nf, cudaStream_t s);
+// sums of squares and max |.| of rows q < nq of c over d < n -> out[2q], out[2q+1]
+// (device; part: [nq][2][CN_BLOCKS] scratch)
+constexpr int CN_BLOCKS = 296;
+void launch_cnorms(const double* c, int64_t stride, int64_t n, int nq, double* part, double* out,
+                   cudaStream_t s);
 void launch_zip_rk4(const DevMesh& m, const double* rhs_oct, int stage, double dt,
                     const double* u_n, double* u_s, double* acc, double* u_out, cudaStream_t s);
 void launch_dof_coords(const DevMesh& m, const int64_t* dof_node, double* xyz,

@@ -69,6 +69,54 @@ __global__ void k_zip_rk4(const int32_t* __restrict__ zip, int32_t n, int64_t no
   }
 }
 
+// ------------------------------------------------- constraint norms (a7)
+// Sum of squares and max |.| of each of nq rows of c over d < n, in a fixed
+// order (deterministic): per-block partials, then one block per row.
+constexpr int CN_THREADS = 256;
+__global__ void k_cnorm_partial(const double* __restrict__ c, int64_t stride, int64_t n,
+                                double* __restrict__ part /*[nq][2][gridDim.x]*/) {
+  const int q = blockIdx.y;
+  double ss = 0.0, mx = 0.0;
+  for (int64_t d = blockIdx.x * int64_t(CN_THREADS) + threadIdx.x; d < n;
+       d += int64_t(gridDim.x) * CN_THREADS) {
+    const double v = c[q * stride + d];
+    ss = fma(v, v, ss);
+    mx = fmax(mx, fabs(v));
+  }
+  __shared__ double s_ss[CN_THREADS], s_mx[CN_THREADS];
+  s_ss[threadIdx.x] = ss;
+  s_mx[threadIdx.x] = mx;
+  __syncthreads();
+  for (int w = CN_THREADS / 2; w > 0; w >>= 1) {
+    if (int(threadIdx.x) < w) {
+      s_ss[threadIdx.x] += s_ss[threadIdx.x + w];
+      s_mx[threadIdx.x] = fmax(s_mx[threadIdx.x], s_mx[threadIdx.x + w]);
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    part[(2 * q) * gridDim.x + blockIdx.x] = s_ss[0];
+    part[(2 * q + 1) * gridDim.x + blockIdx.x] = s_mx[0];
+  }
+}
+__global__ void k_cnorm_final(const double* __restrict__ part, int nblk, double* __restrict__ out) {
+  const int q = blockIdx.x;
+  if (threadIdx.x == 0) {
+    double ss = 0.0, mx = 0.0;
+    for (int b = 0; b < nblk; ++b) {
+      ss += part[(2 * q) * nblk + b];
+      mx = fmax(mx, part[(2 * q + 1) * nblk + b]);
+    }
+    out[2 * q] = ss;
+    out[2 * q + 1] = mx;
+  }
+}
+void launch_cnorms(const double* c, int64_t stride, int64_t n, int nq, double* part, double* out,
+                   cudaStream_t s) {
+  k_cnorm_partial<<<dim3(CN_BLOCKS, nq), CN_THREADS, 0, s>>>(c, stride, n, part);
+  k_cnorm_final<<<nq, 32, 0, s>>>(part, CN_BLOCKS, out);
+}
+
 void launch_zip_rk4(const DevMesh& m, const double* rhs_oct, int stage, double dt,
                     const double* u_n, double* u_s, double* acc, double* u_out, cudaStream_t s) {
   if (m.n_owned_dof <= 0) return;

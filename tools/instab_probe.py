@@ -1,0 +1,28 @@
+"""Where does the C2 instability start?  Position (radius) and value of
+max |H| and of max |rhs| per field group along the run (diagnostic)."""
+import os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np, torch
+import paper_conf_sc_fernandonhzsgb22_b200 as dgr
+from synth import configs, initial
+cfg = configs.c2_schwarzschild()
+m = dgr.Mesh(cfg)
+xyz = m.dof_xyz_host(); n = xyz.shape[1]
+r = np.sqrt((xyz ** 2).sum(axis=0))
+u = torch.zeros((24, m.dof_stride), dtype=torch.float64, device="cuda")
+u[:, :n] = torch.from_numpy(initial.for_config(cfg, xyz, kind="bl"))
+dt = 0.25 * m.info["h_min"]
+names = ["alpha", "chi", "K", "Gt", "beta", "B", "gt", "At"]
+groups = [[0], [1], [2], [3, 4, 5], [6, 7, 8], [9, 10, 11], list(range(12, 18)), list(range(18, 24))]
+for k in range(0, 1200):
+    if k % 96 == 0:
+        c, nm = m.constraints(u)
+        H = c[0, :n].abs().cpu().numpy()
+        i = int(np.argmax(H))
+        rh = m.rhs(u)[:, :n].abs().cpu().numpy()
+        s = " ".join(f"{nm_}:{rh[g].max():.1e}@r={r[np.unravel_index(np.argmax(rh[g]), rh[g].shape)[1]]:.2f}"
+                     for nm_, g in zip(names, groups))
+        print(f"t={k*dt:6.2f} |H|max={H[i]:.2e} at r={r[i]:.3f}  {s}", flush=True)
+        if not np.isfinite(H).all():
+            break
+    m.rk4_step(u, dt)

@@ -232,7 +232,12 @@ dgr_status dgr_constraints(dgr_mesh m, double* u, double* c, double* norms_host,
  *     communicator, else one pass; 1 = always run the interior octants (and the
  *     slots they need) first, then the rest; 2 = interior octants only (test
  *     hook: boundary octants' RHS is not computed). */
-enum { DGR_OPT_FUSED_UNZIP = 1, DGR_OPT_PHASES = 2 };
+/*   DGR_OPT_PREPASS (default 1): fused path without the radiative boundary
+ *     evaluates the six gt_ij fields' derivatives in a separate metric pre-pass
+ *     kernel (two CTAs per SM, 30 values per point through HBM) and the other
+ *     18 fields in the RHS kernel; 0 = all 24 fields in the RHS kernel.  Both
+ *     give bit-identical results. */
+enum { DGR_OPT_FUSED_UNZIP = 1, DGR_OPT_PHASES = 2, DGR_OPT_PREPASS = 3 };
 dgr_status dgr_set_option(dgr_mesh m, int option, int64_t value);
 
 /* Device-side timing helper for benchmarks: number of kernel launches the last

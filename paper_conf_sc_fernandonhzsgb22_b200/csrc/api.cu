@@ -111,6 +111,8 @@ struct dgr_mesh_s {
   cudaStream_t xstream = nullptr;   // ghost exchange stream (N > 1)
   int xsm = 8;                      // SMs k_rhs leaves to NCCL while overlapping
   int phases = 0;                   // DGR_OPT_PHASES
+  bool prepass = true;              // DGR_OPT_PREPASS: gt_ij stages in k_gt_pre
+  double* d_pre = nullptr;          // [30][n_owned][343] metric pre-pass results
   cudaEvent_t ev_ready = nullptr, ev_xdone = nullptr;
   int4* d_iel = nullptr;        // interpolation work per element with slots
   int4* d_igrp = nullptr;       // ... per face group of its slots
@@ -806,6 +808,11 @@ static dgr_status rhs_oct(dgr_mesh m, double* u, const dgr_params* prm, cudaStre
   dgr_status s;
   const int64_t no = m->dm.n_owned, ni = m->n_interior;
   const RhsParams rp = to_rp(prm);
+  double* pre = nullptr;
+  if (m->fused && m->prepass && !(rp.sommerfeld && !m->host.periodic)) {
+    if (!m->d_pre) CUDA_TRY(m->alloc(&m->d_pre, size_t(30) * no * NPT));
+    pre = m->d_pre;
+  }
   if (!m->fused) {
     if ((s = exchange(m, u, st))) return s;
     if ((s = do_unzip(m, u, NF, st))) return s;
@@ -819,10 +826,10 @@ static dgr_status rhs_oct(dgr_mesh m, double* u, const dgr_params* prm, cudaStre
     // hook stops here) the rest — no stream overlap
     if ((s = exchange(m, u, st))) return s;
     if ((s = do_interp(m, u, NF, st, 0))) return s;
-    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, ni, 0, st));
+    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, ni, 0, st, pre));
     if (m->phases == 1) {
       if ((s = do_interp(m, u, NF, st, 1))) return s;
-      PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, ni, no - ni, 0, st));
+      PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, ni, no - ni, 0, st, pre));
     }
   } else if (overlap) {
     if (!m->xstream) {
@@ -835,14 +842,14 @@ static dgr_status rhs_oct(dgr_mesh m, double* u, const dgr_params* prm, cudaStre
     if ((s = exchange(m, u, m->xstream))) return s;
     CUDA_TRY(cudaEventRecord(m->ev_xdone, m->xstream));
     if ((s = do_interp(m, u, NF, st, 0))) return s;
-    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, ni, m->xsm, st));
+    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, ni, m->xsm, st, pre));
     CUDA_TRY(cudaStreamWaitEvent(st, m->ev_xdone, 0));
     if ((s = do_interp(m, u, NF, st, 1))) return s;
-    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, ni, no - ni, 0, st));
+    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, ni, no - ni, 0, st, pre));
   } else {
     if ((s = exchange(m, u, st))) return s;
     if ((s = do_interp(m, u, NF, st))) return s;
-    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, no, 0, st));
+    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, no, 0, st, pre));
   }
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;
@@ -995,6 +1002,7 @@ dgr_status dgr_set_option(dgr_mesh m, int option, int64_t value) {
   if (!m) return fail(DGR_ERR_ARG, "null mesh");
   switch (option) {
     case DGR_OPT_FUSED_UNZIP: m->fused = value != 0; return DGR_OK;
+    case DGR_OPT_PREPASS: m->prepass = value != 0; return DGR_OK;
     case DGR_OPT_PHASES:
       if (value < 0 || value > 2) return fail(DGR_ERR_ARG, "DGR_OPT_PHASES is 0, 1 or 2");
       m->phases = int(value);

@@ -84,8 +84,11 @@ struct RhsParams {
 // slots through gmap (no patch buffer)
 // RHS of the owned octants m.olist[first, first + count); at most
 // n_SM - leave_sm persistent CTAs
+// pre != nullptr (fused, no Sommerfeld): the gt_ij stages run in the metric
+// pre-pass k_gt_pre (pre: [30][n_owned][343] scratch), then k_rhs on the rest
 void launch_rhs(const DevMesh& m, const double* src, double* rhs_oct, const RhsParams& p,
-                bool fused, int64_t first, int64_t count, int leave_sm, cudaStream_t s);
+                bool fused, int64_t first, int64_t count, int leave_sm, cudaStream_t s,
+                double* pre = nullptr);
 size_t rhs_smem_bytes();
 void upload_rhs_tables(const double* wext);
 

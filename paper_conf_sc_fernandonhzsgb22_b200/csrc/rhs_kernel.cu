@@ -66,6 +66,8 @@ static_assert(N_TXL + N_TYL <= RT, "one pencil per thread");
 // field processing order
 __constant__ int c_order[NF] = {12, 13, 14, 15, 16, 17, 1, 0, 3, 4, 5, 6,
                                 7,  8,  2,  18, 19, 20, 21, 22, 23, 9, 10, 11};
+// field order after the metric pre-pass (k_gt_pre): the same without gt_ij
+__constant__ int c_order_pre[NF - 6] = {1, 0, 3, 4, 5, 6, 7, 8, 2, 18, 19, 20, 21, 22, 23, 9, 10, 11};
 
 __device__ __forceinline__ int sidx(int i, int j) {
   // (0,0)0 (0,1)1 (0,2)2 (1,1)3 (1,2)4 (2,2)5
@@ -105,6 +107,10 @@ __device__ __forceinline__ void cp_async8(uint32_t dst, const double* uf, const 
       " cp.async.ca.shared.global [%0], [a], 8;\n}\n" ::"r"(dst),
       "l"(uf), "l"(af), "r"(idx), "r"(ds)
       : "memory");
+}
+// 8-byte asynchronous global->shared copy of *src
+__device__ __forceinline__ void cp_async8u(uint32_t dst, const double* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(dst), "l"(src) : "memory");
 }
 __device__ __forceinline__ void cp_async_commit() {
   asm volatile("cp.async.commit_group;" ::: "memory");
@@ -234,10 +240,14 @@ __device__ __forceinline__ double trace6(const double* gi, const double* X) {
 // the same arithmetic as k_unzip.
 // SOMM: radiative outer boundary (reading R29) compiled in (a separate
 // instantiation, so the default path carries none of its registers).
-template <bool FUSED, bool SOMM>
+template <bool FUSED, bool SOMM, bool PRE>
 __global__ void __launch_bounds__(RT, 1)
     k_rhs(DevMesh m, const double* __restrict__ patches, double* __restrict__ rhs_oct,
-          RhsParams prm, int first, int count) {
+          RhsParams prm, int first, int count, const double* __restrict__ pre) {
+  // PRE: the gt_ij stages were done by k_gt_pre (its 30 values per point are
+  // read in the prologue); the stream holds the 18 other fields
+  constexpr int NS = PRE ? NF - 6 : NF;
+  const int* ORD = PRE ? c_order_pre : c_order;
   extern __shared__ __align__(128) double smem[];
   double* slots = smem;                           // [NSLOT][NPP]
   double* stage = smem + NSLOT * NPP;             // [2][STAGE_DBL]
@@ -307,14 +317,14 @@ __global__ void __launch_bounds__(RT, 1)
   __syncthreads();
   if (FUSED) {
     load_gidx(e);
-    gather(stage, c_order[0]);
-    gather(stage + STAGE_DBL, c_order[1]);
+    gather(stage, ORD[0]);
+    gather(stage + STAGE_DBL, ORD[1]);
   } else if (tid == 0) {
     const double* pb = patches + int64_t(e) * PATCH_PITCH;
-    bulk_load(stage, pb + c_order[0] * fstride, STAGE_DBL * 8, &bars[0]);
-    bulk_load(stage + STAGE_DBL, pb + c_order[1] * fstride, STAGE_DBL * 8, &bars[1]);
-  } else if (tid < NF - 1) {
-    prefetch_l2(patches + int64_t(e) * PATCH_PITCH + c_order[tid + 1] * fstride);
+    bulk_load(stage, pb + ORD[0] * fstride, STAGE_DBL * 8, &bars[0]);
+    bulk_load(stage + STAGE_DBL, pb + ORD[1] * fstride, STAGE_DBL * 8, &bars[1]);
+  } else if (tid < NS - 1) {
+    prefetch_l2(patches + int64_t(e) * PATCH_PITCH + ORD[tid + 1] * fstride);
   }
   uint32_t g = 0;   // global stage counter of this CTA
   for (; li < count; li += gridDim.x) {
@@ -357,6 +367,20 @@ __global__ void __launch_bounds__(RT, 1)
   }
 
   // ---- values at the point (patch interior) -------------------------------
+  if (PRE && active) {
+    // metric pre-pass results -> d gt (S0), gt^lm d_lm gt (A_AT), adv + KO of gt
+    // (A_GAM) slots, asynchronously, in flight while the values are read
+    const double* pr = pre + int64_t(e) * NPT + tab_p[tid];
+    const int64_t pstr = no * NPT;
+#pragma unroll
+    for (int i = 0; i < 18; ++i) cp_async8u(smem_u32(&SL(S0 + i)), pr + i * pstr);
+#pragma unroll
+    for (int q = 0; q < 6; ++q) {
+      cp_async8u(smem_u32(&SL(A_AT + q)), pr + (18 + q) * pstr);
+      cp_async8u(smem_u32(&SL(A_GAM + q)), pr + (24 + q) * pstr);
+    }
+    cp_async_commit();
+  }
   double alpha = 0, chi = 0, Kv = 0, beta[3] = {0, 0, 0};
   if (active) {
     alpha = own(0);
@@ -385,18 +409,114 @@ __global__ void __launch_bounds__(RT, 1)
     SL(G_INV + 5) = (g[0] * g[3] - g[1] * g[1]) * idet;
 #pragma unroll
     for (int q = 0; q < 6; ++q) SL(A_GT + q) = 0.0;     // A_GT, A_BETA
+    if (!PRE) {
 #pragma unroll
-    for (int q = 0; q < 6; ++q) SL(A_GAM + q) = 0.0;
+      for (int q = 0; q < 6; ++q) SL(A_GAM + q) = 0.0;
+    }
   }
   const double chi_e = fmax(chi, prm.chi_floor);
   const double ichi = 1.0 / chi_e;
   double rA = 0.0, rC = 0.0, rK = 0.0;   // accumulators of alpha, chi, K
   double dchi[3] = {0, 0, 0};
 
+  // Christoffel block (eqs 12, 17; readings R1, R7): from d_k gt_ij (S0 slots)
+  // and gt^lm d_lm gt_ij (A_AT slots) — at the last gt stage, or (PRE) right
+  // after the prologue from the metric pre-pass
+  auto christoffel = [&](const double* gi) {
+      // ---------------- Christoffel block (eqs 12, 17; readings R1, R7)
+      double gt[6], At[6];
+#pragma unroll
+      for (int r = 0; r < 6; ++r) {
+        gt[r] = SL(V_GAM + r);
+        At[r] = SL(V_AT + r);
+      }
+      double C[3][6];  // first kind C_k,ij = 1/2 (d_i g_kj + d_j g_ki - d_k g_ij)
+#pragma unroll
+      for (int k = 0; k < 3; ++k)
+#pragma unroll
+        for (int i = 0; i < 3; ++i)
+#pragma unroll
+          for (int j = i; j < 3; ++j)
+            C[k][sidx(i, j)] = 0.5 * (SL(S0 + i * 6 + sidx(k, j)) + SL(S0 + j * 6 + sidx(k, i)) -
+                                      SL(S0 + k * 6 + sidx(i, j)));
+      double Gam[3][6];  // second kind Gt^k_ij = gt^kl C_l,ij
+#pragma unroll
+      for (int k = 0; k < 3; ++k)
+#pragma unroll
+        for (int q2 = 0; q2 < 6; ++q2)
+          Gam[k][q2] = gi[sidx(k, 0)] * C[0][q2] + gi[sidx(k, 1)] * C[1][q2] +
+                       gi[sidx(k, 2)] * C[2][q2];
+      double cal[3];
+#pragma unroll
+      for (int k = 0; k < 3; ++k) cal[k] = trace6(gi, Gam[k]);
+      // Rt_ij without the d Gt terms
+      double Rt[6];
+#pragma unroll
+      for (int i = 0; i < 3; ++i)
+#pragma unroll
+        for (int j = i; j < 3; ++j) {
+          double r = -0.5 * SL(A_AT + sidx(i, j));      // gt^lm d_lm gt_ij
+          double c2 = 0.0;
+#pragma unroll
+          for (int k = 0; k < 3; ++k) c2 += cal[k] * (C[i][sidx(j, k)] + C[j][sidx(i, k)]);
+          r += 0.5 * c2;
+          double qsum = 0.0;
+#pragma unroll
+          for (int l = 0; l < 3; ++l)
+#pragma unroll
+            for (int mm = 0; mm < 3; ++mm) {
+              const double glm = gi[sidx(l, mm)];
+              double t = 0.0;
+#pragma unroll
+              for (int k = 0; k < 3; ++k)
+                t += Gam[k][sidx(l, i)] * C[j][sidx(k, mm)] +
+                     Gam[k][sidx(l, j)] * C[i][sidx(k, mm)] +
+                     Gam[k][sidx(i, mm)] * C[k][sidx(l, j)];
+              qsum += glm * t;
+            }
+          Rt[sidx(i, j)] = r + qsum;
+        }
+      // At_ij = chi alpha TF(Rt)   (first write of the A_AT accumulators)
+      const double trR = trace6(gi, Rt);
+      const double ca = chi * alpha;
+#pragma unroll
+      for (int r = 0; r < 6; ++r) SL(A_AT + r) = ca * (Rt[r] - gt[r] * trR * (1.0 / 3.0));
+      // At^ij = gt^ik gt^jl At_kl ; Gt^i += 2 alpha Gt^i_jk At^jk
+      double Au[6];
+#pragma unroll
+      for (int i = 0; i < 3; ++i)
+#pragma unroll
+        for (int j = i; j < 3; ++j) {
+          double a = 0.0;
+#pragma unroll
+          for (int k = 0; k < 3; ++k)
+#pragma unroll
+            for (int l = 0; l < 3; ++l) a += gi[sidx(i, k)] * gi[sidx(j, l)] * At[sidx(k, l)];
+          Au[sidx(i, j)] = a;
+        }
+#pragma unroll
+      for (int i = 0; i < 3; ++i) SL(A_GT + i) += 2.0 * alpha * trace6(Au, Gam[i]);
+      // keep Gt^k_ij and CalGt^k for the chi, alpha and beta stages
+#pragma unroll
+      for (int k = 0; k < 3; ++k)
+#pragma unroll
+        for (int q2 = 0; q2 < 6; ++q2) SL(S0 + k * 6 + q2) = Gam[k][q2];
+#pragma unroll
+      for (int k = 0; k < 3; ++k) SL(A_B + k) = cal[k];   // (A_B slot reused until B)
+      };
 #ifdef DGR_RHS_TIMING
   long long t_last = clock64();
 #endif
-  for (int st = 0; st < NF; ++st, ++g) {
+  if (PRE && active) {
+    // the metric pre-pass results for this point (copies issued before the
+    // point's values were read), then the Christoffel block
+    asm volatile("cp.async.wait_all;" ::: "memory");
+    double gi[6];
+#pragma unroll
+    for (int r = 0; r < 6; ++r) gi[r] = SL(G_INV + r);
+    christoffel(gi);
+  }
+  for (int st = 0; st < NS; ++st, ++g) {
     const int buf = g & 1;
 #ifdef DGR_RHS_TIMING
     if (tid == 0) {   // per-stage cycle profile (experiment builds only)
@@ -448,7 +568,7 @@ __global__ void __launch_bounds__(RT, 1)
       mbar_wait(&bars[buf], (g >> 1) & 1);
     }
     const double* s = stage + buf * STAGE_DBL;
-    const int f = c_order[st];
+    const int f = ORD[st];
     const bool second = f <= 1 || (f >= 6 && f <= 8) || (f >= 12 && f <= 17);
     if (second) {
       // cooperative first derivatives along x (and y) of the staged field on
@@ -514,7 +634,7 @@ __global__ void __launch_bounds__(RT, 1)
       rhs_oct[int64_t(f) * no * NPT + int64_t(e) * NPT + q] = -xr * ir - (s[c0] - finf) * ir;
     }
     if (c0 >= 0) {
-      if (f >= 12 && f <= 17) {
+      if (!PRE && f >= 12 && f <= 17) {
         // ---------------- conformal metric gt_q: d gt, gt^lm d_lm gt, adv, KO
         const int q = f - 12;
         const Derivs d = derivs2(s, Tx, Ty, c0, ih, ko_scale);
@@ -525,88 +645,7 @@ __global__ void __launch_bounds__(RT, 1)
         for (int k = 0; k < 3; ++k) SL(S0 + k * 6 + q) = d.d1[k];
         SL(A_AT + q) = trace6(gi, d.dd);   // (A_AT slot reused until the Christoffel block)
         SL(A_GAM + q) += beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
-        if (q == 5) {
-          // ---------------- Christoffel block (eqs 12, 17; readings R1, R7)
-          double gt[6], At[6];
-#pragma unroll
-          for (int r = 0; r < 6; ++r) {
-            gt[r] = SL(V_GAM + r);
-            At[r] = SL(V_AT + r);
-          }
-          double C[3][6];  // first kind C_k,ij = 1/2 (d_i g_kj + d_j g_ki - d_k g_ij)
-#pragma unroll
-          for (int k = 0; k < 3; ++k)
-#pragma unroll
-            for (int i = 0; i < 3; ++i)
-#pragma unroll
-              for (int j = i; j < 3; ++j)
-                C[k][sidx(i, j)] = 0.5 * (SL(S0 + i * 6 + sidx(k, j)) + SL(S0 + j * 6 + sidx(k, i)) -
-                                          SL(S0 + k * 6 + sidx(i, j)));
-          double Gam[3][6];  // second kind Gt^k_ij = gt^kl C_l,ij
-#pragma unroll
-          for (int k = 0; k < 3; ++k)
-#pragma unroll
-            for (int q2 = 0; q2 < 6; ++q2)
-              Gam[k][q2] = gi[sidx(k, 0)] * C[0][q2] + gi[sidx(k, 1)] * C[1][q2] +
-                           gi[sidx(k, 2)] * C[2][q2];
-          double cal[3];
-#pragma unroll
-          for (int k = 0; k < 3; ++k) cal[k] = trace6(gi, Gam[k]);
-          // Rt_ij without the d Gt terms
-          double Rt[6];
-#pragma unroll
-          for (int i = 0; i < 3; ++i)
-#pragma unroll
-            for (int j = i; j < 3; ++j) {
-              double r = -0.5 * SL(A_AT + sidx(i, j));      // gt^lm d_lm gt_ij
-              double c2 = 0.0;
-#pragma unroll
-              for (int k = 0; k < 3; ++k) c2 += cal[k] * (C[i][sidx(j, k)] + C[j][sidx(i, k)]);
-              r += 0.5 * c2;
-              double qsum = 0.0;
-#pragma unroll
-              for (int l = 0; l < 3; ++l)
-#pragma unroll
-                for (int mm = 0; mm < 3; ++mm) {
-                  const double glm = gi[sidx(l, mm)];
-                  double t = 0.0;
-#pragma unroll
-                  for (int k = 0; k < 3; ++k)
-                    t += Gam[k][sidx(l, i)] * C[j][sidx(k, mm)] +
-                         Gam[k][sidx(l, j)] * C[i][sidx(k, mm)] +
-                         Gam[k][sidx(i, mm)] * C[k][sidx(l, j)];
-                  qsum += glm * t;
-                }
-              Rt[sidx(i, j)] = r + qsum;
-            }
-          // At_ij = chi alpha TF(Rt)   (first write of the A_AT accumulators)
-          const double trR = trace6(gi, Rt);
-          const double ca = chi * alpha;
-#pragma unroll
-          for (int r = 0; r < 6; ++r) SL(A_AT + r) = ca * (Rt[r] - gt[r] * trR * (1.0 / 3.0));
-          // At^ij = gt^ik gt^jl At_kl ; Gt^i += 2 alpha Gt^i_jk At^jk
-          double Au[6];
-#pragma unroll
-          for (int i = 0; i < 3; ++i)
-#pragma unroll
-            for (int j = i; j < 3; ++j) {
-              double a = 0.0;
-#pragma unroll
-              for (int k = 0; k < 3; ++k)
-#pragma unroll
-                for (int l = 0; l < 3; ++l) a += gi[sidx(i, k)] * gi[sidx(j, l)] * At[sidx(k, l)];
-              Au[sidx(i, j)] = a;
-            }
-#pragma unroll
-          for (int i = 0; i < 3; ++i) SL(A_GT + i) += 2.0 * alpha * trace6(Au, Gam[i]);
-          // keep Gt^k_ij and CalGt^k for the chi, alpha and beta stages
-#pragma unroll
-          for (int k = 0; k < 3; ++k)
-#pragma unroll
-            for (int q2 = 0; q2 < 6; ++q2) SL(S0 + k * 6 + q2) = Gam[k][q2];
-#pragma unroll
-          for (int k = 0; k < 3; ++k) SL(A_B + k) = cal[k];   // (A_B slot reused until B)
-        }
+        if (q == 5) christoffel(gi);
       } else if (f == 1) {
         // ---------------- chi: advection, KO, R^chi (eq 18-19), eq (8) chi term
         const Derivs d = derivs2(s, Tx, Ty, c0, ih, ko_scale);
@@ -797,11 +836,11 @@ __global__ void __launch_bounds__(RT, 1)
     __syncthreads();  // everyone is done with this stage buffer
     if (FUSED) {
       double* dst = stage + buf * STAGE_DBL;
-      if (st + 2 < NF) {
-        gather(dst, c_order[st + 2]);
+      if (st + 2 < NS) {
+        gather(dst, ORD[st + 2]);
       } else {
-        if (st + 2 == NF && en >= 0) load_gidx(en);   // the current octant's gathers are issued
-        if (en >= 0) gather(dst, c_order[st + 2 - NF]);
+        if (st + 2 == NS && en >= 0) load_gidx(en);   // the current octant's gathers are issued
+        if (en >= 0) gather(dst, ORD[st + 2 - NS]);
         else cp_async_commit();                        // (empty group keeps the count uniform)
       }
       continue;
@@ -810,14 +849,14 @@ __global__ void __launch_bounds__(RT, 1)
     // (measured faster than prefetching the current octant at its start,
     // although some prefetched lines are evicted and re-read)
     if (tid == 32 && en >= 0)
-      prefetch_l2(patches + int64_t(en) * PATCH_PITCH + c_order[st] * fstride);
+      prefetch_l2(patches + int64_t(en) * PATCH_PITCH + ORD[st] * fstride);
     if (tid == 0) {
-      if (st + 2 < NF)
-        bulk_load(stage + buf * STAGE_DBL, pbase + c_order[st + 2] * fstride, STAGE_DBL * 8,
+      if (st + 2 < NS)
+        bulk_load(stage + buf * STAGE_DBL, pbase + ORD[st + 2] * fstride, STAGE_DBL * 8,
                   &bars[buf]);
       else if (en >= 0)   // the stream continues with the next octant's first fields
         bulk_load(stage + buf * STAGE_DBL,
-                  patches + int64_t(en) * PATCH_PITCH + c_order[st + 2 - NF] * fstride,
+                  patches + int64_t(en) * PATCH_PITCH + ORD[st + 2 - NS] * fstride,
                   STAGE_DBL * 8, &bars[buf]);
     }
   }
@@ -891,6 +930,225 @@ __global__ void __launch_bounds__(RT, 1)
 #undef SL
 }
 
+// ---------------------------------------------------------------------------
+// Metric pre-pass (DESIGN.md §8c item 1): the six conformal-metric fields
+// gt_q (second derivatives) without any cross-field state, so two CTAs fit on
+// an SM twice (22 warps instead of 11; three CTAs per SM, at 56 registers,
+// measured slower: 1.99 vs 1.53 ms on C3).  Per interior point it writes 30 values to
+// pre[c][n_owned][343]:
+//   c = 6k + q   d_k gt_q                       (k = 0..2, q = 0..5)
+//   c = 18 + q   gt^lm d_l d_m gt_q             (the -1/2 term of Rt, eq 17)
+//   c = 24 + q   beta^k d_k gt_q + KO(gt_q)     (eq 4 advection + dissipation)
+// which k_rhs<..., PRE = true> reads instead of staging the gt fields itself.
+// Same stencils, same gather/extrapolation and same arithmetic order as the
+// gt stages of k_rhs, so both paths give bit-identical results.
+constexpr int NPRE = 30;
+constexpr size_t PRE_SMEM_BYTES = size_t(2) * STAGE_DBL * 8 + size_t(TX_N + TY_N) * 8 + 16 +
+                                  size_t(2) * RT * 2;
+
+template <bool FUSED>
+__global__ void __launch_bounds__(RT, 2)
+    k_gt_pre(DevMesh m, const double* __restrict__ patches, double* __restrict__ pre,
+             RhsParams prm, int first, int count) {
+  extern __shared__ __align__(128) double smem[];
+  double* stage = smem;                           // [2][STAGE_DBL]
+  double* Tx = stage + 2 * STAGE_DBL;             // [TX_N]
+  double* Ty = Tx + TX_N;                         // [TY_N]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(Ty + TY_N);
+  int16_t* tab_c0 = reinterpret_cast<int16_t*>(bars + 2);
+  int16_t* tab_p = tab_c0 + RT;
+  const int tid = threadIdx.x;
+  {
+    const int pp = g_perm[tid];
+    const int q = pp >= 0 ? pp : 0;
+    tab_c0[tid] = pp >= 0 ? int16_t((q % 7 + 3) + 13 * ((q / 7) % 7 + 3) + 169 * (q / 49 + 3)) : -1;
+    tab_p[tid] = int16_t(q);
+  }
+  const int64_t no = m.n_owned;
+  const int64_t fstride = FUSED ? m.dof_stride : no * PATCH_PITCH;
+  const int32_t ds = int32_t(m.dof_stride);
+  const int32_t* ol = m.olist + first;
+  int li = blockIdx.x;
+  if (li >= count) return;
+  int e = ol[li];
+  int gidx[GJ];
+  auto load_gidx = [&](int oct) {
+    const int32_t* gm = m.gmap + int64_t(oct) * GM_PITCH;
+#pragma unroll
+    for (int j = 0; j < GJ; ++j) {
+      const int pt = tid + RT * j;
+      gidx[j] = pt < NPATCH ? max(__ldg(gm + pt), 0) : -1;
+    }
+  };
+  auto gather = [&](double* dst, int f) {
+    const uint32_t d0 = smem_u32(dst + tid);
+    const double* uf = patches + f * fstride;
+    const double* af = m.aux + f * m.aux_stride - m.dof_stride;
+#pragma unroll
+    for (int j = 0; j < GJ - 1; ++j) cp_async8(d0 + 8 * RT * j, uf, af, gidx[j], ds);
+    if (tid + RT * (GJ - 1) < NPATCH) cp_async8(d0 + 8 * RT * (GJ - 1), uf, af, gidx[GJ - 1], ds);
+    cp_async_commit();
+  };
+  if (tid == 0) {
+    mbar_init(&bars[0], 1);
+    mbar_init(&bars[1], 1);
+  }
+  __syncthreads();
+  if (FUSED) {
+    load_gidx(e);
+    gather(stage, 12);
+    gather(stage + STAGE_DBL, 13);
+  } else if (tid == 0) {
+    const double* pb = patches + int64_t(e) * PATCH_PITCH;
+    bulk_load(stage, pb + 12 * fstride, STAGE_DBL * 8, &bars[0]);
+    bulk_load(stage + STAGE_DBL, pb + 13 * fstride, STAGE_DBL * 8, &bars[1]);
+  }
+  uint32_t g = 0;
+  for (; li < count; li += gridDim.x) {
+    e = ol[li];
+    const int en = li + int(gridDim.x) < count ? ol[li + gridDim.x] : -1;
+    const int c0 = tab_c0[tid];
+    const int p = tab_p[tid];
+    const int4 oi = m.oct[e];
+    int omask = 0;
+    if (FUSED && !m.periodic) {
+      const int nside = 1 << m.D, sd = 1 << (m.D - oi.w);
+      omask = (oi.x == 0) | ((oi.y == 0) << 1) | ((oi.z == 0) << 2) | ((oi.x + sd == nside) << 3) |
+              ((oi.y + sd == nside) << 4) | ((oi.z + sd == nside) << 5);
+    }
+    const double ih = (6.0 * double(int64_t(1) << oi.w)) / m.width;   // 1/h
+    const double ko_scale = prm.ko_sigma * ih * (1.0 / 64.0);
+    // values at the point: gt (for gt^ij) and beta (advection)
+    double gi[6] = {0, 0, 0, 0, 0, 0}, beta[3] = {0, 0, 0};
+    if (c0 >= 0) {
+      const int cv = FUSED ? __ldg(m.o2s + int64_t(e) * NPT + p) : c0;
+      auto own = [&](int f) -> double {
+        if (!FUSED) return __ldg(patches + int64_t(e) * PATCH_PITCH + f * fstride + cv);
+        return cv < ds ? __ldg(patches + f * fstride + cv) : __ldg(m.aux + f * m.aux_stride + (cv - ds));
+      };
+      double gq[6];
+#pragma unroll
+      for (int q = 0; q < 6; ++q) gq[q] = own(12 + q);
+#pragma unroll
+      for (int i = 0; i < 3; ++i) beta[i] = own(6 + i);
+      const double a00 = gq[3] * gq[5] - gq[4] * gq[4];
+      const double a01 = gq[2] * gq[4] - gq[1] * gq[5];
+      const double a02 = gq[1] * gq[4] - gq[2] * gq[3];
+      const double det = gq[0] * a00 + gq[1] * a01 + gq[2] * a02;
+      const double idet = 1.0 / det;
+      gi[0] = a00 * idet;
+      gi[1] = a01 * idet;
+      gi[2] = a02 * idet;
+      gi[3] = (gq[0] * gq[5] - gq[2] * gq[2]) * idet;
+      gi[4] = (gq[1] * gq[2] - gq[0] * gq[4]) * idet;
+      gi[5] = (gq[0] * gq[3] - gq[1] * gq[1]) * idet;
+    }
+    double* out = pre + int64_t(e) * NPT + p;
+    const int64_t ostr = no * NPT;
+    for (int q = 0; q < 6; ++q, ++g) {
+      const int buf = g & 1;
+      if (FUSED) {
+        cp_async_wait1();
+        __syncthreads();
+        if (omask) {
+          double* sw = stage + buf * STAGE_DBL;
+          for (int a = 0; a < 3; ++a) {
+            const int sa = a == 0 ? 1 : (a == 1 ? 13 : 169);
+            const int sb = a == 0 ? 13 : 1, sc = a == 2 ? 13 : 169;
+            const int b_ax = a == 0 ? 1 : 0, c_ax = a == 2 ? 1 : 2;
+            for (int side = 0; side < 2; ++side) {
+              if (!((omask >> (a + 3 * side)) & 1)) continue;
+              for (int idx = tid; idx < 3 * 169; idx += RT) {
+                const int k3 = idx % 3, uv = idx / 3;
+                const int cb = uv % 13, cc = uv / 13;
+                if (b_ax > a && ((cb < 3 && ((omask >> b_ax) & 1)) || (cb > 9 && ((omask >> (3 + b_ax)) & 1))))
+                  continue;
+                if (c_ax > a && ((cc < 3 && ((omask >> c_ax) & 1)) || (cc > 9 && ((omask >> (3 + c_ax)) & 1))))
+                  continue;
+                const int ia = side == 0 ? k3 : 10 + k3;
+                const int base = cb * sb + cc * sc;
+                double acc = 0.0;
+                if (side == 0) {
+                  const double* w = c_rWEXT + (2 - ia) * 7;
+#pragma unroll
+                  for (int mm = 0; mm < 7; ++mm) acc = fma(w[mm], sw[base + (3 + mm) * sa], acc);
+                } else {
+                  const double* w = c_rWEXT + (ia - 10) * 7;
+#pragma unroll
+                  for (int mm = 0; mm < 7; ++mm) acc = fma(w[mm], sw[base + (9 - mm) * sa], acc);
+                }
+                sw[base + ia * sa] = acc;
+              }
+            }
+            __syncthreads();
+          }
+        }
+      } else {
+        mbar_wait(&bars[buf], (g >> 1) & 1);
+      }
+      const double* s = stage + buf * STAGE_DBL;
+      // cooperative D1 pass (as in k_rhs)
+      if (tid < N_TXL) {
+        int y, z;
+        if (tid < 91) {
+          z = 3 + tid / 13;
+          y = tid % 13;
+        } else {
+          const int r2 = tid - 91, zz = r2 / 7;
+          z = zz < 3 ? zz : zz + 7;
+          y = 3 + r2 % 7;
+        }
+        const int b = 13 * y + 169 * z;
+        double v[13];
+#pragma unroll
+        for (int k = 0; k < 13; ++k) v[k] = s[b + k];
+#pragma unroll
+        for (int x = 3; x <= 9; ++x)
+          Tx[b + x - TX_OFF] = (v[x + 1] - v[x - 1]) * 45.0 - (v[x + 2] - v[x - 2]) * 9.0 +
+                               (v[x + 3] - v[x - 3]);
+      } else if (tid < N_TXL + N_TYL) {
+        const int qq = tid - N_TXL;
+        const int b = (3 + qq % 7) + 169 * (qq / 7);
+        double v[13];
+#pragma unroll
+        for (int k = 0; k < 13; ++k) v[k] = s[b + 13 * k];
+#pragma unroll
+        for (int y = 3; y <= 9; ++y)
+          Ty[b + 13 * y - TY_OFF] = (v[y + 1] - v[y - 1]) * 45.0 - (v[y + 2] - v[y - 2]) * 9.0 +
+                                    (v[y + 3] - v[y - 3]);
+      }
+      __syncthreads();
+      if (c0 >= 0) {
+        const Derivs d = derivs2(s, Tx, Ty, c0, ih, ko_scale);
+#pragma unroll
+        for (int k = 0; k < 3; ++k) out[(6 * k + q) * ostr] = d.d1[k];
+        out[(18 + q) * ostr] = trace6(gi, d.dd);
+        out[(24 + q) * ostr] = beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
+      }
+      __syncthreads();   // everyone is done with this stage buffer and with Tx/Ty
+      const bool last = q >= 4;   // stages q+2 belong to the next octant
+      if (FUSED) {
+        double* dst = stage + buf * STAGE_DBL;
+        if (!last) {
+          gather(dst, 12 + q + 2);
+        } else {
+          if (q == 4 && en >= 0) load_gidx(en);
+          if (en >= 0) gather(dst, 12 + q + 2 - 6);
+          else cp_async_commit();
+        }
+      } else if (tid == 0) {
+        if (!last)
+          bulk_load(stage + buf * STAGE_DBL, patches + int64_t(e) * PATCH_PITCH + (12 + q + 2) * fstride,
+                    STAGE_DBL * 8, &bars[buf]);
+        else if (en >= 0)
+          bulk_load(stage + buf * STAGE_DBL,
+                    patches + int64_t(en) * PATCH_PITCH + (12 + q + 2 - 6) * fstride, STAGE_DBL * 8,
+                    &bars[buf]);
+      }
+    }
+  }
+}
+
 size_t rhs_smem_bytes() { return SMEM_BYTES; }
 
 #ifdef DGR_RHS_TIMING
@@ -926,31 +1184,43 @@ void upload_rhs_tables(const double* wext) {
 }
 
 void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const RhsParams& p,
-                bool fused, int64_t first, int64_t count, int leave_sm, cudaStream_t s) {
+                bool fused, int64_t first, int64_t count, int leave_sm, cudaStream_t s,
+                double* pre) {
   if (count <= 0) return;
   static int n_sm = 0;
   if (!n_sm) {
-    cudaFuncSetAttribute(k_rhs<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(SMEM_BYTES));
-    cudaFuncSetAttribute(k_rhs<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(SMEM_BYTES));
-    cudaFuncSetAttribute(k_rhs<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(SMEM_BYTES));
-    cudaFuncSetAttribute(k_rhs<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(SMEM_BYTES));
+    const int sb = int(SMEM_BYTES);
+    cudaFuncSetAttribute(k_rhs<false, false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb);
+    cudaFuncSetAttribute(k_rhs<true, false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb);
+    cudaFuncSetAttribute(k_rhs<false, true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb);
+    cudaFuncSetAttribute(k_rhs<true, true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb);
+    cudaFuncSetAttribute(k_rhs<true, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb);
+    cudaFuncSetAttribute(k_gt_pre<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         int(PRE_SMEM_BYTES));
     int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&n_sm, cudaDevAttrMultiProcessorCount, dev);
     if (n_sm <= 0) n_sm = 148;
   }
-  // persistent: one CTA per SM (225 KB of shared memory each)
+  // persistent: one CTA per SM (227 KB of shared memory each)
   const int64_t cap = leave_sm > 0 && n_sm - leave_sm > 0 ? n_sm - leave_sm : n_sm;
   const int grid = int(count < cap ? count : cap);
   const bool somm = p.sommerfeld && !m.periodic;
-  if (fused && !somm)
-    k_rhs<true, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, int(first), int(count));
+  const int a = int(first), c = int(count);
+  if (fused && pre && !somm) {
+    // metric pre-pass (two CTAs per SM), then the 18 remaining fields
+    const int64_t cap2 = 2 * cap;
+    const int grid2 = int(count < cap2 ? count : cap2);
+    k_gt_pre<true><<<grid2, RT, PRE_SMEM_BYTES, s>>>(m, patches, pre, p, a, c);
+    k_rhs<true, false, true><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, pre);
+  } else if (fused && !somm)
+    k_rhs<true, false, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr);
   else if (fused)
-    k_rhs<true, true><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, int(first), int(count));
+    k_rhs<true, true, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr);
   else if (!somm)
-    k_rhs<false, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, int(first), int(count));
+    k_rhs<false, false, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr);
   else
-    k_rhs<false, true><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, int(first), int(count));
+    k_rhs<false, true, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr);
 }
 
 }  // namespace dgr

@@ -121,6 +121,22 @@ def test_fused_unzip_equals_two_pass(case):
     assert torch.equal(r, two), float((r - two).abs().max())
 
 
+def test_metric_prepass_bit_identical(case):
+    """The metric pre-pass split (k_gt_pre + k_rhs on the other 18 fields,
+    DGR_OPT_PREPASS, the default) reproduces the single-kernel RHS bit for bit,
+    for dgr_rhs and for a whole RK4 step."""
+    name, cfg, om, m, u = case
+    ud = to_dev(u, m.dof_stride)
+    r1 = m.rhs(ud)
+    s1 = m.rk4_step(ud.clone(), 1e-3)
+    m.set_prepass(False)
+    r0 = m.rhs(ud)
+    s0 = m.rk4_step(ud.clone(), 1e-3)
+    m.set_prepass(True)
+    assert torch.equal(r0, r1), float((r0 - r1).abs().max())
+    assert torch.equal(s0, s1), float((s0 - s1).abs().max())
+
+
 def test_rk4_step_parity(case):
     name, cfg, om, m, u = case
     dt = ork4.dt_courant(om)

@@ -827,9 +827,11 @@ static dgr_status rhs_oct(dgr_mesh m, double* u, const dgr_params* prm, cudaStre
     if ((s = exchange(m, u, st))) return s;
     if ((s = do_interp(m, u, NF, st, 0))) return s;
     PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, ni, 0, st, pre));
+    if (pre) ++m->launches;   // (k_gt_pre + k_rhs)
     if (m->phases == 1) {
       if ((s = do_interp(m, u, NF, st, 1))) return s;
       PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, ni, no - ni, 0, st, pre));
+    if (pre) ++m->launches;   // (k_gt_pre + k_rhs)
     }
   } else if (overlap) {
     if (!m->xstream) {
@@ -843,13 +845,16 @@ static dgr_status rhs_oct(dgr_mesh m, double* u, const dgr_params* prm, cudaStre
     CUDA_TRY(cudaEventRecord(m->ev_xdone, m->xstream));
     if ((s = do_interp(m, u, NF, st, 0))) return s;
     PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, ni, m->xsm, st, pre));
+    if (pre) ++m->launches;   // (k_gt_pre + k_rhs)
     CUDA_TRY(cudaStreamWaitEvent(st, m->ev_xdone, 0));
     if ((s = do_interp(m, u, NF, st, 1))) return s;
     PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, ni, no - ni, 0, st, pre));
+    if (pre) ++m->launches;   // (k_gt_pre + k_rhs)
   } else {
     if ((s = exchange(m, u, st))) return s;
     if ((s = do_interp(m, u, NF, st))) return s;
     PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, no, 0, st, pre));
+    if (pre) ++m->launches;   // (k_gt_pre + k_rhs)
   }
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;

@@ -943,19 +943,22 @@ __global__ void __launch_bounds__(RT, 1)
 // Same stencils, same gather/extrapolation and same arithmetic order as the
 // gt stages of k_rhs, so both paths give bit-identical results.
 constexpr int NPRE = 30;
-constexpr size_t PRE_SMEM_BYTES = size_t(2) * STAGE_DBL * 8 + size_t(TX_N + TY_N) * 8 + 16 +
+constexpr int PRE_NBUF = 3;   // stage ring depth of the pre-pass
+constexpr size_t PRE_SMEM_BYTES = size_t(PRE_NBUF) * STAGE_DBL * 8 + size_t(TX_N + TY_N) * 8 +
                                   size_t(2) * RT * 2;
 
-template <bool FUSED>
+// Fused path only (patches gathered from u and the slots).  Three-deep stage
+// ring: the CTA barrier that releases stage g's data also proves every thread
+// is done with stage g-1, whose buffer then receives stage g+2 (two stages of
+// latency cover, two barriers per field).
 __global__ void __launch_bounds__(RT, 2)
     k_gt_pre(DevMesh m, const double* __restrict__ patches, double* __restrict__ pre,
              RhsParams prm, int first, int count) {
   extern __shared__ __align__(128) double smem[];
-  double* stage = smem;                           // [2][STAGE_DBL]
-  double* Tx = stage + 2 * STAGE_DBL;             // [TX_N]
+  double* stage = smem;                           // [PRE_NBUF][STAGE_DBL]
+  double* Tx = stage + PRE_NBUF * STAGE_DBL;      // [TX_N]
   double* Ty = Tx + TX_N;                         // [TY_N]
-  uint64_t* bars = reinterpret_cast<uint64_t*>(Ty + TY_N);
-  int16_t* tab_c0 = reinterpret_cast<int16_t*>(bars + 2);
+  int16_t* tab_c0 = reinterpret_cast<int16_t*>(Ty + TY_N);
   int16_t* tab_p = tab_c0 + RT;
   const int tid = threadIdx.x;
   {
@@ -965,7 +968,7 @@ __global__ void __launch_bounds__(RT, 2)
     tab_p[tid] = int16_t(q);
   }
   const int64_t no = m.n_owned;
-  const int64_t fstride = FUSED ? m.dof_stride : no * PATCH_PITCH;
+  const int64_t fstride = m.dof_stride;
   const int32_t ds = int32_t(m.dof_stride);
   const int32_t* ol = m.olist + first;
   int li = blockIdx.x;
@@ -989,20 +992,10 @@ __global__ void __launch_bounds__(RT, 2)
     if (tid + RT * (GJ - 1) < NPATCH) cp_async8(d0 + 8 * RT * (GJ - 1), uf, af, gidx[GJ - 1], ds);
     cp_async_commit();
   };
-  if (tid == 0) {
-    mbar_init(&bars[0], 1);
-    mbar_init(&bars[1], 1);
-  }
   __syncthreads();
-  if (FUSED) {
-    load_gidx(e);
-    gather(stage, 12);
-    gather(stage + STAGE_DBL, 13);
-  } else if (tid == 0) {
-    const double* pb = patches + int64_t(e) * PATCH_PITCH;
-    bulk_load(stage, pb + 12 * fstride, STAGE_DBL * 8, &bars[0]);
-    bulk_load(stage + STAGE_DBL, pb + 13 * fstride, STAGE_DBL * 8, &bars[1]);
-  }
+  load_gidx(e);
+  gather(stage, 12);
+  gather(stage + STAGE_DBL, 13);
   uint32_t g = 0;
   for (; li < count; li += gridDim.x) {
     e = ol[li];
@@ -1011,7 +1004,7 @@ __global__ void __launch_bounds__(RT, 2)
     const int p = tab_p[tid];
     const int4 oi = m.oct[e];
     int omask = 0;
-    if (FUSED && !m.periodic) {
+    if (!m.periodic) {
       const int nside = 1 << m.D, sd = 1 << (m.D - oi.w);
       omask = (oi.x == 0) | ((oi.y == 0) << 1) | ((oi.z == 0) << 2) | ((oi.x + sd == nside) << 3) |
               ((oi.y + sd == nside) << 4) | ((oi.z + sd == nside) << 5);
@@ -1021,9 +1014,8 @@ __global__ void __launch_bounds__(RT, 2)
     // values at the point: gt (for gt^ij) and beta (advection)
     double gi[6] = {0, 0, 0, 0, 0, 0}, beta[3] = {0, 0, 0};
     if (c0 >= 0) {
-      const int cv = FUSED ? __ldg(m.o2s + int64_t(e) * NPT + p) : c0;
+      const int cv = __ldg(m.o2s + int64_t(e) * NPT + p);
       auto own = [&](int f) -> double {
-        if (!FUSED) return __ldg(patches + int64_t(e) * PATCH_PITCH + f * fstride + cv);
         return cv < ds ? __ldg(patches + f * fstride + cv) : __ldg(m.aux + f * m.aux_stride + (cv - ds));
       };
       double gq[6];
@@ -1046,47 +1038,54 @@ __global__ void __launch_bounds__(RT, 2)
     double* out = pre + int64_t(e) * NPT + p;
     const int64_t ostr = no * NPT;
     for (int q = 0; q < 6; ++q, ++g) {
-      const int buf = g & 1;
-      if (FUSED) {
-        cp_async_wait1();
-        __syncthreads();
-        if (omask) {
-          double* sw = stage + buf * STAGE_DBL;
-          for (int a = 0; a < 3; ++a) {
-            const int sa = a == 0 ? 1 : (a == 1 ? 13 : 169);
-            const int sb = a == 0 ? 13 : 1, sc = a == 2 ? 13 : 169;
-            const int b_ax = a == 0 ? 1 : 0, c_ax = a == 2 ? 1 : 2;
-            for (int side = 0; side < 2; ++side) {
-              if (!((omask >> (a + 3 * side)) & 1)) continue;
-              for (int idx = tid; idx < 3 * 169; idx += RT) {
-                const int k3 = idx % 3, uv = idx / 3;
-                const int cb = uv % 13, cc = uv / 13;
-                if (b_ax > a && ((cb < 3 && ((omask >> b_ax) & 1)) || (cb > 9 && ((omask >> (3 + b_ax)) & 1))))
-                  continue;
-                if (c_ax > a && ((cc < 3 && ((omask >> c_ax) & 1)) || (cc > 9 && ((omask >> (3 + c_ax)) & 1))))
-                  continue;
-                const int ia = side == 0 ? k3 : 10 + k3;
-                const int base = cb * sb + cc * sc;
-                double acc = 0.0;
-                if (side == 0) {
-                  const double* w = c_rWEXT + (2 - ia) * 7;
-#pragma unroll
-                  for (int mm = 0; mm < 7; ++mm) acc = fma(w[mm], sw[base + (3 + mm) * sa], acc);
-                } else {
-                  const double* w = c_rWEXT + (ia - 10) * 7;
-#pragma unroll
-                  for (int mm = 0; mm < 7; ++mm) acc = fma(w[mm], sw[base + (9 - mm) * sa], acc);
-                }
-                sw[base + ia * sa] = acc;
-              }
-            }
-            __syncthreads();
-          }
+      const int buf = g % PRE_NBUF;
+      cp_async_wait1();   // this thread's copies of stage g (g+1 may be in flight)
+      __syncthreads();    // everyone's; and everyone is done with stage g-1
+      {
+        // stage g+2 into the buffer of stage g-1
+        double* dst = stage + ((g + 2) % PRE_NBUF) * STAGE_DBL;
+        if (q + 2 < 6) {
+          gather(dst, 12 + q + 2);
+        } else {
+          if (q == 4 && en >= 0) load_gidx(en);
+          if (en >= 0) gather(dst, 12 + q + 2 - 6);
+          else cp_async_commit();
         }
-      } else {
-        mbar_wait(&bars[buf], (g >> 1) & 1);
       }
-      const double* s = stage + buf * STAGE_DBL;
+      double* sw = stage + buf * STAGE_DBL;
+      if (omask) {
+        for (int a = 0; a < 3; ++a) {
+          const int sa = a == 0 ? 1 : (a == 1 ? 13 : 169);
+          const int sb = a == 0 ? 13 : 1, sc = a == 2 ? 13 : 169;
+          const int b_ax = a == 0 ? 1 : 0, c_ax = a == 2 ? 1 : 2;
+          for (int side = 0; side < 2; ++side) {
+            if (!((omask >> (a + 3 * side)) & 1)) continue;
+            for (int idx = tid; idx < 3 * 169; idx += RT) {
+              const int k3 = idx % 3, uv = idx / 3;
+              const int cb = uv % 13, cc = uv / 13;
+              if (b_ax > a && ((cb < 3 && ((omask >> b_ax) & 1)) || (cb > 9 && ((omask >> (3 + b_ax)) & 1))))
+                continue;
+              if (c_ax > a && ((cc < 3 && ((omask >> c_ax) & 1)) || (cc > 9 && ((omask >> (3 + c_ax)) & 1))))
+                continue;
+              const int ia = side == 0 ? k3 : 10 + k3;
+              const int base = cb * sb + cc * sc;
+              double acc = 0.0;
+              if (side == 0) {
+                const double* w = c_rWEXT + (2 - ia) * 7;
+#pragma unroll
+                for (int mm = 0; mm < 7; ++mm) acc = fma(w[mm], sw[base + (3 + mm) * sa], acc);
+              } else {
+                const double* w = c_rWEXT + (ia - 10) * 7;
+#pragma unroll
+                for (int mm = 0; mm < 7; ++mm) acc = fma(w[mm], sw[base + (9 - mm) * sa], acc);
+              }
+              sw[base + ia * sa] = acc;
+            }
+          }
+          __syncthreads();
+        }
+      }
+      const double* s = sw;
       // cooperative D1 pass (as in k_rhs)
       if (tid < N_TXL) {
         int y, z;
@@ -1124,26 +1123,6 @@ __global__ void __launch_bounds__(RT, 2)
         for (int k = 0; k < 3; ++k) out[(6 * k + q) * ostr] = d.d1[k];
         out[(18 + q) * ostr] = trace6(gi, d.dd);
         out[(24 + q) * ostr] = beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
-      }
-      __syncthreads();   // everyone is done with this stage buffer and with Tx/Ty
-      const bool last = q >= 4;   // stages q+2 belong to the next octant
-      if (FUSED) {
-        double* dst = stage + buf * STAGE_DBL;
-        if (!last) {
-          gather(dst, 12 + q + 2);
-        } else {
-          if (q == 4 && en >= 0) load_gidx(en);
-          if (en >= 0) gather(dst, 12 + q + 2 - 6);
-          else cp_async_commit();
-        }
-      } else if (tid == 0) {
-        if (!last)
-          bulk_load(stage + buf * STAGE_DBL, patches + int64_t(e) * PATCH_PITCH + (12 + q + 2) * fstride,
-                    STAGE_DBL * 8, &bars[buf]);
-        else if (en >= 0)
-          bulk_load(stage + buf * STAGE_DBL,
-                    patches + int64_t(en) * PATCH_PITCH + (12 + q + 2 - 6) * fstride, STAGE_DBL * 8,
-                    &bars[buf]);
       }
     }
   }
@@ -1195,7 +1174,7 @@ void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const 
     cudaFuncSetAttribute(k_rhs<false, true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb);
     cudaFuncSetAttribute(k_rhs<true, true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb);
     cudaFuncSetAttribute(k_rhs<true, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb);
-    cudaFuncSetAttribute(k_gt_pre<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaFuncSetAttribute(k_gt_pre, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          int(PRE_SMEM_BYTES));
     int dev = 0;
     cudaGetDevice(&dev);
@@ -1211,7 +1190,7 @@ void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const 
     // metric pre-pass (two CTAs per SM), then the 18 remaining fields
     const int64_t cap2 = 2 * cap;
     const int grid2 = int(count < cap2 ? count : cap2);
-    k_gt_pre<true><<<grid2, RT, PRE_SMEM_BYTES, s>>>(m, patches, pre, p, a, c);
+    k_gt_pre<<<grid2, RT, PRE_SMEM_BYTES, s>>>(m, patches, pre, p, a, c);
     k_rhs<true, false, true><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, pre);
   } else if (fused && !somm)
     k_rhs<true, false, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr);

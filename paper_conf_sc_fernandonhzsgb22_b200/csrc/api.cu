@@ -100,6 +100,8 @@ struct dgr_mesh_s {
   double* d_aux = nullptr;      // [24][aux_stride] interpolation slots
   int32_t* d_o2s = nullptr;     // [n_local][343] element node -> u / slot index
   int32_t* d_gmap = nullptr;    // [n_owned][GM_PITCH] patch point -> u / slot index
+  int32_t* d_gmap_s = nullptr;  // [n_owned][GM_PITCH] the same entries sorted by source
+  int16_t* d_gdst = nullptr;    // [n_owned][GM_PITCH] patch point of each sorted entry
   // k_interp launch ranges, one per dependency depth, per phase: phase 0 =
   // slot elements whose values depend on owned DOFs only, phase 1 = the rest
   // (they wait for the ghost exchange; empty on one rank)
@@ -494,6 +496,27 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
     aux_stride = std::max<int64_t>(32, ((slot + 31) / 32) * 32);
     CUDA_TRY(m->alloc(&m->d_o2s, o2s.size()));
     CUDA_TRY(cudaMemcpy(m->d_o2s, o2s.data(), o2s.size() * 4, cudaMemcpyHostToDevice));
+    {
+      // the fused kernels' gather order: each octant's entries sorted by source
+      // index, so a warp's 32 copies read few distinct lines (fewer
+      // shared-memory write wavefronts per cp.async); gdst keeps the patch point
+      std::vector<int32_t> gs(gm.size(), -1);
+      std::vector<int16_t> gd(gm.size(), 0);
+      std::vector<int> idx(NPATCH);
+      for (int64_t e = 0; e < no; ++e) {
+        const int32_t* row = gm.data() + size_t(e) * GM_PITCH;
+        for (int p = 0; p < NPATCH; ++p) idx[p] = p;
+        std::stable_sort(idx.begin(), idx.end(), [&](int a, int b) { return row[a] < row[b]; });
+        for (int k = 0; k < NPATCH; ++k) {
+          gs[size_t(e) * GM_PITCH + k] = row[idx[k]];
+          gd[size_t(e) * GM_PITCH + k] = int16_t(idx[k]);
+        }
+      }
+      CUDA_TRY(m->alloc(&m->d_gmap_s, gs.size()));
+      CUDA_TRY(cudaMemcpy(m->d_gmap_s, gs.data(), gs.size() * 4, cudaMemcpyHostToDevice));
+      CUDA_TRY(m->alloc(&m->d_gdst, gd.size()));
+      CUDA_TRY(cudaMemcpy(m->d_gdst, gd.data(), gd.size() * 2, cudaMemcpyHostToDevice));
+    }
     CUDA_TRY(m->alloc(&m->d_gmap, gm.size()));
     CUDA_TRY(cudaMemcpy(m->d_gmap, gm.data(), gm.size() * 4, cudaMemcpyHostToDevice));
     CUDA_TRY(m->alloc(&m->d_iel, iel.size()));
@@ -539,6 +562,8 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
   dm.o2s = m->d_o2s;
   dm.gmap = m->d_gmap;
   dm.olist = m->d_olist;
+  dm.gmap_s = m->d_gmap_s;
+  dm.gdst = m->d_gdst;
   dm.iel = m->d_iel;
   dm.igrp = m->d_igrp;
   dm.ipt = m->d_ipt;

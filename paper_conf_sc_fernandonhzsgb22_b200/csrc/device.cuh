@@ -38,6 +38,10 @@ struct DevMesh {
   // gmap[e][p]: index of patch point p of owned octant e, -1 outside a
   // non-periodic domain (extrapolated)
   const int32_t* gmap;      // [n_owned * GM_PITCH]
+  // the fused kernels' gather: gmap entries sorted by source index (gmap_s)
+  // and the patch point each one fills (gdst)
+  const int32_t* gmap_s;
+  const int16_t* gdst;
   // RHS octant order: interior octants (no ghost-dependent gather source)
   // first, then the boundary octants (api.cu, overlap of the ghost exchange)
   const int32_t* olist;     // [n_owned]

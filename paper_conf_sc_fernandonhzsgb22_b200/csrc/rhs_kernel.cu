@@ -270,22 +270,26 @@ __global__ void __launch_bounds__(RT, 1)
   const int64_t fstride = FUSED ? m.dof_stride : no * PATCH_PITCH;
   const int32_t ds = int32_t(m.dof_stride);
   int gidx[GJ];   // FUSED: SRC index of patch points tid + RT*j of the current octant
+  int gdst[GJ];   // FUSED: patch point each of this thread's copies fills
   auto load_gidx = [&](int oct) {
-    const int32_t* gm = m.gmap + int64_t(oct) * GM_PITCH;
+    // entries sorted by source (m.gmap_s): a warp's copies read few lines
+    const int32_t* gm = m.gmap_s + int64_t(oct) * GM_PITCH;
+    const int16_t* gd = m.gdst + int64_t(oct) * GM_PITCH;
 #pragma unroll
     for (int j = 0; j < GJ; ++j) {
       const int pt = tid + RT * j;
       // (extrapolated points, -1, copy a dummy value and are overwritten later)
       gidx[j] = pt < NPATCH ? max(__ldg(gm + pt), 0) : -1;
+      gdst[j] = pt < NPATCH ? int(__ldg(gd + pt)) : 0;
     }
   };
   auto gather = [&](double* dst, int f) {
-    const uint32_t d0 = smem_u32(dst + tid);
+    const uint32_t d0 = smem_u32(dst);
     const double* uf = patches + f * fstride;
     const double* af = m.aux + f * m.aux_stride - m.dof_stride;
 #pragma unroll
-    for (int j = 0; j < GJ - 1; ++j) cp_async8(d0 + 8 * RT * j, uf, af, gidx[j], ds);
-    if (tid + RT * (GJ - 1) < NPATCH) cp_async8(d0 + 8 * RT * (GJ - 1), uf, af, gidx[GJ - 1], ds);
+    for (int j = 0; j < GJ - 1; ++j) cp_async8(d0 + 8 * gdst[j], uf, af, gidx[j], ds);
+    if (tid + RT * (GJ - 1) < NPATCH) cp_async8(d0 + 8 * gdst[GJ - 1], uf, af, gidx[GJ - 1], ds);
     cp_async_commit();
   };
   // FUSED: the value of field f at element node (e, p), through o2s
@@ -975,21 +979,24 @@ __global__ void __launch_bounds__(RT, 2)
   if (li >= count) return;
   int e = ol[li];
   int gidx[GJ];
+  int gdst[GJ];
   auto load_gidx = [&](int oct) {
-    const int32_t* gm = m.gmap + int64_t(oct) * GM_PITCH;
+    const int32_t* gm = m.gmap_s + int64_t(oct) * GM_PITCH;
+    const int16_t* gd = m.gdst + int64_t(oct) * GM_PITCH;
 #pragma unroll
     for (int j = 0; j < GJ; ++j) {
       const int pt = tid + RT * j;
       gidx[j] = pt < NPATCH ? max(__ldg(gm + pt), 0) : -1;
+      gdst[j] = pt < NPATCH ? int(__ldg(gd + pt)) : 0;
     }
   };
   auto gather = [&](double* dst, int f) {
-    const uint32_t d0 = smem_u32(dst + tid);
+    const uint32_t d0 = smem_u32(dst);
     const double* uf = patches + f * fstride;
     const double* af = m.aux + f * m.aux_stride - m.dof_stride;
 #pragma unroll
-    for (int j = 0; j < GJ - 1; ++j) cp_async8(d0 + 8 * RT * j, uf, af, gidx[j], ds);
-    if (tid + RT * (GJ - 1) < NPATCH) cp_async8(d0 + 8 * RT * (GJ - 1), uf, af, gidx[GJ - 1], ds);
+    for (int j = 0; j < GJ - 1; ++j) cp_async8(d0 + 8 * gdst[j], uf, af, gidx[j], ds);
+    if (tid + RT * (GJ - 1) < NPATCH) cp_async8(d0 + 8 * gdst[GJ - 1], uf, af, gidx[GJ - 1], ds);
     cp_async_commit();
   };
   __syncthreads();

@@ -114,7 +114,7 @@ struct dgr_mesh_s {
   int xsm = 8;                      // SMs k_rhs leaves to NCCL while overlapping
   int phases = 0;                   // DGR_OPT_PHASES
   bool prepass = true;              // DGR_OPT_PREPASS: gt_ij stages in k_gt_pre
-  double* d_pre = nullptr;          // [30][n_owned][343] metric pre-pass results
+  double* d_pre = nullptr;          // [30][n_owned][352] metric pre-pass results (by thread)
   cudaEvent_t ev_ready = nullptr, ev_xdone = nullptr;
   int4* d_iel = nullptr;        // interpolation work per element with slots
   int4* d_igrp = nullptr;       // ... per face group of its slots
@@ -835,7 +835,7 @@ static dgr_status rhs_oct(dgr_mesh m, double* u, const dgr_params* prm, cudaStre
   const RhsParams rp = to_rp(prm);
   double* pre = nullptr;
   if (m->fused && m->prepass && !(rp.sommerfeld && !m->host.periodic)) {
-    if (!m->d_pre) CUDA_TRY(m->alloc(&m->d_pre, size_t(30) * no * NPT));
+    if (!m->d_pre) CUDA_TRY(m->alloc(&m->d_pre, size_t(30) * no * 352));
     pre = m->d_pre;
   }
   if (!m->fused) {

@@ -374,8 +374,9 @@ __global__ void __launch_bounds__(RT, 1)
   if (PRE && active) {
     // metric pre-pass results -> d gt (S0), gt^lm d_lm gt (A_AT), adv + KO of gt
     // (A_GAM) slots, asynchronously, in flight while the values are read
-    const double* pr = pre + int64_t(e) * NPT + tab_p[tid];
-    const int64_t pstr = no * NPT;
+    // (pre rows are indexed by thread, [c][n_owned][RT]: coalesced)
+    const double* pr = pre + int64_t(e) * RT + tid;
+    const int64_t pstr = no * RT;
 #pragma unroll
     for (int i = 0; i < 18; ++i) cp_async8u(smem_u32(&SL(S0 + i)), pr + i * pstr);
 #pragma unroll
@@ -939,7 +940,7 @@ __global__ void __launch_bounds__(RT, 1)
 // gt_q (second derivatives) without any cross-field state, so two CTAs fit on
 // an SM twice (22 warps instead of 11; three CTAs per SM, at 56 registers,
 // measured slower: 1.99 vs 1.53 ms on C3).  Per interior point it writes 30 values to
-// pre[c][n_owned][343]:
+// pre[c][n_owned][352] (indexed by the thread of the point, as in k_rhs):
 //   c = 6k + q   d_k gt_q                       (k = 0..2, q = 0..5)
 //   c = 18 + q   gt^lm d_l d_m gt_q             (the -1/2 term of Rt, eq 17)
 //   c = 24 + q   beta^k d_k gt_q + KO(gt_q)     (eq 4 advection + dissipation)
@@ -1042,8 +1043,9 @@ __global__ void __launch_bounds__(RT, 2)
       gi[4] = (gq[1] * gq[2] - gq[0] * gq[4]) * idet;
       gi[5] = (gq[0] * gq[3] - gq[1] * gq[1]) * idet;
     }
-    double* out = pre + int64_t(e) * NPT + p;
-    const int64_t ostr = no * NPT;
+    // rows indexed by thread (the same thread -> point map as k_rhs): coalesced
+    double* out = pre + int64_t(e) * RT + tid;
+    const int64_t ostr = no * RT;
     for (int q = 0; q < 6; ++q, ++g) {
       const int buf = g % PRE_NBUF;
       cp_async_wait1();   // this thread's copies of stage g (g+1 may be in flight)

@@ -505,8 +505,22 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
       std::vector<int> idx(NPATCH);
       for (int64_t e = 0; e < no; ++e) {
         const int32_t* row = gm.data() + size_t(e) * GM_PITCH;
+        // groups: cross points (at most one coordinate in the padding: all a
+        // first-derivative stencil reads, G_CROSS of them), then the slabs
+        // (two: the rest of what the D1 pass and mixed stencils read,
+        // G_SLABS in total), then the 216 corners (read by nothing); sorted
+        // by source inside each group
+        auto grp = [](int p) {
+          const int t[3] = {p % 13, (p / 13) % 13, p / 169};
+          int out = 0;
+          for (int a = 0; a < 3; ++a) out += (t[a] < 3 || t[a] > 9);
+          return out <= 1 ? 0 : (out == 2 ? 1 : 2);
+        };
         for (int p = 0; p < NPATCH; ++p) idx[p] = p;
-        std::stable_sort(idx.begin(), idx.end(), [&](int a, int b) { return row[a] < row[b]; });
+        std::stable_sort(idx.begin(), idx.end(), [&](int a, int b) {
+          const int ga = grp(a), gb = grp(b);
+          return ga != gb ? ga < gb : row[a] < row[b];
+        });
         for (int k = 0; k < NPATCH; ++k) {
           gs[size_t(e) * GM_PITCH + k] = row[idx[k]];
           gd[size_t(e) * GM_PITCH + k] = int16_t(idx[k]);

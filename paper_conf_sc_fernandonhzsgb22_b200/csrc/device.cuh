@@ -11,6 +11,11 @@ constexpr int NF = 24;            // BSSN fields
 constexpr int PATCH_PITCH = 2208; // doubles per patch: 13^3 = 2197 padded to 128 B
 constexpr int STAGE_DBL = 2200;   // smem stage buffer (bulk copy of 2200 doubles)
 constexpr int GM_PITCH = 2200;    // int32 per octant in the fused-unzip gather map (16-B rows)
+// sorted gather rows (gmap_s): the first G_CROSS entries are the points a
+// first-derivative stencil reads, the first G_SLABS those any stencil or the
+// D1 pass reads (the 216 corner points come last and are never read)
+constexpr int G_CROSS = 343 + 6 * 3 * 49;          // 1225
+constexpr int G_SLABS = 2197 - 8 * 27;             // 1981
 
 // Device view of a mesh (plain pointers; passed by value to kernels).
 struct DevMesh {

@@ -284,12 +284,16 @@ __global__ void __launch_bounds__(RT, 1)
     }
   };
   auto gather = [&](double* dst, int f) {
+    // only the points the field's stencils read: the cross region for the
+    // first-derivative-only fields, the three slabs for the others
+    const bool sec = f <= 1 || (f >= 6 && f <= 8) || (f >= 12 && f <= 17);
+    const int n = sec ? G_SLABS : G_CROSS;
     const uint32_t d0 = smem_u32(dst);
     const double* uf = patches + f * fstride;
     const double* af = m.aux + f * m.aux_stride - m.dof_stride;
 #pragma unroll
-    for (int j = 0; j < GJ - 1; ++j) cp_async8(d0 + 8 * gdst[j], uf, af, gidx[j], ds);
-    if (tid + RT * (GJ - 1) < NPATCH) cp_async8(d0 + 8 * gdst[GJ - 1], uf, af, gidx[GJ - 1], ds);
+    for (int j = 0; j < GJ; ++j)
+      if (tid + RT * j < n) cp_async8(d0 + 8 * gdst[j], uf, af, gidx[j], ds);
     cp_async_commit();
   };
   // FUSED: the value of field f at element node (e, p), through o2s
@@ -992,12 +996,13 @@ __global__ void __launch_bounds__(RT, 2)
     }
   };
   auto gather = [&](double* dst, int f) {
+    // (gt fields: the three slabs the stencils and the D1 pass read)
     const uint32_t d0 = smem_u32(dst);
     const double* uf = patches + f * fstride;
     const double* af = m.aux + f * m.aux_stride - m.dof_stride;
 #pragma unroll
-    for (int j = 0; j < GJ - 1; ++j) cp_async8(d0 + 8 * gdst[j], uf, af, gidx[j], ds);
-    if (tid + RT * (GJ - 1) < NPATCH) cp_async8(d0 + 8 * gdst[GJ - 1], uf, af, gidx[GJ - 1], ds);
+    for (int j = 0; j < GJ; ++j)
+      if (tid + RT * j < G_SLABS) cp_async8(d0 + 8 * gdst[j], uf, af, gidx[j], ds);
     cp_async_commit();
   };
   __syncthreads();

@@ -45,9 +45,9 @@ PAPER_FLOPS_PER_POINT = 5502 + 3998               # eq (21a) numerator per point
 # fused 2 x 12.991e9 + 11.129e9 + 6.736e9 = 43.85e9 FLOP / 8,329,412 points = 5,265
 # (the in-kernel extrapolation adds ~12 FLOP/pt); two-pass 43.75e9 / 8,329,412 = 5,253
 # executed fp64 FLOPs per interior point (2 DFMA + DADD + DMUL thread instructions from
-# ncu, C3): fused = k_gt_pre + k_rhs (profiles/r1h_ncu_flops_fused_prepass.csv), two-pass
+# ncu, C3): fused = k_gt_pre + k_rhs (profiles/r1j_flops.csv), two-pass
 # = the single k_rhs (profiles/r1h_ncu_flops_twopass.csv)
-RHS_EXEC_FLOPS_PER_POINT = {"fused": 5351.4, "two-pass": 5265.0}
+RHS_EXEC_FLOPS_PER_POINT = {"fused": 5358.3, "two-pass": 5265.0}
 # DRAM bytes per launch (dram__bytes_read.sum + dram__bytes_write.sum) from one
 # ncu --set full capture of the C3 workload on 1 GPU, per path
 # (profiles/ncu_traffic_c3.json, written by tools/ncu_traffic.py)

@@ -215,6 +215,23 @@ dgr_status dgr_rk4_stage(dgr_mesh m, int s, double dt, double* u_n, double* u_s,
 /* Device: one RK4 step in place on u (library workspace for stages). */
 dgr_status dgr_rk4_step(dgr_mesh m, double dt, double* u, const dgr_params* prm, void* stream);
 
+/* Host buffers: one RK4 step (as dgr_rk4_step) of each of n independent
+ * host-resident states on this mesh, u_out[j] = step(u_in[j]), j = 0..n-1
+ * (Alg. 1 with the state on the host, for callers without device
+ * memory; u_in[j] == u_out[j] is allowed).  Each u_in[j] / u_out[j] is a host
+ * array in the device state layout, [24][dof_stride] doubles; rows are read
+ * and written for the owned DOFs d < n_dof_owned only (ghost values come from
+ * the exchange).  Page-locked (cudaHostAlloc / torch pin_memory) buffers are
+ * required for the copies to overlap: the host->device copy of state j+1 and
+ * the device->host copy of state j-1 run on two library copy streams while
+ * state j steps on `stream`, through three library-owned device state slots
+ * (allocated on first use, 3 x 24 x dof_stride doubles).  Enqueued on `stream`
+ * like the device calls: u_out[j] is complete when `stream` is; the host
+ * arrays must stay valid until then.  n == 0 is a no-op; a null list or entry
+ * is DGR_ERR_ARG.  Collective when nranks > 1 (every rank passes the same n). */
+dgr_status dgr_rk4_step_host(dgr_mesh m, double dt, int64_t n, const double* const* u_in,
+                             double* const* u_out, const dgr_params* prm, void* stream);
+
 /* Device: constraints H, M^0..2, G^0..2 on the owned DOFs,
  * c[q * dof_stride + d], q = 0..6; norms_host[2q] = RMS, [2q+1] = max |.|
  * over owned DOFs (all ranks).  Synchronises `stream`. */

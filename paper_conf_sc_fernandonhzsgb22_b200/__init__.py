@@ -78,7 +78,8 @@ _lib = None
 EXPORTED = ["dgr_status_string", "dgr_last_error", "dgr_version", "dgr_octree_build",
             "dgr_mesh_create", "dgr_mesh_info_get", "dgr_mesh_export_maps", "dgr_mesh_destroy",
             "dgr_dof_coords", "dgr_unzip", "dgr_ghost_exchange", "dgr_rhs_patches", "dgr_rhs",
-            "dgr_rk4_stage", "dgr_rk4_step", "dgr_constraints", "dgr_last_launch_count",
+            "dgr_rk4_stage", "dgr_rk4_step", "dgr_rk4_step_host", "dgr_constraints",
+            "dgr_last_launch_count",
             "dgr_profile_enable", "dgr_profile_read", "dgr_bench_dfma", "dgr_set_option"]
 PROF_CLASSES = ["elements", "hanging", "unzip", "rhs", "zip_rk4", "exchange", "constraints",
                 "interp"]
@@ -109,6 +110,8 @@ def lib():
         L.dgr_rhs.argtypes = [vp, vp, vp, C.POINTER(_Params), vp]
         L.dgr_rk4_stage.argtypes = [vp, i32, dp, vp, vp, vp, C.POINTER(_Params), vp]
         L.dgr_rk4_step.argtypes = [vp, dp, vp, C.POINTER(_Params), vp]
+        L.dgr_rk4_step_host.argtypes = [vp, dp, i64, C.POINTER(vp), C.POINTER(vp),
+                                        C.POINTER(_Params), vp]
         L.dgr_constraints.argtypes = [vp, vp, vp, vp, C.POINTER(_Params), vp]
         L.dgr_last_launch_count.restype = i64
         L.dgr_last_launch_count.argtypes = [vp]
@@ -119,7 +122,7 @@ def lib():
         for f in ["dgr_octree_build", "dgr_mesh_create", "dgr_mesh_info_get",
                   "dgr_mesh_export_maps", "dgr_mesh_destroy", "dgr_dof_coords", "dgr_unzip",
                   "dgr_ghost_exchange", "dgr_rhs_patches", "dgr_rhs", "dgr_rk4_stage",
-                  "dgr_rk4_step", "dgr_constraints", "dgr_profile_enable", "dgr_profile_read", "dgr_set_option",
+                  "dgr_rk4_step", "dgr_rk4_step_host", "dgr_constraints", "dgr_profile_enable", "dgr_profile_read", "dgr_set_option",
                   "dgr_bench_dfma"]:
             getattr(L, f).restype = i32
         _lib = L
@@ -286,6 +289,25 @@ class Mesh:
         p = (prm or Params())._c()
         _check(lib().dgr_rk4_step(self._h, float(dt), _ptr(u), C.byref(p), _stream()))
         return u
+
+    def rk4_step_host(self, u_in, u_out, dt, prm=None):
+        """One RK4 step of each host state: u_out[j] = step(u_in[j]) (dgr_rk4_step_host).
+        u_in / u_out: lists of contiguous fp64 CPU tensors [24, dof_stride], pinned
+        for copy/compute overlap.  Enqueued on the current stream; the tensors must
+        stay alive until it completes."""
+        import torch
+        if len(u_in) != len(u_out):
+            raise ValueError("u_in and u_out differ in length")
+        for t in list(u_in) + list(u_out):
+            if (t.device.type != "cpu" or not t.is_contiguous() or t.dtype != torch.float64
+                    or tuple(t.shape) != (24, self.dof_stride)):
+                raise ValueError("host states must be contiguous fp64 CPU [24, dof_stride]")
+        n = len(u_in)
+        ins = (C.c_void_p * max(n, 1))(*[t.data_ptr() for t in u_in])
+        outs = (C.c_void_p * max(n, 1))(*[t.data_ptr() for t in u_out])
+        p = (prm or Params())._c()
+        _check(lib().dgr_rk4_step_host(self._h, float(dt), n, ins, outs, C.byref(p), _stream()))
+        return u_out
 
     def constraints(self, u, prm=None, out=None):
         import torch

@@ -125,6 +125,11 @@ struct dgr_mesh_s {
   double* d_us = nullptr;       // RK4 stage state [24][dof_stride]
   double* d_acc = nullptr;      // RK4 accumulator
   double* d_cnorm = nullptr;    // constraint norm partials
+  // dgr_rk4_step_host: three device state slots, copy streams and events
+  // (allocated on first use)
+  double* d_hbuf[3] = {nullptr, nullptr, nullptr};
+  cudaStream_t h2d = nullptr, d2h = nullptr;
+  cudaEvent_t ev_in[3] = {}, ev_done[3] = {}, ev_out[3] = {}, ev_host0 = nullptr;
   // multi-rank
   void* comm = nullptr;
   int32_t* d_send = nullptr;
@@ -164,6 +169,14 @@ struct dgr_mesh_s {
     if (ev_ready) cudaEventDestroy(ev_ready);
     if (ev_xdone) cudaEventDestroy(ev_xdone);
     if (xstream) cudaStreamDestroy(xstream);
+    for (int b = 0; b < 3; ++b) {
+      if (ev_in[b]) cudaEventDestroy(ev_in[b]);
+      if (ev_done[b]) cudaEventDestroy(ev_done[b]);
+      if (ev_out[b]) cudaEventDestroy(ev_out[b]);
+    }
+    if (ev_host0) cudaEventDestroy(ev_host0);
+    if (h2d) cudaStreamDestroy(h2d);
+    if (d2h) cudaStreamDestroy(d2h);
   }
 };
 
@@ -985,6 +998,64 @@ dgr_status dgr_rk4_step(dgr_mesh m, double dt, double* u, const dgr_params* prm,
   m->launches = 0;
   for (int k = 0; k < 4; ++k)
     if ((s = stage(m, k, dt, u, m->d_us, m->d_acc, u, prm, st))) return s;
+  return DGR_OK;
+}
+
+// n independent host-resident states, one RK4 step each, through three device
+// slots: the H2D copy of state j+1 (h2d stream) and the D2H copy of state j-1
+// (d2h stream) run on the copy engines while state j steps on `stream`.
+// Slot b = j % 3 is reused by state j+3 only after state j's D2H completed.
+dgr_status dgr_rk4_step_host(dgr_mesh m, double dt, int64_t n, const double* const* u_in,
+                             double* const* u_out, const dgr_params* prm, void* stream) {
+  dgr_status s = need_device(m);
+  if (s) return s;
+  if (n < 0 || (n > 0 && (!u_in || !u_out))) return fail(DGR_ERR_ARG, "bad host state lists");
+  for (int64_t j = 0; j < n; ++j)
+    if (!u_in[j] || !u_out[j]) return fail(DGR_ERR_ARG, "null host state");
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  m->launches = 0;
+  if (n == 0) return DGR_OK;
+  const int64_t stride = m->dm.dof_stride;
+  const size_t pitch = size_t(stride) * 8;
+  const size_t width = size_t(m->host.n_owned_dof) * 8;   // ghosts come from the exchange
+  const int nb = n < 3 ? int(n) : 3;
+  for (int b = 0; b < nb; ++b)
+    if (!m->d_hbuf[b]) {
+      CUDA_TRY(m->alloc(&m->d_hbuf[b], size_t(NF) * stride));
+      CUDA_TRY(cudaMemset(m->d_hbuf[b], 0, size_t(NF) * pitch));   // ghost rows defined
+    }
+  if (!m->h2d) {
+    CUDA_TRY(cudaStreamCreateWithFlags(&m->h2d, cudaStreamNonBlocking));
+    CUDA_TRY(cudaStreamCreateWithFlags(&m->d2h, cudaStreamNonBlocking));
+    CUDA_TRY(cudaEventCreateWithFlags(&m->ev_host0, cudaEventDisableTiming));
+    for (int b = 0; b < 3; ++b) {
+      CUDA_TRY(cudaEventCreateWithFlags(&m->ev_in[b], cudaEventDisableTiming));
+      CUDA_TRY(cudaEventCreateWithFlags(&m->ev_done[b], cudaEventDisableTiming));
+      CUDA_TRY(cudaEventCreateWithFlags(&m->ev_out[b], cudaEventDisableTiming));
+    }
+  }
+  // the copy streams start after the work already on the caller's stream
+  CUDA_TRY(cudaEventRecord(m->ev_host0, st));
+  CUDA_TRY(cudaStreamWaitEvent(m->h2d, m->ev_host0, 0));
+  CUDA_TRY(cudaStreamWaitEvent(m->d2h, m->ev_host0, 0));
+  for (int64_t j = 0; j < n; ++j) {
+    const int b = int(j % 3);
+    double* ub = m->d_hbuf[b];
+    if (j >= 3) CUDA_TRY(cudaStreamWaitEvent(m->h2d, m->ev_out[b], 0));
+    CUDA_TRY(cudaMemcpy2DAsync(ub, pitch, u_in[j], pitch, width, NF, cudaMemcpyHostToDevice,
+                               m->h2d));
+    CUDA_TRY(cudaEventRecord(m->ev_in[b], m->h2d));
+    CUDA_TRY(cudaStreamWaitEvent(st, m->ev_in[b], 0));
+    for (int k = 0; k < 4; ++k)   // (launch counts accumulate over the n steps)
+      if ((s = stage(m, k, dt, ub, m->d_us, m->d_acc, ub, prm, st))) return s;
+    CUDA_TRY(cudaEventRecord(m->ev_done[b], st));
+    CUDA_TRY(cudaStreamWaitEvent(m->d2h, m->ev_done[b], 0));
+    CUDA_TRY(cudaMemcpy2DAsync(u_out[j], pitch, ub, pitch, width, NF, cudaMemcpyDeviceToHost,
+                               m->d2h));
+    CUDA_TRY(cudaEventRecord(m->ev_out[b], m->d2h));
+  }
+  // the caller's stream completes after the last D2H copy
+  CUDA_TRY(cudaStreamWaitEvent(st, m->ev_out[(n - 1) % 3], 0));
   return DGR_OK;
 }
 

@@ -254,7 +254,12 @@ dgr_status dgr_constraints(dgr_mesh m, double* u, double* c, double* norms_host,
  *     kernel (two CTAs per SM, 30 values per point through HBM) and the other
  *     18 fields in the RHS kernel; 0 = all 24 fields in the RHS kernel.  Both
  *     give bit-identical results. */
-enum { DGR_OPT_FUSED_UNZIP = 1, DGR_OPT_PHASES = 2, DGR_OPT_PREPASS = 3 };
+/*   DGR_OPT_ZIP_STORE (default 1): fused path without the radiative boundary
+ *     zips in the RHS kernel's store (each point writes its 24 values to the
+ *     DOF it is the zip owner of) and the RK4 update streams the
+ *     DOF-ordered RHS; 0 = RHS per octant point, then the zip gather (k_zip /
+ *     k_zip_rk4).  Both give bit-identical results. */
+enum { DGR_OPT_FUSED_UNZIP = 1, DGR_OPT_PHASES = 2, DGR_OPT_PREPASS = 3, DGR_OPT_ZIP_STORE = 4 };
 dgr_status dgr_set_option(dgr_mesh m, int option, int64_t value);
 
 /* Device-side timing helper for benchmarks: number of kernel launches the last

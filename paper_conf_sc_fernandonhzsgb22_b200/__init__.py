@@ -27,7 +27,7 @@ NPATCH = 2197
 MAP_OCTANTS, MAP_O2N, MAP_HANGING, MAP_PAD_SRC, MAP_PAD_KIND, MAP_ZIP = 0, 1, 2, 3, 4, 5
 MAP_DOF_GID, MAP_DOF_XYZ, MAP_SEND, MAP_SEND_COUNTS, MAP_RECV_COUNTS = 6, 7, 8, 9, 10
 MAP_LOCAL_OCTS, MAP_O2N_LOCAL, MAP_RHS_ORDER = 11, 12, 13
-OPT_FUSED_UNZIP, OPT_PHASES, OPT_PREPASS = 1, 2, 3
+OPT_FUSED_UNZIP, OPT_PHASES, OPT_PREPASS, OPT_ZIP_STORE = 1, 2, 3, 4
 
 
 class DgrError(RuntimeError):
@@ -331,6 +331,11 @@ class Mesh:
         """DGR_OPT_PREPASS: gt_ij stages in the metric pre-pass kernel (1) or in the
         RHS kernel (0); bit-identical results."""
         _check(lib().dgr_set_option(self._h, OPT_PREPASS, int(bool(on))))
+
+    def set_zip_store(self, on=True):
+        """DGR_OPT_ZIP_STORE: zip in the RHS kernel's store and stream the RK4 update
+        (1) or write the RHS per octant point and zip-gather it (0); bit-identical."""
+        _check(lib().dgr_set_option(self._h, OPT_ZIP_STORE, int(bool(on))))
 
     def set_phases(self, mode=0):
         """DGR_OPT_PHASES: 0 = overlap interior octants with the ghost exchange when

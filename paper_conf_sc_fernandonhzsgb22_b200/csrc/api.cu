@@ -114,6 +114,8 @@ struct dgr_mesh_s {
   int xsm = 8;                      // SMs k_rhs leaves to NCCL while overlapping
   int phases = 0;                   // DGR_OPT_PHASES
   bool prepass = true;              // DGR_OPT_PREPASS: gt_ij stages in k_gt_pre
+  bool zip_store = true;            // DGR_OPT_ZIP_STORE: k_rhs stores in DOF order
+  double* d_rhs_dof = nullptr;      // [24][dof_stride] RHS in DOF order (RK4 stages)
   double* d_pre = nullptr;          // [30][n_owned][352] metric pre-pass results (by thread)
   cudaEvent_t ev_ready = nullptr, ev_xdone = nullptr;
   int4* d_iel = nullptr;        // interpolation work per element with slots
@@ -584,6 +586,7 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
   dm.pmap = m->d_pmap;
   dm.nbr = m->d_nbr;
   dm.zip = m->d_zip;
+  dm.own = m->d_own;
   dm.aux_stride = aux_stride;
   dm.aux = m->d_aux;
   dm.o2s = m->d_o2s;
@@ -856,7 +859,14 @@ static RhsParams to_rp(const dgr_params* p) {
 // octants whose patches need no ghost value — k_rhs then leaves a few SMs
 // free, since it otherwise holds every SM and the NCCL kernels could not
 // start — and the boundary octants follow once the ghosts have landed.
-static dgr_status rhs_oct(dgr_mesh m, double* u, const dgr_params* prm, cudaStream_t st) {
+// The fused path without the radiative boundary zips in k_rhs's store
+static bool zip_by_store(dgr_mesh m, const dgr_params* prm) {
+  return m->fused && m->zip_store && !(prm && prm->sommerfeld && !m->host.periodic);
+}
+
+// (rhs_dof != nullptr: fused path only, k_rhs zips by its store into rhs_dof)
+static dgr_status rhs_oct(dgr_mesh m, double* u, const dgr_params* prm, cudaStream_t st,
+                          double* rhs_dof = nullptr) {
   dgr_status s;
   const int64_t no = m->dm.n_owned, ni = m->n_interior;
   const RhsParams rp = to_rp(prm);
@@ -878,11 +888,11 @@ static dgr_status rhs_oct(dgr_mesh m, double* u, const dgr_params* prm, cudaStre
     // hook stops here) the rest — no stream overlap
     if ((s = exchange(m, u, st))) return s;
     if ((s = do_interp(m, u, NF, st, 0))) return s;
-    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, ni, 0, st, pre));
+    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, ni, 0, st, pre, rhs_dof));
     if (pre) ++m->launches;   // (k_gt_pre + k_rhs)
     if (m->phases == 1) {
       if ((s = do_interp(m, u, NF, st, 1))) return s;
-      PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, ni, no - ni, 0, st, pre));
+      PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, ni, no - ni, 0, st, pre, rhs_dof));
     if (pre) ++m->launches;   // (k_gt_pre + k_rhs)
     }
   } else if (overlap) {
@@ -896,16 +906,16 @@ static dgr_status rhs_oct(dgr_mesh m, double* u, const dgr_params* prm, cudaStre
     if ((s = exchange(m, u, m->xstream))) return s;
     CUDA_TRY(cudaEventRecord(m->ev_xdone, m->xstream));
     if ((s = do_interp(m, u, NF, st, 0))) return s;
-    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, ni, m->xsm, st, pre));
+    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, ni, m->xsm, st, pre, rhs_dof));
     if (pre) ++m->launches;   // (k_gt_pre + k_rhs)
     CUDA_TRY(cudaStreamWaitEvent(st, m->ev_xdone, 0));
     if ((s = do_interp(m, u, NF, st, 1))) return s;
-    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, ni, no - ni, 0, st, pre));
+    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, ni, no - ni, 0, st, pre, rhs_dof));
     if (pre) ++m->launches;   // (k_gt_pre + k_rhs)
   } else {
     if ((s = exchange(m, u, st))) return s;
     if ((s = do_interp(m, u, NF, st))) return s;
-    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, no, 0, st, pre));
+    PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, no, 0, st, pre, rhs_dof));
     if (pre) ++m->launches;   // (k_gt_pre + k_rhs)
   }
   CUDA_TRY(cudaGetLastError());
@@ -962,6 +972,7 @@ dgr_status dgr_rhs(dgr_mesh m, double* u, double* rhs, const dgr_params* prm, vo
   if (!u || !rhs) return fail(DGR_ERR_ARG, "null state");
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   m->launches = 0;
+  if (zip_by_store(m, prm)) return rhs_oct(m, u, prm, st, rhs);
   if ((s = rhs_oct(m, u, prm, st))) return s;
   PROF(m, 4, st, launch_zip(m->dm, m->d_rhs_oct, rhs, NF, st));
   CUDA_TRY(cudaGetLastError());
@@ -974,7 +985,15 @@ static dgr_status stage(dgr_mesh m, int s_, double dt, double* u_n, double* u_s,
   double* cur = s_ == 0 ? u_n : u_s;
   // (applying the zip + RK4 update inside k_rhs measured 10.6 ms vs 7.5 + 0.8 ms
   // for RHS + k_zip_rk4 on C3 — the scattered state loads stall the single
-  // persistent CTA per SM — so the update is a separate kernel)
+  // persistent CTA per SM — so the update is a separate kernel; the zip itself
+  // is only stores, so k_rhs does it by default: DGR_OPT_ZIP_STORE)
+  if (zip_by_store(m, prm)) {
+    if (!m->d_rhs_dof) CUDA_TRY(m->alloc(&m->d_rhs_dof, size_t(NF) * m->dm.dof_stride));
+    if ((s = rhs_oct(m, cur, prm, st, m->d_rhs_dof))) return s;
+    PROF(m, 4, st, launch_rk4(m->dm, m->d_rhs_dof, s_, dt, u_n, u_s, acc, u_out, st));
+    CUDA_TRY(cudaGetLastError());
+    return DGR_OK;
+  }
   if ((s = rhs_oct(m, cur, prm, st))) return s;
   PROF(m, 4, st, launch_zip_rk4(m->dm, m->d_rhs_oct, s_, dt, u_n, u_s, acc, u_out, st));
   CUDA_TRY(cudaGetLastError());
@@ -1118,6 +1137,7 @@ dgr_status dgr_set_option(dgr_mesh m, int option, int64_t value) {
   switch (option) {
     case DGR_OPT_FUSED_UNZIP: m->fused = value != 0; return DGR_OK;
     case DGR_OPT_PREPASS: m->prepass = value != 0; return DGR_OK;
+    case DGR_OPT_ZIP_STORE: m->zip_store = value != 0; return DGR_OK;
     case DGR_OPT_PHASES:
       if (value < 0 || value > 2) return fail(DGR_ERR_ARG, "DGR_OPT_PHASES is 0, 1 or 2");
       m->phases = int(value);

@@ -32,6 +32,7 @@ struct DevMesh {
   const uint8_t* pmap;      // [n_owned * 2197]
   const NbrEntry* nbr;      // [n_owned * NBR_MAX]
   const int32_t* zip;       // [n_owned_dof] local octant * 343 + node
+  const int32_t* own;       // [n_owned * 343] owned DOF whose zip owner is (e, p), or -1
   // Gather maps.  Index space of every value a patch needs:
   // i < dof_stride -> u[f * dof_stride + i] (a DOF of the state), else
   // aux[f * aux_stride + i - dof_stride] (an interpolation slot: one distinct
@@ -74,6 +75,9 @@ void launch_cnorms(const double* c, int64_t stride, int64_t n, int nq, double* p
                    cudaStream_t s);
 void launch_zip_rk4(const DevMesh& m, const double* rhs_oct, int stage, double dt,
                     const double* u_n, double* u_s, double* acc, double* u_out, cudaStream_t s);
+// RK4 stage update from an already zipped RHS rhs[24][dof_stride] (streaming)
+void launch_rk4(const DevMesh& m, const double* rhs, int stage, double dt, const double* u_n,
+                double* u_s, double* acc, double* u_out, cudaStream_t s);
 void launch_dof_coords(const DevMesh& m, const int64_t* dof_node, double* xyz,
                        const double xmin[3], cudaStream_t s);
 void launch_gather_pack(const double* u, int64_t stride, const int32_t* list, int64_t n,
@@ -95,9 +99,12 @@ struct RhsParams {
 // n_SM - leave_sm persistent CTAs
 // pre != nullptr (fused, no Sommerfeld): the gt_ij stages run in the metric
 // pre-pass k_gt_pre (pre: [30][n_owned][343] scratch), then k_rhs on the rest
+// rhs_dof != nullptr (fused, no Sommerfeld): the zip is done by the store — each
+// point writes its 24 values to rhs_dof[f * dof_stride + d] iff it is the zip
+// owner of DOF d (m.own), and rhs_oct is not written
 void launch_rhs(const DevMesh& m, const double* src, double* rhs_oct, const RhsParams& p,
                 bool fused, int64_t first, int64_t count, int leave_sm, cudaStream_t s,
-                double* pre = nullptr);
+                double* pre = nullptr, double* rhs_dof = nullptr);
 size_t rhs_smem_bytes();
 void upload_rhs_tables(const double* wext);
 

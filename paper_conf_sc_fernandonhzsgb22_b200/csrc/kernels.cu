@@ -69,6 +69,47 @@ __global__ void k_zip_rk4(const int32_t* __restrict__ zip, int32_t n, int64_t no
   }
 }
 
+// The same update from an RHS already in DOF order (written by k_rhs's zip-
+// by-store epilogue): every array is streamed, no zip gather.
+template <int S>
+__global__ void k_rk4(int32_t n, int64_t stride, double dt, const double* __restrict__ rhs,
+                      const double* __restrict__ u_n, double* __restrict__ u_s,
+                      double* __restrict__ acc, double* __restrict__ u_out) {
+  const int f = blockIdx.y;
+  for (int d = blockIdx.x * blockDim.x + threadIdx.x; d < n; d += gridDim.x * blockDim.x) {
+    const int64_t i = f * stride + d;
+    const double k = __ldcs(rhs + i);
+    if (S == 0) {
+      const double un = u_n[i];
+      acc[i] = un + (dt / 6.0) * k;
+      u_s[i] = un + (dt / 2.0) * k;
+    } else if (S == 1) {
+      acc[i] += (dt / 3.0) * k;
+      u_s[i] = u_n[i] + (dt / 2.0) * k;
+    } else if (S == 2) {
+      acc[i] += (dt / 3.0) * k;
+      u_s[i] = u_n[i] + dt * k;
+    } else {
+      u_out[i] = acc[i] + (dt / 6.0) * k;
+    }
+  }
+}
+
+void launch_rk4(const DevMesh& m, const double* rhs, int stage, double dt, const double* u_n,
+                double* u_s, double* acc, double* u_out, cudaStream_t s) {
+  if (m.n_owned_dof <= 0) return;
+  int blocks = (m.n_owned_dof + 255) / 256;
+  if (blocks > 148 * 8) blocks = 148 * 8;
+  const dim3 g(blocks, NF);
+  const int32_t n = m.n_owned_dof;
+  switch (stage) {
+    case 0: k_rk4<0><<<g, 256, 0, s>>>(n, m.dof_stride, dt, rhs, u_n, u_s, acc, u_out); break;
+    case 1: k_rk4<1><<<g, 256, 0, s>>>(n, m.dof_stride, dt, rhs, u_n, u_s, acc, u_out); break;
+    case 2: k_rk4<2><<<g, 256, 0, s>>>(n, m.dof_stride, dt, rhs, u_n, u_s, acc, u_out); break;
+    default: k_rk4<3><<<g, 256, 0, s>>>(n, m.dof_stride, dt, rhs, u_n, u_s, acc, u_out); break;
+  }
+}
+
 // ------------------------------------------------- constraint norms (a7)
 // Sum of squares and max |.| of each of nq rows of c over d < n, in a fixed
 // order (deterministic): per-block partials, then one block per row.

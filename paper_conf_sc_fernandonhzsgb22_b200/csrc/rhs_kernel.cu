@@ -243,7 +243,8 @@ __device__ __forceinline__ double trace6(const double* gi, const double* X) {
 template <bool FUSED, bool SOMM, bool PRE>
 __global__ void __launch_bounds__(RT, 1)
     k_rhs(DevMesh m, const double* __restrict__ patches, double* __restrict__ rhs_oct,
-          RhsParams prm, int first, int count, const double* __restrict__ pre) {
+          RhsParams prm, int first, int count, const double* __restrict__ pre,
+          double* __restrict__ rhs_dof) {
   // PRE: the gt_ij stages were done by k_gt_pre (its 30 values per point are
   // read in the prologue); the stream holds the 18 other fields
   constexpr int NS = PRE ? NF - 6 : NF;
@@ -888,6 +889,8 @@ __global__ void __launch_bounds__(RT, 1)
       At[r] = SL(V_AT + r);
     }
     const int cb = FUSED ? __ldg(m.o2s + int64_t(e) * NPT + p) : tab_c0[tid];
+    // (zip by the store: the DOF this point is the zip owner of, or -1)
+    const int dz = rhs_dof ? __ldg(m.own + int64_t(e) * NPT + p) : -1;
 #pragma unroll
     for (int i = 0; i < 3; ++i)
       B[i] = !FUSED ? __ldg(pbase + (9 + i) * fstride + cb)
@@ -930,7 +933,12 @@ __global__ void __launch_bounds__(RT, 1)
       }
     double* out = rhs_oct + int64_t(e) * NPT + p;
     const int64_t ostr = no * NPT;
-    if (!SOMM || !bpt) {
+    if (!SOMM && rhs_dof) {
+      if (dz >= 0) {
+#pragma unroll
+        for (int f = 0; f < NF; ++f) rhs_dof[f * int64_t(m.dof_stride) + dz] = r[f];
+      }
+    } else if (!SOMM || !bpt) {
 #pragma unroll
       for (int f = 0; f < NF; ++f) out[f * ostr] = r[f];
     }
@@ -1178,7 +1186,7 @@ void upload_rhs_tables(const double* wext) {
 
 void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const RhsParams& p,
                 bool fused, int64_t first, int64_t count, int leave_sm, cudaStream_t s,
-                double* pre) {
+                double* pre, double* rhs_dof) {
   if (count <= 0) return;
   static int n_sm = 0;
   if (!n_sm) {
@@ -1205,15 +1213,15 @@ void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const 
     const int64_t cap2 = 2 * cap;
     const int grid2 = int(count < cap2 ? count : cap2);
     k_gt_pre<<<grid2, RT, PRE_SMEM_BYTES, s>>>(m, patches, pre, p, a, c);
-    k_rhs<true, false, true><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, pre);
+    k_rhs<true, false, true><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, pre, rhs_dof);
   } else if (fused && !somm)
-    k_rhs<true, false, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr);
+    k_rhs<true, false, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr, rhs_dof);
   else if (fused)
-    k_rhs<true, true, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr);
+    k_rhs<true, true, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr, nullptr);
   else if (!somm)
-    k_rhs<false, false, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr);
+    k_rhs<false, false, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr, nullptr);
   else
-    k_rhs<false, true, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr);
+    k_rhs<false, true, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr, nullptr);
 }
 
 }  // namespace dgr

@@ -137,6 +137,25 @@ def test_metric_prepass_bit_identical(case):
     assert torch.equal(s0, s1), float((s0 - s1).abs().max())
 
 
+def test_zip_store_bit_identical(case):
+    """DGR_OPT_ZIP_STORE: the RHS kernel zipping by its store (each point writes
+    the DOF it is the zip owner of) gives the RHS and the RK4 step bit-identical
+    to the per-point RHS followed by the zip gather."""
+    name, cfg, om, m, u = case
+    dt = ork4.dt_courant(om)
+    out = {}
+    for zs in (False, True):
+        m.set_zip_store(zs)
+        ud = to_dev(u, m.dof_stride)
+        r = m.rhs(ud, out=torch.full_like(ud, np.nan))
+        m.rk4_step(ud, dt)
+        out[zs] = (r[:, :om.n_dof].clone(), ud[:, :om.n_dof].clone())
+    m.set_zip_store(True)
+    assert torch.isfinite(out[True][0]).all(), name   # every owned DOF written
+    assert torch.equal(out[False][0], out[True][0]), name
+    assert torch.equal(out[False][1], out[True][1]), name
+
+
 def test_rk4_step_parity(case):
     name, cfg, om, m, u = case
     dt = ork4.dt_courant(om)

@@ -14,7 +14,7 @@ for r in rows:
     v = v / 1e6 if u == "ns" else (v / 1e3 if u == "us" else v)
     agg[k][0] += 1
     agg[k][1] += v
-STEP = ("k_rhs", "k_gt_pre", "k_interp", "k_zip_rk4", "k_pack")   # kernels of an RK4 stage
+STEP = ("k_rhs", "k_gt_pre", "k_interp", "k_zip_rk4", "k_rk4", "k_pack")   # kernels of an RK4 stage
 step = {k: v for k, v in agg.items() if any(s in k for s in STEP)}
 tot = sum(v[1] for v in step.values())
 print(sys.argv[2] if len(sys.argv) > 2 else "ncu launch list (cold-cache serialised per-launch times)")

@@ -10,7 +10,7 @@ hdr, units = rows[0], rows[1]
 scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
 # (the bench's "rhs" class brackets the whole RHS launch: k_gt_pre + k_rhs)
 names = {"k_gt_pre": "rhs", "k_rhs": "rhs", "k_unzip": "unzip", "k_interp": "interp",
-         "k_zip_rk4": "zip_rk4"}
+         "k_zip_rk4": "zip_rk4", "k_rk4": "zip_rk4"}
 res = json.load(open(outp)) if os.path.exists(outp) else {}
 res[path] = {}
 last = {}

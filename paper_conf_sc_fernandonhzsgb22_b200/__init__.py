@@ -171,6 +171,8 @@ def _ptr(t):
 
 def _stream():
     import torch
+    if not torch.cuda.is_available():   # (host-only meshes: the library refuses device calls)
+        return C.c_void_p(None)
     return C.c_void_p(torch.cuda.current_stream().cuda_stream)
 
 

@@ -141,3 +141,20 @@ def test_host_mesh_rejects_device_calls():
     assert st == -6          # DGR_ERR_STATE: host-only mesh
     st = dgr.lib().dgr_unzip(None, None, None, 24, None)
     assert st == -1          # DGR_ERR_ARG
+
+
+def test_host_only_mesh_refuses_device_calls():
+    """Device entry points (dgr_rk4_step_host included) on a host-only mesh
+    return DGR_ERR_STATE before touching any buffer; a mismatched host-state
+    list is rejected by the binding."""
+    import torch
+    cfg = configs.small_adaptive(lmax=4, rho=0.5)
+    m = dgr.Mesh(cfg, device=False)
+    h = torch.zeros((24, m.dof_stride), dtype=torch.float64)
+    with pytest.raises(dgr.DgrError) as e:
+        m.rk4_step_host([h], [h], 1e-3)
+    assert e.value.status == -6
+    with pytest.raises(ValueError):
+        m.rk4_step_host([h], [], 1e-3)
+    with pytest.raises(ValueError):
+        m.rk4_step_host([h[:, :-1].contiguous()], [h], 1e-3)

@@ -461,30 +461,39 @@ __global__ void __launch_bounds__(RT, 1)
       for (int k = 0; k < 3; ++k) cal[k] = trace6(gi, Gam[k]);
       // Rt_ij without the d Gt terms
       double Rt[6];
+      // gt^lm (Gt^k_li C_j,km + Gt^k_lj C_i,km + Gt^k_im C_k,lj) with the metric
+      // contracted first: Cu[a][b][c] = gt^cm C_a,bm, so each (i,j) needs 27 FMAs
+      // (Gt^k_li Cu[j][k][l] + Gt^k_lj Cu[i][k][l] + Gt^k_im Cu[k][j][m])
 #pragma unroll
       for (int i = 0; i < 3; ++i)
 #pragma unroll
         for (int j = i; j < 3; ++j) {
-          double r = -0.5 * SL(A_AT + sidx(i, j));      // gt^lm d_lm gt_ij
           double c2 = 0.0;
 #pragma unroll
           for (int k = 0; k < 3; ++k) c2 += cal[k] * (C[i][sidx(j, k)] + C[j][sidx(i, k)]);
-          r += 0.5 * c2;
+          Rt[sidx(i, j)] = -0.5 * SL(A_AT + sidx(i, j)) + 0.5 * c2;
+        }
+      double Cu[3][3][3];
+#pragma unroll
+      for (int a = 0; a < 3; ++a)
+#pragma unroll
+        for (int b = 0; b < 3; ++b)
+#pragma unroll
+          for (int c = 0; c < 3; ++c)
+            Cu[a][b][c] = gi[sidx(c, 0)] * C[a][sidx(b, 0)] + gi[sidx(c, 1)] * C[a][sidx(b, 1)] +
+                          gi[sidx(c, 2)] * C[a][sidx(b, 2)];
+#pragma unroll
+      for (int i = 0; i < 3; ++i)
+#pragma unroll
+        for (int j = i; j < 3; ++j) {
           double qsum = 0.0;
 #pragma unroll
-          for (int l = 0; l < 3; ++l)
+          for (int k = 0; k < 3; ++k)
 #pragma unroll
-            for (int mm = 0; mm < 3; ++mm) {
-              const double glm = gi[sidx(l, mm)];
-              double t = 0.0;
-#pragma unroll
-              for (int k = 0; k < 3; ++k)
-                t += Gam[k][sidx(l, i)] * C[j][sidx(k, mm)] +
-                     Gam[k][sidx(l, j)] * C[i][sidx(k, mm)] +
-                     Gam[k][sidx(i, mm)] * C[k][sidx(l, j)];
-              qsum += glm * t;
-            }
-          Rt[sidx(i, j)] = r + qsum;
+            for (int l = 0; l < 3; ++l)
+              qsum += Gam[k][sidx(l, i)] * Cu[j][k][l] + Gam[k][sidx(l, j)] * Cu[i][k][l] +
+                      Gam[k][sidx(i, l)] * Cu[k][j][l];
+          Rt[sidx(i, j)] += qsum;
         }
       // At_ij = chi alpha TF(Rt)   (first write of the A_AT accumulators)
       const double trR = trace6(gi, Rt);

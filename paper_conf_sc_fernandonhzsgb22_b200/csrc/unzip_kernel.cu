@@ -32,7 +32,10 @@ void upload_unzip_tables(const double* w13, const double* wext) {
 namespace {
 constexpr int UZ_WARPS = 8;                 // = fields per CTA
 constexpr int UZ_THREADS = 32 * UZ_WARPS;
-constexpr int IP_FG = 4;                    // fields per k_interp CTA
+#ifndef DGR_IP_FG
+#define DGR_IP_FG 4
+#endif
+constexpr int IP_FG = DGR_IP_FG;            // fields per k_interp CTA
 constexpr int IP_THREADS = 256;
 // sweep scratch per field: a face group's box is at most IP_N1 = 4 points thick
 // along its first sweep axis (host-checked in api.cu), so T1 = 49 x n1 and

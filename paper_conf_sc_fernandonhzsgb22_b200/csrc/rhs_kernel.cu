@@ -230,6 +230,22 @@ __device__ __forceinline__ double trace6(const double* gi, const double* X) {
          2.0 * (gi[1] * X[1] + gi[2] * X[2] + gi[4] * X[4]);
 }
 
+// v^i = At^ij w_j with At^ij = gt^ik gt^jl At_kl, contracted vector-first
+// (w^l = gt^lj w_j, y_k = At_kl w^l, v^i = gt^ik y_k: 27 FMAs)
+__device__ __forceinline__ void at_up_w(const double* gi, const double* At, const double* w,
+                                        double* v) {
+  double wu[3], y[3];
+#pragma unroll
+  for (int l = 0; l < 3; ++l)
+    wu[l] = gi[sidx(l, 0)] * w[0] + gi[sidx(l, 1)] * w[1] + gi[sidx(l, 2)] * w[2];
+#pragma unroll
+  for (int k = 0; k < 3; ++k)
+    y[k] = At[sidx(k, 0)] * wu[0] + At[sidx(k, 1)] * wu[1] + At[sidx(k, 2)] * wu[2];
+#pragma unroll
+  for (int i = 0; i < 3; ++i)
+    v[i] = gi[sidx(i, 0)] * y[0] + gi[sidx(i, 1)] * y[1] + gi[sidx(i, 2)] * y[2];
+}
+
 }  // namespace
 
 // FUSED = false: `patches` is the 13^3 patch buffer [24][n_owned][PATCH_PITCH]
@@ -502,17 +518,21 @@ __global__ void __launch_bounds__(RT, 1)
       for (int r = 0; r < 6; ++r) SL(A_AT + r) = ca * (Rt[r] - gt[r] * trR * (1.0 / 3.0));
       // At^ij = gt^ik gt^jl At_kl ; Gt^i += 2 alpha Gt^i_jk At^jk
       double Au[6];
+      {
+        double M[3][3];   // At_k^j = At_kl gt^lj
 #pragma unroll
-      for (int i = 0; i < 3; ++i)
+        for (int k = 0; k < 3; ++k)
 #pragma unroll
-        for (int j = i; j < 3; ++j) {
-          double a = 0.0;
+          for (int j = 0; j < 3; ++j)
+            M[k][j] = At[sidx(k, 0)] * gi[sidx(0, j)] + At[sidx(k, 1)] * gi[sidx(1, j)] +
+                      At[sidx(k, 2)] * gi[sidx(2, j)];
 #pragma unroll
-          for (int k = 0; k < 3; ++k)
+        for (int i = 0; i < 3; ++i)
 #pragma unroll
-            for (int l = 0; l < 3; ++l) a += gi[sidx(i, k)] * gi[sidx(j, l)] * At[sidx(k, l)];
-          Au[sidx(i, j)] = a;
-        }
+          for (int j = i; j < 3; ++j)
+            Au[sidx(i, j)] = gi[sidx(i, 0)] * M[0][j] + gi[sidx(i, 1)] * M[1][j] +
+                             gi[sidx(i, 2)] * M[2][j];
+      }
 #pragma unroll
       for (int i = 0; i < 3; ++i) SL(A_GT + i) += 2.0 * alpha * trace6(Au, Gam[i]);
       // keep Gt^k_ij and CalGt^k for the chi, alpha and beta stages
@@ -693,19 +713,11 @@ __global__ void __launch_bounds__(RT, 1)
 #pragma unroll
         for (int r = 0; r < 6; ++r) SL(A_AT + r) += ca * (Rc[r] - gt[r] * trR * (1.0 / 3.0));
         // Gt^i += -3 alpha / chi At^ij d_j chi
+        {
+          double v[3];
+          at_up_w(gi, At, dchi, v);
 #pragma unroll
-        for (int i = 0; i < 3; ++i) {
-          double v = 0.0;
-#pragma unroll
-          for (int j = 0; j < 3; ++j) {
-            double a = 0.0;
-#pragma unroll
-            for (int k = 0; k < 3; ++k)
-#pragma unroll
-              for (int l = 0; l < 3; ++l) a += gi[sidx(i, k)] * gi[sidx(j, l)] * At[sidx(k, l)];
-            v += a * dchi[j];
-          }
-          SL(A_GT + i) += -3.0 * alpha * ichi * v;
+          for (int i = 0; i < 3; ++i) SL(A_GT + i) += -3.0 * alpha * ichi * v[i];
         }
       } else if (f == 0) {
         // ---------------- alpha: advection, KO, D_i D_j alpha (eqs 13-15)
@@ -740,19 +752,11 @@ __global__ void __launch_bounds__(RT, 1)
         rK += -chi * trD;
 #pragma unroll
         for (int r = 0; r < 6; ++r) SL(A_AT + r) += -chi * (DD[r] - gt[r] * trD * (1.0 / 3.0));
+        {
+          double v[3];
+          at_up_w(gi, At, da, v);
 #pragma unroll
-        for (int i = 0; i < 3; ++i) {
-          double v = 0.0;
-#pragma unroll
-          for (int j = 0; j < 3; ++j) {
-            double a = 0.0;
-#pragma unroll
-            for (int k = 0; k < 3; ++k)
-#pragma unroll
-              for (int l = 0; l < 3; ++l) a += gi[sidx(i, k)] * gi[sidx(j, l)] * At[sidx(k, l)];
-            v += a * da[j];
-          }
-          SL(A_GT + i) += -2.0 * v;
+          for (int i = 0; i < 3; ++i) SL(A_GT + i) += -2.0 * v[i];
         }
       } else if (f >= 3 && f <= 5) {
         // ---------------- Gt^k: Ricci d Gt term, advection + KO kept apart (eq 3)

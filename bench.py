@@ -40,14 +40,12 @@ INTERP_BYTES_PER_SLOT = 24 * 8                     # write every slot once
 INTERP_BYTES_PER_ELEM = 24 * 343 * 8 + 343 * 4    # read the element's nodal values once (+ o2s)
 RHS_BYTES_PER_OCT = 24 * (2197 + 343) * 8         # patch read + rhs write (eq 21a denominator)
 PAPER_FLOPS_PER_POINT = 5502 + 3998               # eq (21a) numerator per point, O_A from Q_L = 6.68
-# executed fp64 FLOPs per interior point of k_rhs (2 per DFMA + DADD + DMUL), from
-# ncu sm__sass_thread_inst_executed_op_d{fma,add,mul}_pred_on on C3 (profiles/r1c_ncu_flops.csv):
-# fused 2 x 12.991e9 + 11.129e9 + 6.736e9 = 43.85e9 FLOP / 8,329,412 points = 5,265
-# (the in-kernel extrapolation adds ~12 FLOP/pt); two-pass 43.75e9 / 8,329,412 = 5,253
 # executed fp64 FLOPs per interior point (2 DFMA + DADD + DMUL thread instructions from
-# ncu, C3): fused = k_gt_pre + k_rhs (profiles/r1j_flops.csv), two-pass
-# = the single k_rhs (profiles/r1h_ncu_flops_twopass.csv)
-RHS_EXEC_FLOPS_PER_POINT = {"fused": 5358.3, "two-pass": 5265.0}
+# ncu sm__sass_thread_inst_executed_op_d{fma,add,mul}_pred_on, C3, 8,329,412 points):
+# fused = k_gt_pre 8.134e9 + k_rhs 29.526e9 (profiles/r1n_flops.csv), two-pass = the
+# single k_rhs 36.932e9 (profiles/r1n_flops_twopass.csv).  (Round-1 history: 5,358 /
+# 5,265 before the Ricci and At^ij contraction-order changes removed ~840 FLOP/point.)
+RHS_EXEC_FLOPS_PER_POINT = {"fused": 4521.4, "two-pass": 4434.0}
 # DRAM bytes per launch (dram__bytes_read.sum + dram__bytes_write.sum) from one
 # ncu --set full capture of the C3 workload on 1 GPU, per path
 # (profiles/ncu_traffic_c3.json, written by tools/ncu_traffic.py)

@@ -224,6 +224,17 @@ __device__ __forceinline__ Derivs derivs2(const double* __restrict__ s,
   return d;
 }
 
+// stores of results read back only by a later kernel (the pre-pass rows, the
+// DOF-ordered RHS): DGR_STREAM_STORES marks them evict-first so they do not
+// push the gather sources out of L2
+__device__ __forceinline__ void st_out(double* p, double v) {
+#ifdef DGR_STREAM_STORES
+  __stcs(p, v);
+#else
+  *p = v;
+#endif
+}
+
 // trace with the inverse metric: gt^ij X_ij (symmetric storage)
 __device__ __forceinline__ double trace6(const double* gi, const double* X) {
   return gi[0] * X[0] + gi[3] * X[3] + gi[5] * X[5] +
@@ -949,7 +960,7 @@ __global__ void __launch_bounds__(RT, 1)
     if (!SOMM && rhs_dof) {
       if (dz >= 0) {
 #pragma unroll
-        for (int f = 0; f < NF; ++f) rhs_dof[f * int64_t(m.dof_stride) + dz] = r[f];
+        for (int f = 0; f < NF; ++f) st_out(&rhs_dof[f * int64_t(m.dof_stride) + dz], r[f]);
       }
     } else if (!SOMM || !bpt) {
 #pragma unroll
@@ -1155,9 +1166,9 @@ __global__ void __launch_bounds__(RT, 2)
       if (c0 >= 0) {
         const Derivs d = derivs2(s, Tx, Ty, c0, ih, ko_scale);
 #pragma unroll
-        for (int k = 0; k < 3; ++k) out[(6 * k + q) * ostr] = d.d1[k];
-        out[(18 + q) * ostr] = trace6(gi, d.dd);
-        out[(24 + q) * ostr] = beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
+        for (int k = 0; k < 3; ++k) st_out(&out[(6 * k + q) * ostr], d.d1[k]);
+        st_out(&out[(18 + q) * ostr], trace6(gi, d.dd));
+        st_out(&out[(24 + q) * ostr], beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko);
       }
     }
   }

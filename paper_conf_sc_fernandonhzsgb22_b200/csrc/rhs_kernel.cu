@@ -235,6 +235,16 @@ __device__ __forceinline__ void st_out(double* p, double v) {
 #endif
 }
 
+// TF_ONCE (default): the trace-free projection of eq (6)'s chi[..]^TF terms is
+// linear, so it is applied once in the epilogue (sum c X - gt/3 sum c tr X)
+// instead of in each of the six stages that contribute (C3 RHS 7.12 -> 7.03 ms);
+// -DDGR_TF_PER_STAGE restores the per-stage projection (experiment builds)
+#ifdef DGR_TF_PER_STAGE
+constexpr bool TF_ONCE = false;
+#else
+constexpr bool TF_ONCE = true;
+#endif
+
 // trace with the inverse metric: gt^ij X_ij (symmetric storage)
 __device__ __forceinline__ double trace6(const double* gi, const double* X) {
   return gi[0] * X[0] + gi[3] * X[3] + gi[5] * X[5] +
@@ -454,6 +464,7 @@ __global__ void __launch_bounds__(RT, 1)
   const double chi_e = fmax(chi, prm.chi_floor);
   const double ichi = 1.0 / chi_e;
   double rA = 0.0, rC = 0.0, rK = 0.0;   // accumulators of alpha, chi, K
+  double ttr = 0.0;   // (TF_ONCE) sum of c * gt^ij X_ij over the trace-free terms of eq (6)
   double dchi[3] = {0, 0, 0};
 
   // Christoffel block (eqs 12, 17; readings R1, R7): from d_k gt_ij (S0 slots)
@@ -525,8 +536,14 @@ __global__ void __launch_bounds__(RT, 1)
       // At_ij = chi alpha TF(Rt)   (first write of the A_AT accumulators)
       const double trR = trace6(gi, Rt);
       const double ca = chi * alpha;
+      if (TF_ONCE) {
 #pragma unroll
-      for (int r = 0; r < 6; ++r) SL(A_AT + r) = ca * (Rt[r] - gt[r] * trR * (1.0 / 3.0));
+        for (int r = 0; r < 6; ++r) SL(A_AT + r) = ca * Rt[r];
+        ttr += ca * trR;
+      } else {
+#pragma unroll
+        for (int r = 0; r < 6; ++r) SL(A_AT + r) = ca * (Rt[r] - gt[r] * trR * (1.0 / 3.0));
+      }
       // At^ij = gt^ik gt^jl At_kl ; Gt^i += 2 alpha Gt^i_jk At^jk
       double Au[6];
       {
@@ -721,8 +738,14 @@ __global__ void __launch_bounds__(RT, 1)
           }
         const double trR = trace6(gi, Rc);
         const double ca = chi * alpha;
+        if (TF_ONCE) {
 #pragma unroll
-        for (int r = 0; r < 6; ++r) SL(A_AT + r) += ca * (Rc[r] - gt[r] * trR * (1.0 / 3.0));
+          for (int r = 0; r < 6; ++r) SL(A_AT + r) += ca * Rc[r];
+          ttr += ca * trR;
+        } else {
+#pragma unroll
+          for (int r = 0; r < 6; ++r) SL(A_AT + r) += ca * (Rc[r] - gt[r] * trR * (1.0 / 3.0));
+        }
         // Gt^i += -3 alpha / chi At^ij d_j chi
         {
           double v[3];
@@ -761,8 +784,14 @@ __global__ void __launch_bounds__(RT, 1)
           }
         const double trD = trace6(gi, DD);
         rK += -chi * trD;
+        if (TF_ONCE) {
 #pragma unroll
-        for (int r = 0; r < 6; ++r) SL(A_AT + r) += -chi * (DD[r] - gt[r] * trD * (1.0 / 3.0));
+          for (int r = 0; r < 6; ++r) SL(A_AT + r) += -chi * DD[r];
+          ttr += -chi * trD;
+        } else {
+#pragma unroll
+          for (int r = 0; r < 6; ++r) SL(A_AT + r) += -chi * (DD[r] - gt[r] * trD * (1.0 / 3.0));
+        }
         {
           double v[3];
           at_up_w(gi, At, da, v);
@@ -787,8 +816,14 @@ __global__ void __launch_bounds__(RT, 1)
             Rg[sidx(i, j)] = 0.5 * (gt[sidx(kk, i)] * d.d1[j] + gt[sidx(kk, j)] * d.d1[i]);
         const double trR = trace6(gi, Rg);
         const double ca = chi * alpha;
+        if (TF_ONCE) {
 #pragma unroll
-        for (int r = 0; r < 6; ++r) SL(A_AT + r) += ca * (Rg[r] - gt[r] * trR * (1.0 / 3.0));
+          for (int r = 0; r < 6; ++r) SL(A_AT + r) += ca * Rg[r];
+          ttr += ca * trR;
+        } else {
+#pragma unroll
+          for (int r = 0; r < 6; ++r) SL(A_AT + r) += ca * (Rg[r] - gt[r] * trR * (1.0 / 3.0));
+        }
       } else if (f >= 6 && f <= 8) {
         // ---------------- beta^kk: Lie derivative terms, eq (2), eq (8) shift terms
         const int kk = f - 6;
@@ -953,7 +988,8 @@ __global__ void __launch_bounds__(RT, 1)
         r[12 + q] = SL(A_GAM + q) - 2.0 * alpha * At[q];                          // (4)
         const double AAij = At[sidx(i, 0)] * Am[0][j] + At[sidx(i, 1)] * Am[1][j] +
                             At[sidx(i, 2)] * Am[2][j];
-        r[18 + q] = SL(A_AT + q) + alpha * (Kv * At[q] - 2.0 * AAij);             // (6)
+        const double atf = TF_ONCE ? SL(A_AT + q) - SL(V_GAM + q) * ttr * (1.0 / 3.0) : SL(A_AT + q);
+        r[18 + q] = atf + alpha * (Kv * At[q] - 2.0 * AAij);                        // (6)
       }
     double* out = rhs_oct + int64_t(e) * NPT + p;
     const int64_t ostr = no * NPT;

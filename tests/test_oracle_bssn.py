@@ -155,24 +155,25 @@ def test_gauge_sector_textbook_odes():
 
 
 def test_constant_shift_is_advection():
-    """beta = const b adds exactly b.grad(f) to every RHS except beta's own."""
+    """beta -> beta + b (constant b, Galilean boost of the coordinates' shift)
+    adds exactly b.grad(f) to the RHS of EVERY field, beta's own included
+    (eq 2: beta^j d_j beta^i; the transposed beta^j d_i beta^j would add
+    b^j d_i beta^j instead) and B's (eq 3: the b.grad Gt that d_t Gt gains
+    from eq 8 cancels against -beta^j d_j Gt^i, leaving b.grad B)."""
     cfg = MeshConfig(name="u2p", xmin=(0, 0, 0), width=1.0, periodic=True, level_min=2)
     m = OracleMesh(cfg)
     u = initial.random_smooth(m.dof_coords(), 1.0, seed=11)
-    u[6:9] = 0.0
     P0 = unzip(m, u)
     b = np.array([0.3, -0.2, 0.5])
     P1 = P0.copy()
     for i in range(3):
-        P1[6 + i] = b[i]
+        P1[6 + i] = P0[6 + i] + b[i]
     h = rk4.octant_h(m)
     r0 = bssn.rhs_patches(P0, h, PRM)
     r1 = bssn.rhs_patches(P1, h, PRM)
     hh = h[:, None, None, None]
+    assert np.max(np.abs(fd.grad(P0[6], hh))) > 1e-2          # beta really varies
     for f in range(24):
-        if 6 <= f <= 8:
-            assert np.max(np.abs(r1[f] - r0[f])) < 1e-12
-            continue
         g = fd.grad(P0[f], hh)
         want = b[0] * g[0] + b[1] * g[1] + b[2] * g[2]
         assert np.max(np.abs(r1[f] - r0[f] - want)) < 1e-11 * (1 + np.max(np.abs(want))), f
@@ -248,3 +249,110 @@ def test_rk4_temporal_order():
     ref = run(4096)
     e1, e2 = abs(run(16) - ref), abs(run(32) - ref)
     assert 3.7 < np.log2(e1 / e2) < 4.3
+
+
+# ------------------------------------------- shift-wave pins of eqs (2), (3), (8)
+
+def _shift_wave(kvec, evec, eps):
+    """Flat data (gt = delta, alpha = chi = 1, K = At = Gt = B = 0) with the
+    shift plane wave beta^i = eps e^i sin(k.x): every term of eqs (1)-(8) is a
+    closed form in e, k."""
+    ph = sum(sp.Rational(kvec[a]) * V for a, V in enumerate(ex.XYZ))
+    beta = [sp.Rational(eps) * sp.Rational(evec[i]) * sp.sin(ph) for i in range(3)]
+    return ([sp.Integer(1), sp.Integer(1), sp.Integer(0)] + [sp.Integer(0)] * 3 + beta
+            + [sp.Integer(0)] * 3
+            + [sp.Integer(1 if i == j else 0) for (i, j) in ex.SYM] + [sp.Integer(0)] * 6), ph
+
+
+def _closed_form_shift_wave(kvec, evec, eps, pts):
+    k = np.array(kvec, float)
+    e = np.array(evec, float)
+    ph = np.einsum("a,an->n", k, pts)
+    s, c = np.sin(ph), np.cos(ph)
+    beta = eps * e[:, None] * s                       # [i, n]
+    dbeta = eps * np.einsum("i,j->ji", e, k)[..., None] * c   # d_j beta^i -> [j, i, n]
+    div = eps * (e @ k) * c
+    return k, e, s, c, beta, dbeta, div
+
+
+@pytest.mark.parametrize("kvec,evec", [((2, -1, 3), (1, 2, 0)),       # transverse: e.k = 0
+                                       ((0, 3, -2), (5, 0, 0))])
+def test_transverse_shift_wave(kvec, evec):
+    """Transverse shift wave (e perpendicular to k): eq (2) gives
+    d_t beta^i = beta^j d_j beta^i = eps^2 sin cos (e.k) e^i = 0 exactly (the
+    transposed beta^j d_i beta^j would give eps^2 |e|^2 sin cos k^i); eq (8)
+    gives d_t Gt^i = gt^jk d_j d_k beta^i = -|k|^2 beta^i (the divergence term
+    vanishes, CalGt = 0); eq (3) then gives d_t B^i = d_t Gt^i = -|k|^2 beta^i
+    (B = 0, Gt = 0).  P:L101 (eq 2), P:L103 (eq 3), P:L117-119 (eq 8)."""
+    eps = sp.Rational(3, 10)
+    fields, _ = _shift_wave(kvec, evec, eps)
+    pts = _pts(5, -1.0, 1.0, 7)
+    d = ex.pointdata(fields, pts)
+    r = bssn.algebra(d, PRM)
+    k, e, s, c, beta, dbeta, div = _closed_form_shift_wave(kvec, evec, float(eps), pts)
+    assert e @ k == 0
+    k2 = k @ k
+    scale = 1 + k2
+    assert np.max(np.abs(r[6:9])) < 1e-13 * scale                        # eq (2)
+    assert np.max(np.abs(r[3:6] + k2 * beta)) < 1e-12 * scale            # eq (8)
+    assert np.max(np.abs(r[9:12] + k2 * beta)) < 1e-12 * scale           # eq (3)
+    # control: the transposed advection term is not small on these points
+    transposed = np.einsum("jn,ijn->in", beta, dbeta)        # beta^j d_i beta^j
+    assert np.max(np.abs(transposed)) > 1e-3
+    # the rest of the system is closed form too: eq (4) Lie derivative of delta
+    # (w = -2/3, div beta = 0): d_t gt_ij = d_i beta^j + d_j beta^i; eq (5) 0;
+    # eqs (1), (6), (7): 0 (no curvature, alpha' = 0, K = At = 0)
+    want_gt = np.stack([dbeta[j, i] + dbeta[i, j] for (i, j) in ex.SYM])
+    assert np.max(np.abs(r[12:18] - want_gt)) < 1e-13 * scale
+    assert np.max(np.abs(r[[0, 1, 2] + list(range(18, 24))])) < 1e-13 * scale
+
+
+def test_longitudinal_shift_wave():
+    """Longitudinal shift wave (e parallel to k): eq (8) gives
+    d_t Gt^i = -|k|^2 beta^i - (1/3)|k|^2 beta^i = -(4/3)|k|^2 beta^i, eq (3)
+    d_t B^i = the same, eq (2) d_t beta^i = eps^2 |k| sin cos khat^i, eq (5)
+    d_t chi = -(2/3) div beta, eq (4) d_t gt_ij = 2 d_(i beta_j) - (2/3) delta_ij
+    div beta.  P:L99-119."""
+    kvec, evec = (1, 2, -2), (1, 2, -2)
+    eps = sp.Rational(1, 5)
+    fields, _ = _shift_wave(kvec, evec, eps)
+    pts = _pts(5, -1.0, 1.0, 8)
+    d = ex.pointdata(fields, pts)
+    r = bssn.algebra(d, PRM)
+    k, e, s, c, beta, dbeta, div = _closed_form_shift_wave(kvec, evec, float(eps), pts)
+    k2 = k @ k
+    scale = 1 + k2 * k2
+    assert np.max(np.abs(r[3:6] + (4.0 / 3.0) * k2 * beta)) < 1e-12 * scale
+    assert np.max(np.abs(r[9:12] + (4.0 / 3.0) * k2 * beta)) < 1e-12 * scale
+    adv = np.einsum("jn,jin->in", beta, dbeta)                # beta^j d_j beta^i
+    assert np.max(np.abs(r[6:9] - adv)) < 1e-13 * scale
+    assert np.max(np.abs(adv)) > 1e-3
+    assert np.max(np.abs(r[1] + (2.0 / 3.0) * div)) < 1e-13 * scale
+    want_gt = np.stack([dbeta[j, i] + dbeta[i, j] - (2.0 / 3.0) * (i == j) * div
+                        for (i, j) in ex.SYM])
+    assert np.max(np.abs(r[12:18] - want_gt)) < 1e-13 * scale
+
+
+def test_b_equation_couples_to_gt_evolution():
+    """Eq (3) with a nonzero, varying Gt^i and shift: d_t B^i - d_t Gt^i =
+    -eta B^i + beta^j d_j B^i - beta^j d_j Gt^i exactly, whatever the rest of
+    eq (8) is.  Deleting the d_t Gt - beta.grad Gt coupling, or the
+    beta.grad B term, fails."""
+    rng = np.random.default_rng(5)
+    c = [sp.Rational(int(v), 10) for v in rng.integers(-9, 10, size=12)]
+    Gt = [c[0] * sp.sin(X + 2 * Y), c[1] * sp.cos(Z - X), c[2] * X * Y]
+    beta = [c[3] + c[4] * sp.sin(Y), c[5] + c[6] * Z * X, c[7] + c[8] * sp.cos(X + Z)]
+    B = [c[9] * sp.cos(Y + Z), c[10] * X * X, c[11] * sp.sin(Z)]
+    gt = [1 + X * Y / 10, Z / 20, 0, 1 + sp.sin(X) / 10, Y / 30, 1]
+    fields = [1 + X / 10, 1 + Y * Z / 10, X * Z / 5] + Gt + beta + B + gt \
+        + [X / 10, 0, Y / 10, Z / 10, 0, X * Y / 10]
+    fields = [sp.sympify(f) for f in fields]
+    pts = _pts(6, -0.5, 0.5, 9)
+    d = ex.pointdata(fields, pts)
+    prm = bssn.Params(eta=1.3)
+    r = bssn.algebra(d, prm)
+    adv = lambda g: np.einsum("jn,jin->in", d.beta, g)
+    want = -1.3 * d.B + adv(d.d_B) - adv(d.d_Gt)
+    assert np.max(np.abs((r[9:12] - r[3:6]) - want)) < 1e-13
+    assert np.max(np.abs(r[3:6])) > 1e-2          # d_t Gt is not trivially zero here
+    assert np.max(np.abs(adv(d.d_Gt))) > 1e-3

@@ -158,8 +158,12 @@ enum {
   DGR_MAP_RECV_COUNTS = 10, /* int64 [nranks]: ghost DOFs received from each peer  */
   DGR_MAP_LOCAL_OCTS = 11,  /* int32 [n_oct_local + n_oct_ghost]: global octant ids */
   DGR_MAP_O2N_LOCAL = 12,   /* int32 [n_oct_local + n_oct_ghost][343]: local DOF id or -1 */
-  DGR_MAP_RHS_ORDER = 13    /* int32 [n_oct_local]: owned octants (local ids) in RHS order,
+  DGR_MAP_RHS_ORDER = 13,   /* int32 [n_oct_local]: owned octants (local ids) in RHS order,
                                the first n_oct_interior need no ghost value (device meshes) */
+  DGR_MAP_SENDBUF = 14      /* double [sum_p NF * n_p]: the send buffer of the last ghost
+                               exchange, peer-major — for peer p a [NF][n_p] block, row f
+                               holding u[f][DGR_MAP_SEND entries of p] (test hook; device
+                               meshes; synchronises the device) */
 };
 
 const char* dgr_status_string(dgr_status s);
@@ -190,7 +194,14 @@ dgr_status dgr_dof_coords(dgr_mesh m, double* xyz, void* stream);
  * current (see dgr_ghost_exchange). */
 dgr_status dgr_unzip(dgr_mesh m, const double* u, double* patches, int nfields, void* stream);
 
-/* Device: ghost exchange of all 24 fields of u (NCCL, nranks > 1; no-op else). */
+/* Device: ghost exchange of all 24 fields of u (Alg. 1 line 5 halo_exchange,
+ * P:L215; NCCL, nranks > 1; no-op with one rank).  The owned DOFs each peer
+ * needs are packed into a peer-major send buffer (one [24][n_p] block per peer
+ * p, DGR_MAP_SEND order), exchanged as ONE grouped ncclSend/ncclRecv pair per
+ * peer, and unpacked into u's ghost slice (DOFs n_dof_owned.., grouped by
+ * owning rank).  DGR_ERR_STATE on meshes without a communicator
+ * (external-exchange mode: the caller refreshes the ghosts; grouped meshes:
+ * dgr_group_ghost_exchange); NCCL failures give DGR_ERR_NCCL. */
 dgr_status dgr_ghost_exchange(dgr_mesh m, double* u, void* stream);
 
 /* Device: BSSN RHS (eqs 1-8 + KO) at the interior points of given patches
@@ -212,7 +223,11 @@ dgr_status dgr_rhs(dgr_mesh m, double* u, double* rhs, const dgr_params* prm, vo
 dgr_status dgr_rk4_stage(dgr_mesh m, int s, double dt, double* u_n, double* u_s, double* acc,
                          const dgr_params* prm, void* stream);
 
-/* Device: one RK4 step in place on u (library workspace for stages). */
+/* Device: one RK4 step in place on u (library workspace for stages).
+ * nranks > 1 needs a communicator: on an external-exchange or grouped mesh it
+ * returns DGR_ERR_STATE (step those with dgr_rk4_stage + the caller's ghost
+ * refresh, or dgr_group_rk4_step).  dgr_rhs, dgr_rk4_stage and dgr_constraints
+ * do work on external-exchange meshes: they read the ghost DOFs as given. */
 dgr_status dgr_rk4_step(dgr_mesh m, double dt, double* u, const dgr_params* prm, void* stream);
 
 /* Host buffers: one RK4 step (as dgr_rk4_step) of each of n independent
@@ -237,6 +252,25 @@ dgr_status dgr_rk4_step_host(dgr_mesh m, double dt, int64_t n, const double* con
  * over owned DOFs (all ranks).  Synchronises `stream`. */
 dgr_status dgr_constraints(dgr_mesh m, double* u, double* c, double* norms_host,
                            const dgr_params* prm, void* stream);
+
+/* In-process rank group: n meshes of one octree, meshes[r] = rank r of n,
+ * each created with nccl_id = NULL (one per device, or several on one device),
+ * driven by ONE process.  Their ghost exchange is libdgr's own (SURVEY §8e
+ * with the NCCL transport replaced): the same peer-major pack kernel and send
+ * buffers as dgr_ghost_exchange, one cudaMemcpyPeerAsync per (rank, peer)
+ * pair into the peer's receive buffer (NVLink between devices), the same
+ * unpack kernel.  The group borrows the meshes: destroy it before them
+ * (dgr_mesh_destroy of a grouped mesh is DGR_ERR_STATE).  u[r] / streams[r]:
+ * rank r's state and cudaStream_t (arrays of n); streams may coincide. */
+typedef struct dgr_group_s* dgr_group;
+dgr_status dgr_group_create(dgr_mesh* meshes, int n, dgr_group* out);
+/* ghost exchange of every rank's u[r]; complete on streams[r] */
+dgr_status dgr_group_ghost_exchange(dgr_group g, double* const* u, void* const* streams);
+/* one RK4 step in place on every u[r] (as dgr_rk4_step), the exchange of each
+ * stage overlapped with the interior octants of every rank */
+dgr_status dgr_group_rk4_step(dgr_group g, double dt, double* const* u, const dgr_params* prm,
+                              void* const* streams);
+dgr_status dgr_group_destroy(dgr_group g);
 
 /* Execution options of a mesh (host-side switch, takes effect at the next call):
  *   DGR_OPT_FUSED_UNZIP (default 1): 1 = dgr_rhs / dgr_rk4_* gather every patch

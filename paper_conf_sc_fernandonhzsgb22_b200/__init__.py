@@ -26,7 +26,7 @@ NPATCH = 2197
 
 MAP_OCTANTS, MAP_O2N, MAP_HANGING, MAP_PAD_SRC, MAP_PAD_KIND, MAP_ZIP = 0, 1, 2, 3, 4, 5
 MAP_DOF_GID, MAP_DOF_XYZ, MAP_SEND, MAP_SEND_COUNTS, MAP_RECV_COUNTS = 6, 7, 8, 9, 10
-MAP_LOCAL_OCTS, MAP_O2N_LOCAL, MAP_RHS_ORDER = 11, 12, 13
+MAP_LOCAL_OCTS, MAP_O2N_LOCAL, MAP_RHS_ORDER, MAP_SENDBUF = 11, 12, 13, 14
 OPT_FUSED_UNZIP, OPT_PHASES, OPT_PREPASS, OPT_ZIP_STORE = 1, 2, 3, 4
 
 
@@ -80,7 +80,9 @@ EXPORTED = ["dgr_status_string", "dgr_last_error", "dgr_version", "dgr_octree_bu
             "dgr_dof_coords", "dgr_unzip", "dgr_ghost_exchange", "dgr_rhs_patches", "dgr_rhs",
             "dgr_rk4_stage", "dgr_rk4_step", "dgr_rk4_step_host", "dgr_constraints",
             "dgr_last_launch_count",
-            "dgr_profile_enable", "dgr_profile_read", "dgr_bench_dfma", "dgr_set_option"]
+            "dgr_profile_enable", "dgr_profile_read", "dgr_bench_dfma", "dgr_set_option",
+            "dgr_group_create", "dgr_group_ghost_exchange", "dgr_group_rk4_step",
+            "dgr_group_destroy"]
 PROF_CLASSES = ["elements", "hanging", "unzip", "rhs", "zip_rk4", "exchange", "constraints",
                 "interp"]
 
@@ -119,11 +121,16 @@ def lib():
         L.dgr_profile_read.argtypes = [vp, vp, vp, i32]
         L.dgr_bench_dfma.argtypes = [i32, i32, vp, C.POINTER(dp), C.POINTER(dp)]
         L.dgr_set_option.argtypes = [vp, i32, i64]
+        L.dgr_group_create.argtypes = [C.POINTER(vp), i32, C.POINTER(vp)]
+        L.dgr_group_ghost_exchange.argtypes = [vp, C.POINTER(vp), C.POINTER(vp)]
+        L.dgr_group_rk4_step.argtypes = [vp, dp, C.POINTER(vp), C.POINTER(_Params), C.POINTER(vp)]
+        L.dgr_group_destroy.argtypes = [vp]
         for f in ["dgr_octree_build", "dgr_mesh_create", "dgr_mesh_info_get",
                   "dgr_mesh_export_maps", "dgr_mesh_destroy", "dgr_dof_coords", "dgr_unzip",
                   "dgr_ghost_exchange", "dgr_rhs_patches", "dgr_rhs", "dgr_rk4_stage",
                   "dgr_rk4_step", "dgr_rk4_step_host", "dgr_constraints", "dgr_profile_enable", "dgr_profile_read", "dgr_set_option",
-                  "dgr_bench_dfma"]:
+                  "dgr_bench_dfma", "dgr_group_create", "dgr_group_ghost_exchange",
+                  "dgr_group_rk4_step", "dgr_group_destroy"]:
             getattr(L, f).restype = i32
         _lib = L
     return _lib
@@ -167,6 +174,20 @@ def octree_build(cfg) -> np.ndarray:
 
 def _ptr(t):
     return C.c_void_p(t.data_ptr())
+
+
+def _dev(t, shape, what):
+    """Validate a device tensor handed to libdgr (the kernels trust their sizes):
+    CUDA, float64, contiguous, and at least `shape` (leading dims exact)."""
+    import torch
+    if not isinstance(t, torch.Tensor):
+        raise TypeError(f"{what}: expected a torch tensor")
+    if t.device.type != "cuda" or t.dtype != torch.float64 or not t.is_contiguous():
+        raise ValueError(f"{what}: must be a contiguous float64 CUDA tensor "
+                         f"(got {t.dtype} on {t.device}, contiguous={t.is_contiguous()})")
+    if t.dim() != len(shape) or any(a != b for a, b in zip(t.shape, shape)):
+        raise ValueError(f"{what}: shape {tuple(t.shape)}, expected {tuple(shape)}")
+    return _ptr(t)
 
 
 def _stream():
@@ -244,6 +265,9 @@ class Mesh:
         return self.info["n_dof_owned"] + self.info["n_dof_ghost"]
 
     # -------------------------------------------------------- device calls
+    def _state(self, t, what):
+        return _dev(t, (NF, self.dof_stride), what)
+
     def new_state(self, dtype=None):
         import torch
         return torch.zeros((NF, self.dof_stride), dtype=torch.float64, device="cuda")
@@ -251,7 +275,7 @@ class Mesh:
     def dof_coords(self):
         import torch
         xyz = torch.empty((3, self.dof_stride), dtype=torch.float64, device="cuda")
-        _check(lib().dgr_dof_coords(self._h, _ptr(xyz), _stream()))
+        _check(lib().dgr_dof_coords(self._h, _dev(xyz, (3, self.dof_stride), "xyz"), _stream()))
         return xyz
 
     def unzip(self, u, nfields=NF, patches=None):
@@ -259,7 +283,10 @@ class Mesh:
         if patches is None:
             patches = torch.empty((nfields, self.info["n_oct_local"], self.info["patch_pitch"]),
                                   dtype=torch.float64, device="cuda")
-        _check(lib().dgr_unzip(self._h, _ptr(u), _ptr(patches), nfields, _stream()))
+        _check(lib().dgr_unzip(self._h, self._state(u, "u"),
+                               _dev(patches, (nfields, self.info["n_oct_local"],
+                                              self.info["patch_pitch"]), "patches"),
+                               nfields, _stream()))
         return patches
 
     def rhs_patches(self, patches, prm=None, out=None):
@@ -268,28 +295,32 @@ class Mesh:
             out = torch.empty((NF, self.info["n_oct_local"], NPT), dtype=torch.float64,
                               device="cuda")
         p = (prm or Params())._c()
-        _check(lib().dgr_rhs_patches(self._h, _ptr(patches), _ptr(out), C.byref(p), _stream()))
+        no, pp = self.info["n_oct_local"], self.info["patch_pitch"]
+        _check(lib().dgr_rhs_patches(self._h, _dev(patches, (NF, no, pp), "patches"),
+                                     _dev(out, (NF, no, NPT), "out"), C.byref(p), _stream()))
         return out
 
     def ghost_exchange(self, u):
-        _check(lib().dgr_ghost_exchange(self._h, _ptr(u), _stream()))
+        _check(lib().dgr_ghost_exchange(self._h, self._state(u, "u"), _stream()))
 
     def rhs(self, u, prm=None, out=None):
         import torch
         if out is None:
             out = torch.zeros_like(u)
         p = (prm or Params())._c()
-        _check(lib().dgr_rhs(self._h, _ptr(u), _ptr(out), C.byref(p), _stream()))
+        _check(lib().dgr_rhs(self._h, self._state(u, "u"), self._state(out, "out"), C.byref(p),
+                             _stream()))
         return out
 
     def rk4_stage(self, s, dt, u_n, u_s, acc, prm=None):
         p = (prm or Params())._c()
-        _check(lib().dgr_rk4_stage(self._h, s, float(dt), _ptr(u_n), _ptr(u_s), _ptr(acc),
+        _check(lib().dgr_rk4_stage(self._h, s, float(dt), self._state(u_n, "u_n"),
+                                   self._state(u_s, "u_s"), self._state(acc, "acc"),
                                    C.byref(p), _stream()))
 
     def rk4_step(self, u, dt, prm=None):
         p = (prm or Params())._c()
-        _check(lib().dgr_rk4_step(self._h, float(dt), _ptr(u), C.byref(p), _stream()))
+        _check(lib().dgr_rk4_step(self._h, float(dt), self._state(u, "u"), C.byref(p), _stream()))
         return u
 
     def rk4_step_host(self, u_in, u_out, dt, prm=None):
@@ -317,8 +348,9 @@ class Mesh:
             out = torch.zeros((7, self.dof_stride), dtype=torch.float64, device="cuda")
         norms = np.zeros(14)
         p = (prm or Params())._c()
-        _check(lib().dgr_constraints(self._h, _ptr(u), _ptr(out), norms.ctypes.data, C.byref(p),
-                                     _stream()))
+        _check(lib().dgr_constraints(self._h, self._state(u, "u"),
+                                     _dev(out, (7, self.dof_stride), "out"), norms.ctypes.data,
+                                     C.byref(p), _stream()))
         return out, norms.reshape(7, 2)
 
     def last_launch_count(self):
@@ -359,6 +391,49 @@ class Mesh:
         n = np.zeros(8, dtype=np.int64)
         _check(lib().dgr_profile_read(self._h, ms.ctypes.data, n.ctypes.data, int(reset)))
         return {PROF_CLASSES[i]: (float(ms[i]), int(n[i])) for i in range(8) if n[i]}
+
+
+class Group:
+    """dgr_group: rank-meshes [rank 0 .. n-1] of one octree driven by this process
+    (external-exchange meshes, nccl_id=None); libdgr does their ghost exchange
+    (pack kernel, peer copies, unpack kernel).  Destroy (close) before the meshes."""
+
+    def __init__(self, meshes):
+        L = lib()
+        self.meshes = list(meshes)
+        hs = (C.c_void_p * len(self.meshes))(*[m._h.value for m in self.meshes])
+        g = C.c_void_p()
+        _check(L.dgr_group_create(hs, len(self.meshes), C.byref(g)))
+        self._g = g
+
+    def _lists(self, states, streams):
+        n = len(self.meshes)
+        if len(states) != n:
+            raise ValueError("one state per rank")
+        us = (C.c_void_p * n)(*[m._state(u, f"u[{r}]").value
+                                for r, (m, u) in enumerate(zip(self.meshes, states))])
+        if streams is None:
+            streams = [_stream().value] * n
+        ss = (C.c_void_p * n)(*streams)
+        return us, ss
+
+    def ghost_exchange(self, states, streams=None):
+        us, ss = self._lists(states, streams)
+        _check(lib().dgr_group_ghost_exchange(self._g, us, ss))
+
+    def rk4_step(self, states, dt, prm=None, streams=None):
+        us, ss = self._lists(states, streams)
+        p = (prm or Params())._c()
+        _check(lib().dgr_group_rk4_step(self._g, float(dt), us, C.byref(p), ss))
+        return states
+
+    def close(self):
+        g = getattr(self, "_g", None)
+        if g is not None and g.value and _lib is not None:
+            _lib.dgr_group_destroy(g)
+            self._g = None
+
+    __del__ = close
 
 
 def bench_dfma(blocks=148 * 8, iters=200000):

@@ -82,6 +82,7 @@ constexpr int NCCL_FLOAT64 = 8, NCCL_SUM = 0, NCCL_MAX = 2;
 }  // namespace
 
 // ----------------------------------------------------------------- mesh
+struct dgr_group_s;
 struct dgr_mesh_s {
   HostMesh host;
   bool device = false;
@@ -132,11 +133,14 @@ struct dgr_mesh_s {
   double* d_hbuf[3] = {nullptr, nullptr, nullptr};
   cudaStream_t h2d = nullptr, d2h = nullptr;
   cudaEvent_t ev_in[3] = {}, ev_done[3] = {}, ev_out[3] = {}, ev_host0 = nullptr;
-  // multi-rank
+  // multi-rank: peer-major send / receive buffers (one [NF][n_p] block per
+  // peer p), per-peer prefix offsets, NCCL communicator or in-process group
   void* comm = nullptr;
+  dgr_group_s* group = nullptr;     // linked in-process ranks (dgr_group_create)
   int32_t* d_send = nullptr;
   double* d_sendbuf = nullptr;
   double* d_recvbuf = nullptr;
+  PeerOffsets po_send{}, po_recv{};
   int64_t launches = 0;
   bool fused = true;            // DGR_OPT_FUSED_UNZIP (C3: 40.4 ms/step fused, 41.2 two-pass)
   // profiling
@@ -605,6 +609,14 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
                           cudaMemcpyHostToDevice));
     CUDA_TRY(m->alloc(&m->d_sendbuf, size_t(NF) * h.send_list.size()));
     CUDA_TRY(m->alloc(&m->d_recvbuf, size_t(NF) * h.n_ghost_dof));
+    m->po_send.np = m->po_recv.np = h.nranks;
+    m->po_send.off[0] = m->po_recv.off[0] = 0;
+    for (int p = 0; p < h.nranks; ++p) {
+      m->po_send.off[p + 1] = m->po_send.off[p] + h.send_counts[p];
+      m->po_recv.off[p + 1] = m->po_recv.off[p] + h.recv_counts[p];
+    }
+    if (m->po_recv.off[h.nranks] != h.n_ghost_dof || m->po_send.off[h.nranks] != int64_t(h.send_list.size()))
+      return fail(DGR_ERR_TREE, "send/receive counts inconsistent with the ghost layer");
   }
   CUDA_TRY(m->alloc(&m->d_cnorm, 16 + size_t(7) * 2 * CN_BLOCKS));   // [16] result + partials
   CUDA_TRY(cudaStreamSynchronize(st));
@@ -615,6 +627,8 @@ dgr_status dgr_mesh_create(const dgr_mesh_desc* desc, const dgr_octant* octs, in
                            void* stream, dgr_mesh* out) {
   if (!desc || !octs || !out || n <= 0) return fail(DGR_ERR_ARG, "null argument or n <= 0");
   *out = nullptr;
+  if (desc->nranks < 1 || desc->nranks > MAX_RANKS || desc->rank < 0 || desc->rank >= desc->nranks)
+    return fail(DGR_ERR_ARG, "rank / nranks out of range (1 <= nranks <= 64)");
   std::unique_ptr<dgr_mesh_s> m;
   try {
     m.reset(new dgr_mesh_s());
@@ -745,6 +759,17 @@ dgr_status dgr_mesh_export_maps(dgr_mesh m, int which, void* host_buf, size_t* n
       return put(h.local_oct.data(), h.local_oct.size() * 4);
     case DGR_MAP_O2N_LOCAL:
       return put(h.o2n_local.data(), h.o2n_local.size() * 4);
+    case DGR_MAP_SENDBUF: {   // test hook: the last packed (peer-major) send buffer
+      if (!m->device) return fail(DGR_ERR_STATE, "send buffer exists on device meshes only");
+      const size_t nd = size_t(NF) * h.send_list.size();
+      std::vector<double> v(nd);
+      if (nd) {
+        cudaError_t e = cudaDeviceSynchronize();
+        if (e == cudaSuccess) e = cudaMemcpy(v.data(), m->d_sendbuf, nd * 8, cudaMemcpyDeviceToHost);
+        if (e != cudaSuccess) return fail(DGR_ERR_CUDA, cudaGetErrorString(e));
+      }
+      return put(v.data(), v.size() * 8);
+    }
     case DGR_MAP_RHS_ORDER: {
       if (!m->device) return fail(DGR_ERR_STATE, "RHS order exists on device meshes only");
       std::vector<int32_t> v(static_cast<size_t>(no));
@@ -759,6 +784,7 @@ dgr_status dgr_mesh_export_maps(dgr_mesh m, int which, void* host_buf, size_t* n
 }
 
 dgr_status dgr_mesh_destroy(dgr_mesh m) {
+  if (m && m->group) return fail(DGR_ERR_STATE, "mesh is in a group: dgr_group_destroy first");
   delete m;
   return DGR_OK;
 }
@@ -793,28 +819,35 @@ static bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 
     }                                                            \
   } while (0)
 
-// ghost exchange: pack owned DOFs each peer needs, grouped send/recv, unpack
+#define NCCL_TRY(x)                                                                   \
+  do {                                                                                \
+    int _r = (x);                                                                     \
+    if (_r != 0) return fail(DGR_ERR_NCCL, std::string(#x) + " failed: ncclResult " + std::to_string(_r)); \
+  } while (0)
+
+// Ghost exchange over NCCL (Alg. 1 line 5 halo_exchange): pack the
+// owned DOFs each peer needs into the peer-major send buffer, one grouped
+// ncclSend / ncclRecv per peer (a single [NF][n_p] message each way), unpack
+// the peer-major receive buffer into u's ghost slice.  All on stream `st`.
 static dgr_status exchange(dgr_mesh m, double* u, cudaStream_t st) {
   const HostMesh& h = m->host;
-  if (h.nranks <= 1 || !m->comm) return DGR_OK;   // single rank / external exchange
+  // single rank; or no communicator: external-exchange / grouped meshes, whose
+  // ghosts the caller (DGR_MAP_SEND) or the group driver (dgr_group_*) refreshes
+  if (h.nranks <= 1 || !m->comm) return DGR_OK;
   const int64_t stride = m->dm.dof_stride;
-  const int64_t nsend = int64_t(h.send_list.size());
-  PROF(m, 5, st, launch_gather_pack(u, stride, m->d_send, nsend, m->d_sendbuf, st));
+  PROF(m, 5, st, launch_gather_pack(u, stride, m->d_send, m->po_send, m->d_sendbuf, st));
   CUDA_TRY(cudaGetLastError());
-  // sendbuf is [f][nsend] with peers contiguous inside each field row; send
-  // one message per (peer, field) row segment inside a single group
-  if (g_nccl.GroupStart() != 0) return fail(DGR_ERR_NCCL, "ncclGroupStart");
-  int64_t soff = 0, roff = 0;
+  NCCL_TRY(g_nccl.GroupStart());
   for (int peer = 0; peer < h.nranks; ++peer) {
     const int64_t ns = h.send_counts[peer], nr = h.recv_counts[peer];
-    for (int f = 0; f < NF; ++f) {
-      if (ns) g_nccl.Send(m->d_sendbuf + f * nsend + soff, size_t(ns), NCCL_FLOAT64, peer, m->comm, st);
-      if (nr) g_nccl.Recv(u + f * stride + h.n_owned_dof + roff, size_t(nr), NCCL_FLOAT64, peer, m->comm, st);
-    }
-    soff += ns;
-    roff += nr;
+    if (ns) NCCL_TRY(g_nccl.Send(m->d_sendbuf + NF * m->po_send.off[peer], size_t(NF * ns),
+                                 NCCL_FLOAT64, peer, m->comm, st));
+    if (nr) NCCL_TRY(g_nccl.Recv(m->d_recvbuf + NF * m->po_recv.off[peer], size_t(NF * nr),
+                                 NCCL_FLOAT64, peer, m->comm, st));
   }
-  if (g_nccl.GroupEnd() != 0) return fail(DGR_ERR_NCCL, "ncclGroupEnd");
+  NCCL_TRY(g_nccl.GroupEnd());
+  PROF(m, 5, st, launch_scatter_unpack(u, stride, h.n_owned_dof, m->d_recvbuf, m->po_recv, st));
+  CUDA_TRY(cudaGetLastError());
   return DGR_OK;
 }
 
@@ -832,15 +865,17 @@ static dgr_status do_interp(dgr_mesh m, const double* u, int nf, cudaStream_t st
   return DGR_OK;
 }
 
-// explicit unzip into the patch buffer (two-pass path, dgr_unzip, constraints)
-static dgr_status do_unzip(dgr_mesh m, const double* u, int nf, cudaStream_t st) {
-  if (!m->d_patch) {
+// explicit unzip into the patch buffer (two-pass path, constraints) or straight
+// into the caller's buffer (dgr_unzip: same [nf][n_owned][PATCH_PITCH] layout)
+static dgr_status do_unzip(dgr_mesh m, const double* u, int nf, cudaStream_t st,
+                           double* out = nullptr) {
+  if (!out && !m->d_patch) {
     CUDA_TRY(m->alloc(&m->d_patch, size_t(NF) * m->dm.n_owned * PATCH_PITCH));
     CUDA_TRY(cudaMemsetAsync(m->d_patch, 0, size_t(NF) * m->dm.n_owned * PATCH_PITCH * 8, st));
   }
   dgr_status s = do_interp(m, u, nf, st);
   if (s) return s;
-  PROF(m, 2, st, launch_unzip(m->dm, u, m->d_patch, nf, st));
+  PROF(m, 2, st, launch_unzip(m->dm, u, out ? out : m->d_patch, nf, st));
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;
 }
@@ -864,9 +899,22 @@ static bool zip_by_store(dgr_mesh m, const dgr_params* prm) {
   return m->fused && m->zip_store && !(prm && prm->sommerfeld && !m->host.periodic);
 }
 
+static dgr_status ensure_xstream(dgr_mesh m) {
+  if (!m->xstream) {
+    CUDA_TRY(cudaStreamCreateWithFlags(&m->xstream, cudaStreamNonBlocking));
+    CUDA_TRY(cudaEventCreateWithFlags(&m->ev_ready, cudaEventDisableTiming));
+    CUDA_TRY(cudaEventCreateWithFlags(&m->ev_xdone, cudaEventDisableTiming));
+  }
+  return DGR_OK;
+}
+
 // (rhs_dof != nullptr: fused path only, k_rhs zips by its store into rhs_dof)
+// preissued: the ghost exchange of u was already enqueued on m->xstream by the
+// group driver (dgr_group_*) and completes at m->ev_xdone; otherwise it is done
+// here (NCCL) — on the caller's stream, or on m->xstream overlapped with the
+// interior octants.
 static dgr_status rhs_oct(dgr_mesh m, double* u, const dgr_params* prm, cudaStream_t st,
-                          double* rhs_dof = nullptr) {
+                          double* rhs_dof = nullptr, bool preissued = false) {
   dgr_status s;
   const int64_t no = m->dm.n_owned, ni = m->n_interior;
   const RhsParams rp = to_rp(prm);
@@ -875,45 +923,52 @@ static dgr_status rhs_oct(dgr_mesh m, double* u, const dgr_params* prm, cudaStre
     if (!m->d_pre) CUDA_TRY(m->alloc(&m->d_pre, size_t(30) * no * 352));
     pre = m->d_pre;
   }
+  // ghosts current on `st` (no overlap)
+  auto ghosts_now = [&]() -> dgr_status {
+    if (preissued) {
+      CUDA_TRY(cudaStreamWaitEvent(st, m->ev_xdone, 0));
+      return DGR_OK;
+    }
+    return exchange(m, u, st);
+  };
   if (!m->fused) {
-    if ((s = exchange(m, u, st))) return s;
+    if ((s = ghosts_now())) return s;
     if ((s = do_unzip(m, u, NF, st))) return s;
     PROF(m, 3, st, launch_rhs(m->dm, m->d_patch, m->d_rhs_oct, rp, false, 0, no, 0, st));
     CUDA_TRY(cudaGetLastError());
     return DGR_OK;
   }
-  const bool overlap = m->host.nranks > 1 && m->comm && ni > 0 && ni < no && m->phases == 0;
+  const bool multi = m->host.nranks > 1 && (m->comm || preissued);
+  const bool overlap = multi && ni > 0 && ni < no && m->phases == 0;
   if (m->phases > 0) {
     // interior octants and the slots they need first, then (unless the test
     // hook stops here) the rest — no stream overlap
-    if ((s = exchange(m, u, st))) return s;
+    if ((s = ghosts_now())) return s;
     if ((s = do_interp(m, u, NF, st, 0))) return s;
     PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, ni, 0, st, pre, rhs_dof));
     if (pre) ++m->launches;   // (k_gt_pre + k_rhs)
     if (m->phases == 1) {
       if ((s = do_interp(m, u, NF, st, 1))) return s;
       PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, ni, no - ni, 0, st, pre, rhs_dof));
-    if (pre) ++m->launches;   // (k_gt_pre + k_rhs)
+      if (pre) ++m->launches;
     }
   } else if (overlap) {
-    if (!m->xstream) {
-      CUDA_TRY(cudaStreamCreateWithFlags(&m->xstream, cudaStreamNonBlocking));
-      CUDA_TRY(cudaEventCreateWithFlags(&m->ev_ready, cudaEventDisableTiming));
-      CUDA_TRY(cudaEventCreateWithFlags(&m->ev_xdone, cudaEventDisableTiming));
+    if (!preissued) {
+      if ((s = ensure_xstream(m))) return s;
+      CUDA_TRY(cudaEventRecord(m->ev_ready, st));
+      CUDA_TRY(cudaStreamWaitEvent(m->xstream, m->ev_ready, 0));
+      if ((s = exchange(m, u, m->xstream))) return s;
+      CUDA_TRY(cudaEventRecord(m->ev_xdone, m->xstream));
     }
-    CUDA_TRY(cudaEventRecord(m->ev_ready, st));
-    CUDA_TRY(cudaStreamWaitEvent(m->xstream, m->ev_ready, 0));
-    if ((s = exchange(m, u, m->xstream))) return s;
-    CUDA_TRY(cudaEventRecord(m->ev_xdone, m->xstream));
     if ((s = do_interp(m, u, NF, st, 0))) return s;
     PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, ni, m->xsm, st, pre, rhs_dof));
     if (pre) ++m->launches;   // (k_gt_pre + k_rhs)
     CUDA_TRY(cudaStreamWaitEvent(st, m->ev_xdone, 0));
     if ((s = do_interp(m, u, NF, st, 1))) return s;
     PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, ni, no - ni, 0, st, pre, rhs_dof));
-    if (pre) ++m->launches;   // (k_gt_pre + k_rhs)
+    if (pre) ++m->launches;
   } else {
-    if ((s = exchange(m, u, st))) return s;
+    if ((s = ghosts_now())) return s;
     if ((s = do_interp(m, u, NF, st))) return s;
     PROF(m, 3, st, launch_rhs(m->dm, u, m->d_rhs_oct, rp, true, 0, no, 0, st, pre, rhs_dof));
     if (pre) ++m->launches;   // (k_gt_pre + k_rhs)
@@ -947,12 +1002,8 @@ dgr_status dgr_unzip(dgr_mesh m, const double* u, double* patches, int nfields, 
   if (!u || !patches || nfields < 1 || nfields > NF) return fail(DGR_ERR_ARG, "bad unzip args");
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   m->launches = 0;
-  s = do_unzip(m, u, nfields, st);
-  if (s) return s;
-  const size_t bytes = size_t(nfields) * m->dm.n_owned * PATCH_PITCH * 8;
-  if (patches != m->d_patch)
-    CUDA_TRY(cudaMemcpyAsync(patches, m->d_patch, bytes, cudaMemcpyDeviceToDevice, st));
-  return DGR_OK;
+  if (!aligned16(patches)) return fail(DGR_ERR_ARG, "patches must be 16-byte aligned");
+  return do_unzip(m, u, nfields, st, patches);
 }
 
 dgr_status dgr_rhs_patches(dgr_mesh m, const double* patches, double* rhs_oct,
@@ -980,7 +1031,8 @@ dgr_status dgr_rhs(dgr_mesh m, double* u, double* rhs, const dgr_params* prm, vo
 }
 
 static dgr_status stage(dgr_mesh m, int s_, double dt, double* u_n, double* u_s, double* acc,
-                        double* u_out, const dgr_params* prm, cudaStream_t st) {
+                        double* u_out, const dgr_params* prm, cudaStream_t st,
+                        bool preissued = false) {
   dgr_status s;
   double* cur = s_ == 0 ? u_n : u_s;
   // (applying the zip + RK4 update inside k_rhs measured 10.6 ms vs 7.5 + 0.8 ms
@@ -989,12 +1041,12 @@ static dgr_status stage(dgr_mesh m, int s_, double dt, double* u_n, double* u_s,
   // is only stores, so k_rhs does it by default: DGR_OPT_ZIP_STORE)
   if (zip_by_store(m, prm)) {
     if (!m->d_rhs_dof) CUDA_TRY(m->alloc(&m->d_rhs_dof, size_t(NF) * m->dm.dof_stride));
-    if ((s = rhs_oct(m, cur, prm, st, m->d_rhs_dof))) return s;
+    if ((s = rhs_oct(m, cur, prm, st, m->d_rhs_dof, preissued))) return s;
     PROF(m, 4, st, launch_rk4(m->dm, m->d_rhs_dof, s_, dt, u_n, u_s, acc, u_out, st));
     CUDA_TRY(cudaGetLastError());
     return DGR_OK;
   }
-  if ((s = rhs_oct(m, cur, prm, st))) return s;
+  if ((s = rhs_oct(m, cur, prm, st, nullptr, preissued))) return s;
   PROF(m, 4, st, launch_zip_rk4(m->dm, m->d_rhs_oct, s_, dt, u_n, u_s, acc, u_out, st));
   CUDA_TRY(cudaGetLastError());
   return DGR_OK;
@@ -1013,6 +1065,9 @@ dgr_status dgr_rk4_step(dgr_mesh m, double dt, double* u, const dgr_params* prm,
   dgr_status s = need_device(m);
   if (s) return s;
   if (!u) return fail(DGR_ERR_ARG, "null state");
+  if (m->host.nranks > 1 && !m->comm)
+    return fail(DGR_ERR_STATE, "dgr_rk4_step needs a communicator: external-exchange meshes step "
+                               "with dgr_rk4_stage, grouped meshes with dgr_group_rk4_step");
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   m->launches = 0;
   for (int k = 0; k < 4; ++k)
@@ -1031,6 +1086,9 @@ dgr_status dgr_rk4_step_host(dgr_mesh m, double dt, int64_t n, const double* con
   if (n < 0 || (n > 0 && (!u_in || !u_out))) return fail(DGR_ERR_ARG, "bad host state lists");
   for (int64_t j = 0; j < n; ++j)
     if (!u_in[j] || !u_out[j]) return fail(DGR_ERR_ARG, "null host state");
+  if (m->host.nranks > 1 && !m->comm)
+    return fail(DGR_ERR_STATE, "dgr_rk4_step_host needs a communicator (the stages refresh the "
+                               "ghost DOFs by NCCL)");
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   m->launches = 0;
   if (n == 0) return DGR_OK;
@@ -1113,8 +1171,8 @@ dgr_status dgr_constraints(dgr_mesh m, double* u, double* c, double* norms_host,
       sums[7] = ntot;
       CUDA_TRY(cudaMemcpyAsync(d, sums, 64, cudaMemcpyHostToDevice, st));
       CUDA_TRY(cudaMemcpyAsync(d + 8, maxs, 56, cudaMemcpyHostToDevice, st));
-      g_nccl.AllReduce(d, d, 8, NCCL_FLOAT64, NCCL_SUM, m->comm, st);
-      g_nccl.AllReduce(d + 8, d + 8, 7, NCCL_FLOAT64, NCCL_MAX, m->comm, st);
+      NCCL_TRY(g_nccl.AllReduce(d, d, 8, NCCL_FLOAT64, NCCL_SUM, m->comm, st));
+      NCCL_TRY(g_nccl.AllReduce(d + 8, d + 8, 7, NCCL_FLOAT64, NCCL_MAX, m->comm, st));
       CUDA_TRY(cudaMemcpyAsync(sums, d, 64, cudaMemcpyDeviceToHost, st));
       CUDA_TRY(cudaMemcpyAsync(maxs, d + 8, 56, cudaMemcpyDeviceToHost, st));
       CUDA_TRY(cudaStreamSynchronize(st));
@@ -1195,6 +1253,157 @@ dgr_status dgr_bench_dfma(int blocks, int iters, void* stream, double* ms, doubl
   cudaFree(out);
   *ms = double(t);
   *flops = double(blocks) * 256.0 * 8.0 * double(iters) * 2.0;
+  return DGR_OK;
+}
+
+}  // extern "C"
+
+// ------------------------------------------------------- in-process rank group
+// R rank-meshes of one octree driven by one process (one per device, or several
+// on one device).  The exchange is libdgr's own: k_pack into each rank's
+// peer-major send buffer, one peer copy per (rank, peer) pair into the peer's
+// receive buffer (cudaMemcpyPeerAsync: NVLink between devices, a device copy
+// on one device), k_unpack into the ghost slice — the same buffers, offsets and
+// kernels as the NCCL path, with the transport replaced.
+struct dgr_group_s {
+  std::vector<dgr_mesh> m;
+  std::vector<cudaEvent_t> ev_packed;   // per rank: its send buffer is packed
+  ~dgr_group_s() {
+    for (auto e : ev_packed) if (e) cudaEventDestroy(e);
+    for (dgr_mesh x : m) if (x && x->group == this) x->group = nullptr;
+  }
+};
+
+namespace {
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int d) { cudaGetDevice(&prev); if (d >= 0 && d != prev) cudaSetDevice(d); }
+  ~DeviceGuard() { if (prev >= 0) cudaSetDevice(prev); }
+};
+}  // namespace
+
+// enqueue the exchange of every rank's state u[r]; rank r's ghosts are current
+// at m[r]->ev_xdone (recorded on m[r]->xstream).  Work starts after what is
+// already enqueued on streams[r].
+static dgr_status group_exchange(dgr_group_s* g, double* const* u, void* const* streams) {
+  const int R = int(g->m.size());
+  for (int r = 0; r < R; ++r) {
+    dgr_mesh m = g->m[r];
+    DeviceGuard dg(m->dev_id);
+    cudaStream_t st = static_cast<cudaStream_t>(streams[r]);
+    dgr_status s = ensure_xstream(m);
+    if (s) return s;
+    CUDA_TRY(cudaEventRecord(m->ev_ready, st));
+    CUDA_TRY(cudaStreamWaitEvent(m->xstream, m->ev_ready, 0));
+    // the previous exchange's peer copies out of this send buffer are done
+    for (int p = 0; p < R; ++p)
+      if (p != r && m->host.send_counts[p]) CUDA_TRY(cudaStreamWaitEvent(m->xstream, g->m[p]->ev_xdone, 0));
+    PROF(m, 5, m->xstream, launch_gather_pack(u[r], m->dm.dof_stride, m->d_send, m->po_send,
+                                              m->d_sendbuf, m->xstream));
+    CUDA_TRY(cudaGetLastError());
+    CUDA_TRY(cudaEventRecord(g->ev_packed[r], m->xstream));
+  }
+  for (int p = 0; p < R; ++p) {
+    dgr_mesh mp = g->m[p];
+    DeviceGuard dg(mp->dev_id);
+    for (int r = 0; r < R; ++r) {
+      const int64_t n = mp->host.recv_counts[r];
+      if (r == p || !n) continue;
+      dgr_mesh mr = g->m[r];
+      CUDA_TRY(cudaStreamWaitEvent(mp->xstream, g->ev_packed[r], 0));
+      CUDA_TRY(cudaMemcpyPeerAsync(mp->d_recvbuf + NF * mp->po_recv.off[r], mp->dev_id,
+                                   mr->d_sendbuf + NF * mr->po_send.off[p], mr->dev_id,
+                                   size_t(NF) * n * sizeof(double), mp->xstream));
+    }
+    PROF(mp, 5, mp->xstream, launch_scatter_unpack(u[p], mp->dm.dof_stride, mp->host.n_owned_dof,
+                                                   mp->d_recvbuf, mp->po_recv, mp->xstream));
+    CUDA_TRY(cudaGetLastError());
+    CUDA_TRY(cudaEventRecord(mp->ev_xdone, mp->xstream));
+  }
+  return DGR_OK;
+}
+
+static dgr_status group_check(dgr_group g, const void* const* a, const void* const* b) {
+  if (!g || !a || !b) return fail(DGR_ERR_ARG, "null group argument");
+  for (size_t r = 0; r < g->m.size(); ++r)
+    if (!a[r] || !b[r]) return fail(DGR_ERR_ARG, "null state or stream entry");
+  return DGR_OK;
+}
+
+extern "C" {
+
+dgr_status dgr_group_create(dgr_mesh* meshes, int n, dgr_group* out) {
+  if (!meshes || !out || n < 1) return fail(DGR_ERR_ARG, "null argument or n < 1");
+  *out = nullptr;
+  for (int r = 0; r < n; ++r) {
+    dgr_mesh m = meshes[r];
+    if (!m || !m->device) return fail(DGR_ERR_ARG, "null or host-only mesh in the group");
+    if (m->host.nranks != n || m->host.rank != r)
+      return fail(DGR_ERR_ARG, "meshes[r] must be rank r of n ranks");
+    if (m->comm || m->group) return fail(DGR_ERR_STATE, "mesh already has a communicator or group");
+    if (m->host.oct.size() != meshes[0]->host.oct.size())
+      return fail(DGR_ERR_ARG, "meshes of different octrees");
+  }
+  for (int p = 0; p < n; ++p)
+    for (int r = 0; r < n; ++r)
+      if (p != r && meshes[p]->host.recv_counts[r] != meshes[r]->host.send_counts[p])
+        return fail(DGR_ERR_TREE, "send/receive counts of a rank pair disagree");
+  std::unique_ptr<dgr_group_s> g(new dgr_group_s());
+  g->m.assign(meshes, meshes + n);
+  g->ev_packed.assign(size_t(n), nullptr);
+  for (int r = 0; r < n; ++r) {
+    DeviceGuard dg(meshes[r]->dev_id);
+    CUDA_TRY(cudaEventCreateWithFlags(&g->ev_packed[r], cudaEventDisableTiming));
+    for (int p = 0; p < n; ++p)
+      if (p != r && meshes[r]->dev_id != meshes[p]->dev_id) {
+        int ok = 0;
+        CUDA_TRY(cudaDeviceCanAccessPeer(&ok, meshes[r]->dev_id, meshes[p]->dev_id));
+        if (ok) {
+          cudaError_t e = cudaDeviceEnablePeerAccess(meshes[p]->dev_id, 0);
+          if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
+          else CUDA_TRY(e);
+        }
+      }
+  }
+  for (int r = 0; r < n; ++r) meshes[r]->group = g.get();
+  *out = g.release();
+  return DGR_OK;
+}
+
+dgr_status dgr_group_ghost_exchange(dgr_group g, double* const* u, void* const* streams) {
+  dgr_status s = group_check(g, reinterpret_cast<const void* const*>(u), streams);
+  if (s) return s;
+  if ((s = group_exchange(g, u, streams))) return s;
+  for (size_t r = 0; r < g->m.size(); ++r) {
+    DeviceGuard dg(g->m[r]->dev_id);
+    CUDA_TRY(cudaStreamWaitEvent(static_cast<cudaStream_t>(streams[r]), g->m[r]->ev_xdone, 0));
+  }
+  return DGR_OK;
+}
+
+dgr_status dgr_group_rk4_step(dgr_group g, double dt, double* const* u, const dgr_params* prm,
+                              void* const* streams) {
+  dgr_status s = group_check(g, reinterpret_cast<const void* const*>(u), streams);
+  if (s) return s;
+  const int R = int(g->m.size());
+  for (dgr_mesh m : g->m) m->launches = 0;
+  for (int k = 0; k < 4; ++k) {
+    std::vector<double*> cur(R);
+    for (int r = 0; r < R; ++r) cur[r] = k == 0 ? u[r] : g->m[r]->d_us;
+    if ((s = group_exchange(g, cur.data(), streams))) return s;
+    for (int r = 0; r < R; ++r) {
+      dgr_mesh m = g->m[r];
+      DeviceGuard dg(m->dev_id);
+      if ((s = stage(m, k, dt, u[r], m->d_us, m->d_acc, u[r], prm,
+                     static_cast<cudaStream_t>(streams[r]), true)))
+        return s;
+    }
+  }
+  return DGR_OK;
+}
+
+dgr_status dgr_group_destroy(dgr_group g) {
+  delete g;
   return DGR_OK;
 }
 

@@ -80,10 +80,18 @@ void launch_rk4(const DevMesh& m, const double* rhs, int stage, double dt, const
                 double* u_s, double* acc, double* u_out, cudaStream_t s);
 void launch_dof_coords(const DevMesh& m, const int64_t* dof_node, double* xyz,
                        const double xmin[3], cudaStream_t s);
-void launch_gather_pack(const double* u, int64_t stride, const int32_t* list, int64_t n,
+// per-peer prefix offsets of a peer-major message buffer (passed by value)
+constexpr int MAX_RANKS = 64;
+struct PeerOffsets {
+  int np;                       // number of peers (= nranks)
+  int64_t off[MAX_RANKS + 1];   // off[p] = entries before peer p's block
+};
+// buf (peer-major, one [NF][n_p] block per peer p) <- u[f][list[i]]
+void launch_gather_pack(const double* u, int64_t stride, const int32_t* list, const PeerOffsets& po,
                         double* buf, cudaStream_t s);
-void launch_scatter_unpack(double* u, int64_t stride, int64_t offset, const double* buf,
-                           int64_t n_total, cudaStream_t s);
+// u[f][n_owned + i] <- peer-major receive buffer
+void launch_scatter_unpack(double* u, int64_t stride, int64_t n_owned, const double* buf,
+                           const PeerOffsets& po, cudaStream_t s);
 
 void launch_dfma(int blocks, int iters, double* out, cudaStream_t s);
 

@@ -197,37 +197,58 @@ void launch_dof_coords(const DevMesh& m, const int64_t* dof_node, double* xyz,
 }
 
 // ------------------------------------------------------- ghost pack/unpack
-__global__ void k_pack(const double* __restrict__ u, int64_t stride,
-                       const int32_t* __restrict__ list, int64_t n, double* __restrict__ buf) {
-  // buf layout [f][n] per peer block is produced by the caller's offsets
-  const int f = blockIdx.y;
-  for (int64_t i = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; i < n;
-       i += int64_t(gridDim.x) * blockDim.x)
-    buf[f * n + i] = u[f * stride + list[i]];
+// Peer-major message layout (one contiguous message per peer):
+// the n_p entries for peer p occupy buf[NF * off[p], NF * off[p + 1]) as a
+// [NF][n_p] block, off = prefix sums of the per-peer counts (nranks + 1 entries,
+// nranks <= MAX_RANKS).  Entry i belongs to the peer p with off[p] <= i < off[p+1].
+__device__ __forceinline__ int peer_of(const int64_t* off, int np, int64_t i) {
+  int p = 0;
+  while (p + 1 < np && off[p + 1] <= i) ++p;
+  return p;
 }
 
-void launch_gather_pack(const double* u, int64_t stride, const int32_t* list, int64_t n,
+__global__ void k_pack(const double* __restrict__ u, int64_t stride,
+                       const int32_t* __restrict__ list, PeerOffsets po, double* __restrict__ buf) {
+  const int f = blockIdx.y;
+  const int64_t n = po.off[po.np];
+  for (int64_t i = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; i < n;
+       i += int64_t(gridDim.x) * blockDim.x) {
+    const int p = peer_of(po.off, po.np, i);
+    const int64_t o = po.off[p], np_ = po.off[p + 1] - o;
+    buf[NF * o + f * np_ + (i - o)] = u[f * stride + list[i]];
+  }
+}
+
+void launch_gather_pack(const double* u, int64_t stride, const int32_t* list, const PeerOffsets& po,
                         double* buf, cudaStream_t s) {
+  const int64_t n = po.off[po.np];
   if (n <= 0) return;
   int blocks = int((n + 255) / 256);
   if (blocks > 148 * 4) blocks = 148 * 4;
-  k_pack<<<dim3(blocks, NF), 256, 0, s>>>(u, stride, list, n, buf);
+  k_pack<<<dim3(blocks, NF), 256, 0, s>>>(u, stride, list, po, buf);
 }
 
-__global__ void k_unpack(double* __restrict__ u, int64_t stride, int64_t offset,
-                         const double* __restrict__ buf, int64_t n) {
+// ghost slice of u (peer-major: DOFs received from peer p at n_owned + off[p] ..)
+// from the peer-major receive buffer
+__global__ void k_unpack(double* __restrict__ u, int64_t stride, int64_t n_owned,
+                         const double* __restrict__ buf, PeerOffsets po) {
   const int f = blockIdx.y;
+  const int64_t n = po.off[po.np];
   for (int64_t i = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; i < n;
-       i += int64_t(gridDim.x) * blockDim.x)
-    u[f * stride + offset + i] = buf[f * n + i];
+       i += int64_t(gridDim.x) * blockDim.x) {
+    const int p = peer_of(po.off, po.np, i);
+    const int64_t o = po.off[p], np_ = po.off[p + 1] - o;
+    u[f * stride + n_owned + i] = buf[NF * o + f * np_ + (i - o)];
+  }
 }
 
-void launch_scatter_unpack(double* u, int64_t stride, int64_t offset, const double* buf,
-                           int64_t n_total, cudaStream_t s) {
-  if (n_total <= 0) return;
-  int blocks = int((n_total + 255) / 256);
+void launch_scatter_unpack(double* u, int64_t stride, int64_t n_owned, const double* buf,
+                           const PeerOffsets& po, cudaStream_t s) {
+  const int64_t n = po.off[po.np];
+  if (n <= 0) return;
+  int blocks = int((n + 255) / 256);
   if (blocks > 148 * 4) blocks = 148 * 4;
-  k_unpack<<<dim3(blocks, NF), 256, 0, s>>>(u, stride, offset, buf, n_total);
+  k_unpack<<<dim3(blocks, NF), 256, 0, s>>>(u, stride, n_owned, buf, po);
 }
 
 // ------------------------------------------------------ fp64 microbenchmark

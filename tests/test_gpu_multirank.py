@@ -120,3 +120,108 @@ def test_interior_octants_need_no_ghost_values(world):
         assert sel.sum() > 0
         assert np.isfinite(got[:, sel]).all(), f"rank {r}: an interior octant read a ghost value"
         assert np.array_equal(got[:, sel], rfull[:, gid[:n_own]][:, sel]), f"rank {r} differs"
+
+
+# ------------------------------------------------ libdgr's own exchange (group)
+
+def _rank_meshes(cfg, world, u):
+    meshes, states, gids = [], [], []
+    for r in range(world):
+        m = dgr.Mesh(cfg, rank=r, nranks=world)
+        gid = m.export(dgr.MAP_DOF_GID, np.int64)
+        st = torch.zeros((NF, m.dof_stride), dtype=torch.float64, device="cuda")
+        st[:, :m.info["n_dof_owned"]] = torch.from_numpy(u[:, gid[:m.info["n_dof_owned"]]])
+        meshes.append(m)
+        states.append(st)
+        gids.append(gid)
+    return meshes, states, gids
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_group_exchange_pack_and_ghosts(world):
+    """libdgr's exchange code path (k_pack -> peer copies -> k_unpack, the
+    buffers and offsets the NCCL transport uses): the packed send buffer equals
+    u[f][DGR_MAP_SEND] laid out peer-major ([24][n_p] per peer), and after the
+    exchange every ghost DOF holds its owner's value (DGR_MAP_DOF_GID)."""
+    need_gpu()
+    cfg = configs.small_bbh(lmax=6, rho=0.5)
+    om = OracleMesh(cfg)
+    om.build_dofs()
+    u = initial.for_config(cfg, om.dof_coords(), kind="random", seed=4)
+    meshes, states, gids = _rank_meshes(cfg, world, u)
+    g = dgr.Group(meshes)
+    g.ghost_exchange(states)
+    torch.cuda.synchronize()
+    for r, m in enumerate(meshes):
+        send = m.export(dgr.MAP_SEND, np.int32)
+        sc = m.export(dgr.MAP_SEND_COUNTS, np.int64)
+        buf = m.export(dgr.MAP_SENDBUF, np.float64)
+        host = states[r].cpu().numpy()
+        want, off = [], 0
+        for p in range(world):
+            ids = send[off:off + sc[p]]
+            off += sc[p]
+            want.append(host[:, ids].reshape(-1))      # [24][n_p] block
+        want = np.concatenate(want) if want else np.zeros(0)
+        assert np.array_equal(buf, want), f"rank {r}: packed send buffer"
+        no, nd = m.info["n_dof_owned"], m.n_dof
+        assert np.array_equal(host[:, no:nd], u[:, gids[r][no:nd]]), f"rank {r}: ghosts"
+    g.close()
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_group_rk4_bit_identical(world):
+    """dgr_group_rk4_step (libdgr's exchange, overlapped with the interior
+    octants on the mesh's exchange stream) gives owned DOFs bit-identical to
+    the single-rank dgr_rk4_step after RK4 steps."""
+    need_gpu()
+    cfg = configs.small_bbh(lmax=6, rho=0.5)
+    om = OracleMesh(cfg)
+    om.build_dofs()
+    u = initial.for_config(cfg, om.dof_coords())
+    dt = ork4.dt_courant(om)
+    ref = dgr.Mesh(cfg)
+    ur = to_dev(u, ref.dof_stride)
+    meshes, states, gids = _rank_meshes(cfg, world, u)
+    assert any(0 < m.info["n_oct_interior"] < m.info["n_oct_local"] for m in meshes)
+    g = dgr.Group(meshes)
+    side = [torch.cuda.Stream() for _ in range(world)]   # one stream per rank
+    for _ in range(2):
+        ref.rk4_step(ur, dt)
+        g.rk4_step(states, dt, streams=[s.cuda_stream for s in side])
+    torch.cuda.synchronize()
+    full = ur[:, :om.n_dof].cpu().numpy()
+    for r, m in enumerate(meshes):
+        no = m.info["n_dof_owned"]
+        assert np.array_equal(states[r][:, :no].cpu().numpy(), full[:, gids[r][:no]]), r
+    g.close()
+
+
+def test_step_without_communicator_is_rejected():
+    """on an external-exchange mesh dgr_rk4_step / dgr_rk4_step_host
+    would read stale ghosts, so they return DGR_ERR_STATE (-6)."""
+    need_gpu()
+    cfg = configs.small_bbh(lmax=6, rho=0.5)
+    m = dgr.Mesh(cfg, rank=0, nranks=2)
+    st = m.new_state()
+    with pytest.raises(dgr.DgrError) as e:
+        m.rk4_step(st, 0.01)
+    assert e.value.status == -6
+    h = torch.zeros((NF, m.dof_stride), dtype=torch.float64)
+    with pytest.raises(dgr.DgrError) as e:
+        m.rk4_step_host([h], [h], 0.01)
+    assert e.value.status == -6
+    with pytest.raises(dgr.DgrError) as e:
+        m.ghost_exchange(st)
+    assert e.value.status == -6
+
+
+def test_device_calls_validate_tensors():
+    need_gpu()
+    m = dgr.Mesh(configs.c1_uniform())
+    with pytest.raises(ValueError):
+        m.rhs(torch.zeros((NF, m.dof_stride), dtype=torch.float32, device="cuda"))
+    with pytest.raises(ValueError):
+        m.rhs(torch.zeros((NF, m.dof_stride), dtype=torch.float64))          # CPU
+    with pytest.raises(ValueError):
+        m.rk4_step(torch.zeros((NF, m.dof_stride - 32), dtype=torch.float64, device="cuda"), 0.1)

@@ -14,7 +14,14 @@ cases = {
   "c1_gw": (configs.c1_uniform(), "gauge_wave"),
   "c1_rand": (configs.c1_uniform(), "random"),
   "bbh_small": (configs.small_bbh(lmax=6, rho=0.5), "bl"),
+  "bbh_small_rand": (configs.small_bbh(lmax=6, rho=0.5), "random"),
+  "bbh5_bl": (configs.small_bbh(lmax=5, rho=0.4), "bl"),
+  "bbh5_rand": (configs.small_bbh(lmax=5, rho=0.4), "random"),
+  "small_rand": (configs.small_adaptive(lmax=5, rho=0.5), "random"),
 }
+only = sys.argv[1:]
+if only:
+    cases = {k: v for k, v in cases.items() if k in only}
 for name, (cfg, kind) in cases.items():
     m = dgr.Mesh(cfg)
     xyz = m.dof_xyz_host(); n = xyz.shape[1]

@@ -253,6 +253,27 @@ dgr_status dgr_rk4_step_host(dgr_mesh m, double dt, int64_t n, const double* con
 dgr_status dgr_constraints(dgr_mesh m, double* u, double* c, double* norms_host,
                            const dgr_params* prm, void* stream);
 
+/* The paper's code-generation study (§IV-B, Table II; SURVEY
+ * §8(f) row 3) — not the default path (dgr_rhs fuses the derivatives with the
+ * algebra and never stores them):
+ * dgr_rhs_inputs: the 234 inputs of the algebraic part A at every interior
+ *   point of the owned octants, in[k * ld + e * 343 + p] (ld >= n_oct_local *
+ *   343): k < 24 field values, then 72 first derivatives (24 + 3 f + a), 66
+ *   second derivatives of alpha, chi, beta^i, gt_ij (96 + 6 s + q, q over
+ *   xx xy xz yy yz zz), 72 Kreiss-Oliger terms (162 + 3 f + a, scaled by
+ *   sigma / (64 h)) — the layout of codegen/bssn_sym.py.  Ghost exchange +
+ *   unzip into the library's patch buffer + one derivative kernel.
+ * dgr_rhs_algebra: out[f * ld + i] = A_f + KO_f at n points of in (same ld) by
+ *   the generated kernel `variant`: 0 SymPyGR-style global CSE, 1 binary
+ *   reduction over the expression DAG (Alg. 3), 2 staged CSE; occ = 1 selects
+ *   the occupancy-constrained build (256 threads x 4 CTAs, <= 64 registers,
+ *   the analogue of the paper's __launch_bounds__(343,3)).  Device pointers;
+ *   no mesh. */
+dgr_status dgr_rhs_inputs(dgr_mesh m, double* u, double* in, int64_t ld, const dgr_params* prm,
+                          void* stream);
+dgr_status dgr_rhs_algebra(int variant, int occ, const double* in, double* out, int64_t n,
+                           int64_t ld, const dgr_params* prm, void* stream);
+
 /* In-process rank group: n meshes of one octree, meshes[r] = rank r of n,
  * each created with nccl_id = NULL (one per device, or several on one device),
  * driven by ONE process.  Their ghost exchange is libdgr's own (SURVEY §8e
@@ -293,7 +314,14 @@ dgr_status dgr_group_destroy(dgr_group g);
  *     DOF it is the zip owner of) and the RK4 update streams the
  *     DOF-ordered RHS; 0 = RHS per octant point, then the zip gather (k_zip /
  *     k_zip_rk4).  Both give bit-identical results. */
-enum { DGR_OPT_FUSED_UNZIP = 1, DGR_OPT_PHASES = 2, DGR_OPT_PREPASS = 3, DGR_OPT_ZIP_STORE = 4 };
+/*   DGR_OPT_GRAPH (default 1): dgr_rk4_step replays a CUDA graph of its four
+ *     stages: the first call with given (u, dt, params) runs eagerly, the second
+ *     captures the launch sequence on a library stream, later calls launch the
+ *     graph on `stream` (one launch instead of 16+).  Changing any option or
+ *     the arguments re-captures.  Not used while profiling (dgr_profile_enable)
+ *     or on NCCL meshes.  Bit-identical to the eager sequence. */
+enum { DGR_OPT_FUSED_UNZIP = 1, DGR_OPT_PHASES = 2, DGR_OPT_PREPASS = 3, DGR_OPT_ZIP_STORE = 4,
+       DGR_OPT_GRAPH = 5 };
 dgr_status dgr_set_option(dgr_mesh m, int option, int64_t value);
 
 /* Device-side timing helper for benchmarks: number of kernel launches the last

@@ -27,7 +27,7 @@ NPATCH = 2197
 MAP_OCTANTS, MAP_O2N, MAP_HANGING, MAP_PAD_SRC, MAP_PAD_KIND, MAP_ZIP = 0, 1, 2, 3, 4, 5
 MAP_DOF_GID, MAP_DOF_XYZ, MAP_SEND, MAP_SEND_COUNTS, MAP_RECV_COUNTS = 6, 7, 8, 9, 10
 MAP_LOCAL_OCTS, MAP_O2N_LOCAL, MAP_RHS_ORDER, MAP_SENDBUF = 11, 12, 13, 14
-OPT_FUSED_UNZIP, OPT_PHASES, OPT_PREPASS, OPT_ZIP_STORE = 1, 2, 3, 4
+OPT_FUSED_UNZIP, OPT_PHASES, OPT_PREPASS, OPT_ZIP_STORE, OPT_GRAPH = 1, 2, 3, 4, 5
 
 
 class DgrError(RuntimeError):
@@ -370,6 +370,11 @@ class Mesh:
         """DGR_OPT_ZIP_STORE: zip in the RHS kernel's store and stream the RK4 update
         (1) or write the RHS per octant point and zip-gather it (0); bit-identical."""
         _check(lib().dgr_set_option(self._h, OPT_ZIP_STORE, int(bool(on))))
+
+    def set_graph(self, on=True):
+        """DGR_OPT_GRAPH: rk4_step replays a CUDA graph of its four stages (captured
+        at the second call with the same arguments); bit-identical to eager."""
+        _check(lib().dgr_set_option(self._h, OPT_GRAPH, int(bool(on))))
 
     def set_phases(self, mode=0):
         """DGR_OPT_PHASES: 0 = overlap interior octants with the ghost exchange when

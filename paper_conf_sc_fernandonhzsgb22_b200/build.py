@@ -26,7 +26,8 @@ CU_FLAGS = ARCH + ["-O3", "-lineinfo", "-std=c++17", "--expt-relaxed-constexpr",
                    "-Xcompiler", "-fPIC,-ffp-contract=off", "-I", INC, "-I", CSRC]
 CXX_FLAGS = ["-O2", "-fPIC", "-fopenmp", "-ffp-contract=off", "-std=c++17", "-I", INC, "-I", CSRC]
 
-SOURCES_CU = ["api.cu", "kernels.cu", "unzip_kernel.cu", "rhs_kernel.cu", "constraints_kernel.cu"]
+SOURCES_CU = ["api.cu", "kernels.cu", "unzip_kernel.cu", "rhs_kernel.cu", "constraints_kernel.cu",
+              "rhs_inputs.cu", "gen/rhs_alg.cu"]
 SOURCES_CXX = ["host_mesh.cpp"]
 
 
@@ -76,7 +77,7 @@ def build(verbose: bool = False, ptxas_verbose: bool = False, variant: str = "")
             changed = True
     for s in SOURCES_CU:
         src = os.path.join(CSRC, s)
-        obj = os.path.join(objdir, s + ".o")
+        obj = os.path.join(objdir, s.replace("/", "_") + ".o")
         objs.append(obj)
         if _stale(obj, src):
             extra = ["-Xptxas", "-v"] if ptxas_verbose else []

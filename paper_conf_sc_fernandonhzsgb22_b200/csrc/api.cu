@@ -143,6 +143,19 @@ struct dgr_mesh_s {
   PeerOffsets po_send{}, po_recv{};
   int64_t launches = 0;
   bool fused = true;            // DGR_OPT_FUSED_UNZIP (C3: 40.4 ms/step fused, 41.2 two-pass)
+  // DGR_OPT_GRAPH: dgr_rk4_step replays a CUDA graph of its 4 stages (captured
+  // on a library stream at the second call with the same arguments)
+  bool use_graph = true;
+  cudaStream_t gstream = nullptr;
+  cudaGraphExec_t gexec = nullptr;
+  int64_t glaunches = 0;
+  struct GraphKey { const double* u; double dt; dgr_params prm; bool has_prm; } gkey{};
+  int gseen = 0;                // calls with the current key (0: none)
+  void drop_graph() {
+    if (gexec) cudaGraphExecDestroy(gexec);
+    gexec = nullptr;
+    gseen = 0;
+  }
   // profiling
   bool prof = false;
   struct Pend { int cls; cudaEvent_t a, b; };
@@ -181,6 +194,8 @@ struct dgr_mesh_s {
       if (ev_out[b]) cudaEventDestroy(ev_out[b]);
     }
     if (ev_host0) cudaEventDestroy(ev_host0);
+    if (gexec) cudaGraphExecDestroy(gexec);
+    if (gstream) cudaStreamDestroy(gstream);
     if (h2d) cudaStreamDestroy(h2d);
     if (d2h) cudaStreamDestroy(d2h);
   }
@@ -1061,6 +1076,11 @@ dgr_status dgr_rk4_stage(dgr_mesh m, int s_, double dt, double* u_n, double* u_s
   return stage(m, s_, dt, u_n, u_s, acc, acc, prm, static_cast<cudaStream_t>(stream));
 }
 
+static bool same_key(const dgr_mesh_s::GraphKey& a, const dgr_mesh_s::GraphKey& b) {
+  return a.u == b.u && std::memcmp(&a.dt, &b.dt, sizeof(double)) == 0 && a.has_prm == b.has_prm &&
+         (!a.has_prm || std::memcmp(&a.prm, &b.prm, sizeof(dgr_params)) == 0);
+}
+
 dgr_status dgr_rk4_step(dgr_mesh m, double dt, double* u, const dgr_params* prm, void* stream) {
   dgr_status s = need_device(m);
   if (s) return s;
@@ -1069,9 +1089,42 @@ dgr_status dgr_rk4_step(dgr_mesh m, double dt, double* u, const dgr_params* prm,
     return fail(DGR_ERR_STATE, "dgr_rk4_step needs a communicator: external-exchange meshes step "
                                "with dgr_rk4_stage, grouped meshes with dgr_group_rk4_step");
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  m->launches = 0;
-  for (int k = 0; k < 4; ++k)
-    if ((s = stage(m, k, dt, u, m->d_us, m->d_acc, u, prm, st))) return s;
+  auto eager = [&](cudaStream_t q) -> dgr_status {
+    m->launches = 0;
+    for (int k = 0; k < 4; ++k)
+      if (dgr_status e = stage(m, k, dt, u, m->d_us, m->d_acc, u, prm, q)) return e;
+    return DGR_OK;
+  };
+  // CUDA graph of the step (the 16+ launches of the 4 stages, and with N > 1
+  // the exchange stream's pack / NCCL / unpack, captured once): the first call
+  // with given arguments runs eagerly (lazy allocations happen there), the
+  // second captures on a library stream and instantiates, later calls replay.
+  // Profiling (per-launch events) and NCCL meshes run eagerly.
+  if (!m->use_graph || m->prof || m->comm) return eager(st);
+  dgr_mesh_s::GraphKey key{u, dt, prm ? *prm : dgr_params{}, prm != nullptr};
+  if (!same_key(key, m->gkey)) {
+    m->drop_graph();
+    m->gkey = key;
+  }
+  if (m->gseen++ == 0) return eager(st);
+  if (!m->gexec) {
+    if (!m->gstream) CUDA_TRY(cudaStreamCreateWithFlags(&m->gstream, cudaStreamNonBlocking));
+    CUDA_TRY(cudaStreamBeginCapture(m->gstream, cudaStreamCaptureModeThreadLocal));
+    dgr_status e = eager(m->gstream);
+    cudaGraph_t graph = nullptr;
+    cudaError_t ce = cudaStreamEndCapture(m->gstream, &graph);
+    if (e) {
+      if (graph) cudaGraphDestroy(graph);
+      return e;
+    }
+    CUDA_TRY(ce);
+    ce = cudaGraphInstantiate(&m->gexec, graph, 0);
+    cudaGraphDestroy(graph);
+    CUDA_TRY(ce);
+    m->glaunches = m->launches;
+  }
+  CUDA_TRY(cudaGraphLaunch(m->gexec, st));
+  m->launches = m->glaunches;
   return DGR_OK;
 }
 
@@ -1190,15 +1243,44 @@ dgr_status dgr_constraints(dgr_mesh m, double* u, double* c, double* norms_host,
   return DGR_OK;
 }
 
+dgr_status dgr_rhs_inputs(dgr_mesh m, double* u, double* in, int64_t ld, const dgr_params* prm,
+                          void* stream) {
+  dgr_status s = need_device(m);
+  if (s) return s;
+  const int64_t n = int64_t(m->dm.n_owned) * NPT;
+  if (!u || !in || ld < n) return fail(DGR_ERR_ARG, "bad rhs_inputs args (ld >= n_oct_local * 343)");
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  m->launches = 0;
+  if ((s = exchange(m, u, st))) return s;
+  if ((s = do_unzip(m, u, NF, st))) return s;
+  const RhsParams rp = to_rp(prm);
+  PROF(m, 3, st, launch_rhs_inputs(m->dm, m->d_patch, in, ld, rp.ko_sigma, st));
+  CUDA_TRY(cudaGetLastError());
+  return DGR_OK;
+}
+
+dgr_status dgr_rhs_algebra(int variant, int occ, const double* in, double* out, int64_t n,
+                           int64_t ld, const dgr_params* prm, void* stream) {
+  if (variant < 0 || variant > 2 || !in || !out || n < 0 || ld < n)
+    return fail(DGR_ERR_ARG, "bad rhs_algebra args (variant 0..2, ld >= n)");
+  const RhsParams rp = to_rp(prm);
+  const AlgParams ap{rp.eta, rp.lambda_f0, rp.lambda_f1, rp.chi_floor};
+  launch_rhs_alg(variant, occ ? 1 : 0, in, out, n, ld, ap, static_cast<cudaStream_t>(stream));
+  CUDA_TRY(cudaGetLastError());
+  return DGR_OK;
+}
+
 dgr_status dgr_set_option(dgr_mesh m, int option, int64_t value) {
   if (!m) return fail(DGR_ERR_ARG, "null mesh");
   switch (option) {
-    case DGR_OPT_FUSED_UNZIP: m->fused = value != 0; return DGR_OK;
-    case DGR_OPT_PREPASS: m->prepass = value != 0; return DGR_OK;
-    case DGR_OPT_ZIP_STORE: m->zip_store = value != 0; return DGR_OK;
+    case DGR_OPT_GRAPH: m->use_graph = value != 0; m->drop_graph(); return DGR_OK;
+    case DGR_OPT_FUSED_UNZIP: m->fused = value != 0; m->drop_graph(); return DGR_OK;
+    case DGR_OPT_PREPASS: m->prepass = value != 0; m->drop_graph(); return DGR_OK;
+    case DGR_OPT_ZIP_STORE: m->zip_store = value != 0; m->drop_graph(); return DGR_OK;
     case DGR_OPT_PHASES:
       if (value < 0 || value > 2) return fail(DGR_ERR_ARG, "DGR_OPT_PHASES is 0, 1 or 2");
       m->phases = int(value);
+      m->drop_graph();
       return DGR_OK;
   }
   return fail(DGR_ERR_ARG, "unknown option");
@@ -1207,6 +1289,7 @@ dgr_status dgr_set_option(dgr_mesh m, int option, int64_t value) {
 dgr_status dgr_profile_enable(dgr_mesh m, int on) {
   if (!m) return fail(DGR_ERR_ARG, "null mesh");
   m->prof = on != 0;
+  m->drop_graph();
   return DGR_OK;
 }
 
@@ -1325,8 +1408,8 @@ static dgr_status group_exchange(dgr_group_s* g, double* const* u, void* const* 
 
 static dgr_status group_check(dgr_group g, const void* const* a, const void* const* b) {
   if (!g || !a || !b) return fail(DGR_ERR_ARG, "null group argument");
-  for (size_t r = 0; r < g->m.size(); ++r)
-    if (!a[r] || !b[r]) return fail(DGR_ERR_ARG, "null state or stream entry");
+  for (size_t r = 0; r < g->m.size(); ++r)   // (a null stream is the legacy default stream)
+    if (!a[r]) return fail(DGR_ERR_ARG, "null state entry");
   return DGR_OK;
 }
 
@@ -1354,6 +1437,9 @@ dgr_status dgr_group_create(dgr_mesh* meshes, int n, dgr_group* out) {
   for (int r = 0; r < n; ++r) {
     DeviceGuard dg(meshes[r]->dev_id);
     CUDA_TRY(cudaEventCreateWithFlags(&g->ev_packed[r], cudaEventDisableTiming));
+    // every rank's exchange stream and events exist before the first exchange
+    // (rank r's pack waits on its peers' ev_xdone)
+    if (dgr_status e = ensure_xstream(meshes[r])) return e;
     for (int p = 0; p < n; ++p)
       if (p != r && meshes[r]->dev_id != meshes[p]->dev_id) {
         int ok = 0;

@@ -309,12 +309,10 @@ __global__ void __launch_bounds__(CT, 1)
 void launch_constraints(const DevMesh& m, const double* patches, double* c_oct,
                         const RhsParams& p, cudaStream_t s) {
   if (m.n_owned <= 0) return;
-  static bool attr = false;
-  if (!attr) {
+  static std::atomic<bool> done[MAX_DEVICES];
+  if (first_on_device(done))
     cudaFuncSetAttribute(k_constraints, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          int(SMEM_BYTES));
-    attr = true;
-  }
   k_constraints<<<m.n_owned, CT, SMEM_BYTES, s>>>(m, patches, c_oct, p);
 }
 

@@ -3,9 +3,19 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <atomic>
+
 #include "host_mesh.hpp"
 
 namespace dgr {
+
+// Per-device one-time setup (kernel attributes are per device context): true
+// the first time it is called for the current device with this flag array;
+// thread-safe (a static bool / SM count cached from the first
+// device broke meshes created on a second GPU in the same process).
+constexpr int MAX_DEVICES = 64;
+bool first_on_device(std::atomic<bool>* flags);
+int sm_count();
 
 constexpr int NF = 24;            // BSSN fields
 constexpr int PATCH_PITCH = 2208; // doubles per patch: 13^3 = 2197 padded to 128 B
@@ -115,6 +125,19 @@ void launch_rhs(const DevMesh& m, const double* src, double* rhs_oct, const RhsP
                 double* pre = nullptr, double* rhs_dof = nullptr);
 size_t rhs_smem_bytes();
 void upload_rhs_tables(const double* wext);
+
+// gen/rhs_alg.cu (generated by codegen/gen.py): the algebraic part A of the RHS
+// in the paper's code-generation styles (Table II), in[234][ld] -> out[24][ld];
+// variant 0 sympygr_cse, 1 binary_reduce, 2 staged_cse; occ = 1: the
+// occupancy-constrained build (256 threads x 4 CTAs per SM, <= 64 registers)
+struct AlgParams {
+  double eta, lambda_f0, lambda_f1, chi_floor;
+};
+void launch_rhs_alg(int variant, int occ, const double* in, double* out, int64_t n, int64_t ld,
+                    const AlgParams& p, cudaStream_t s);
+// rhs_inputs.cu: the 234 inputs of A per interior point from the patch buffer
+void launch_rhs_inputs(const DevMesh& m, const double* patches, double* in, int64_t ld,
+                       double ko_sigma, cudaStream_t s);
 
 // constraints_kernel.cu
 void launch_constraints(const DevMesh& m, const double* patches, double* c_oct,

@@ -196,6 +196,28 @@ void launch_dof_coords(const DevMesh& m, const int64_t* dof_node, double* xyz,
                                       unit);
 }
 
+// ------------------------------------------------------- per-device setup
+bool first_on_device(std::atomic<bool>* flags) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 0 || dev >= MAX_DEVICES) return false;
+  return !flags[dev].exchange(true);
+}
+
+int sm_count() {
+  static std::atomic<int> cache[MAX_DEVICES];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 0 || dev >= MAX_DEVICES) return 148;
+  int n = cache[dev].load();
+  if (!n) {
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (n <= 0) n = 148;
+    cache[dev].store(n);
+  }
+  return n;
+}
+
 // ------------------------------------------------------- ghost pack/unpack
 // Peer-major message layout (one contiguous message per peer):
 // the n_p entries for peer p occupy buf[NF * off[p], NF * off[p + 1]) as a

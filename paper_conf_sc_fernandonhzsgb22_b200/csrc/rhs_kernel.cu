@@ -1248,8 +1248,8 @@ void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const 
                 bool fused, int64_t first, int64_t count, int leave_sm, cudaStream_t s,
                 double* pre, double* rhs_dof) {
   if (count <= 0) return;
-  static int n_sm = 0;
-  if (!n_sm) {
+  static std::atomic<bool> done[MAX_DEVICES];
+  if (first_on_device(done)) {
     const int sb = int(SMEM_BYTES);
     cudaFuncSetAttribute(k_rhs<false, false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb);
     cudaFuncSetAttribute(k_rhs<true, false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb);
@@ -1258,11 +1258,8 @@ void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const 
     cudaFuncSetAttribute(k_rhs<true, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb);
     cudaFuncSetAttribute(k_gt_pre, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          int(PRE_SMEM_BYTES));
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&n_sm, cudaDevAttrMultiProcessorCount, dev);
-    if (n_sm <= 0) n_sm = 148;
   }
+  const int n_sm = sm_count();
   // persistent: one CTA per SM (227 KB of shared memory each)
   const int64_t cap = leave_sm > 0 && n_sm - leave_sm > 0 ? n_sm - leave_sm : n_sm;
   const int grid = int(count < cap ? count : cap);

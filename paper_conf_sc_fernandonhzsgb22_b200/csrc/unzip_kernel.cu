@@ -192,11 +192,9 @@ void launch_interp(const DevMesh& m, const double* u, int nf, int64_t first, int
                    cudaStream_t s) {
   if (count <= 0) return;
   const size_t dyn = size_t(IP_FG) * IP_FIELD * sizeof(double);
-  static bool attr = false;
-  if (!attr) {
+  static std::atomic<bool> done[MAX_DEVICES];
+  if (first_on_device(done))
     cudaFuncSetAttribute(k_interp, cudaFuncAttributeMaxDynamicSharedMemorySize, int(dyn));
-    attr = true;
-  }
   k_interp<<<dim3(unsigned(count), (nf + IP_FG - 1) / IP_FG), IP_THREADS, dyn, s>>>(m, u, nf,
                                                                                     first);
 }

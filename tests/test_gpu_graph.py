@@ -1,0 +1,45 @@
+"""CUDA-graph replay of dgr_rk4_step (DGR_OPT_GRAPH, SURVEY §8d timing
+hygiene): the captured step is bit-identical to the eager launch sequence,
+re-captures when the arguments or options change, and reports the same
+launch count."""
+import numpy as np
+import pytest
+
+import paper_conf_sc_fernandonhzsgb22_b200 as dgr
+from synth import configs, initial
+
+from .gpu_util import need_gpu, to_dev, torch
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.mark.parametrize("cfgf", [configs.c1_uniform, lambda: configs.small_bbh(lmax=5, rho=0.4)])
+def test_graph_step_bit_identical(cfgf):
+    need_gpu()
+    cfg = cfgf()
+    m = dgr.Mesh(cfg)
+    xyz = m.dof_xyz_host()
+    u = initial.for_config(cfg, xyz, seed=2)
+    dt = 0.25 * m.info["h_min"]
+    a = to_dev(u, m.dof_stride)
+    b = a.clone()
+    m.set_graph(False)
+    for _ in range(4):
+        m.rk4_step(a, dt)
+    n_eager = m.last_launch_count()
+    m.set_graph(True)
+    for k in range(4):            # eager, capture+launch, launch, launch
+        m.rk4_step(b, dt)
+        assert m.last_launch_count() == n_eager, k
+    torch.cuda.synchronize()
+    assert torch.equal(a, b)
+    # other arguments -> re-capture; still identical
+    c, d = a.clone(), a.clone()
+    m.rk4_step(c, 0.5 * dt)
+    m.rk4_step(c, 0.5 * dt)
+    m.set_graph(False)
+    m.rk4_step(d, 0.5 * dt)
+    m.rk4_step(d, 0.5 * dt)
+    torch.cuda.synchronize()
+    assert torch.equal(c, d)
+    assert np.isfinite(c.cpu().numpy()).all()

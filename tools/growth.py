@@ -1,6 +1,6 @@
 """Sensitivity of 100 RK4 steps to a 1e-13 relative perturbation (GPU, libdgr).
 Tells whether 1e-8 parity after 100 steps is attainable for a setup."""
-import sys, os
+import sys, os, dataclasses
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
 import paper_conf_sc_fernandonhzsgb22_b200 as dgr
@@ -18,6 +18,13 @@ cases = {
   "bbh5_bl": (configs.small_bbh(lmax=5, rho=0.4), "bl"),
   "bbh5_rand": (configs.small_bbh(lmax=5, rho=0.4), "random"),
   "small_rand": (configs.small_adaptive(lmax=5, rho=0.5), "random"),
+  # smooth constraint-satisfying data (gauge wave, A = 0.1, one wavelength
+  # across the domain) on the adaptive puncture meshes (mesh from the
+  # punctures, data independent of them)
+  "bbh_small_gw": (configs.small_bbh(lmax=6, rho=0.5), "gauge_wave"),
+  "bbh5_gw": (configs.small_bbh(lmax=5, rho=0.4), "gauge_wave"),
+  "small_gw": (configs.small_adaptive(lmax=5, rho=0.5), "gauge_wave"),
+  "bbh_small_gw_per": (dataclasses.replace(configs.small_bbh(lmax=6, rho=0.5), periodic=True), "gauge_wave"),
 }
 only = sys.argv[1:]
 if only:

@@ -66,7 +66,8 @@ MUTATIONS = [
     (B, 'DDa_tr = d.chi * np.einsum', 'DDa_tr = np.einsum', "eq14 drop chi"),
     # constraints
     (C, '+ (2.0 / 3.0) * d.K * d.K - np.einsum', '+ (1.0 / 3.0) * d.K * d.K - np.einsum', "H 2/3 -> 1/3"),
-    (C, 'M = (np.einsum("jij...->i...", d_Aup)', 'M = (np.einsum("iij...->j...", d_Aup)', "M divergence index"),
+    # (d_j At^ij -> d_i At^ij is an equivalent mutant: At^ij is symmetric)
+    (C, 'M = (np.einsum("jij...->i...", d_Aup)', 'M = (np.einsum("ijj...->i...", d_Aup)', "M divergence -> gradient of trace"),
     (C, '- 1.5 / chi * np.einsum("ij...,j...->i...", A_up, d.d_chi))', ')', "M drop chi term"),
     (C, 'Gc = d.Gt - G["CalGt"]', 'Gc = d.Gt + G["CalGt"]', "G sign"),
 ]

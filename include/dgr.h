@@ -274,6 +274,33 @@ dgr_status dgr_rhs_inputs(dgr_mesh m, double* u, double* in, int64_t ld, const d
 dgr_status dgr_rhs_algebra(int variant, int occ, const double* in, double* out, int64_t n,
                            int64_t ld, const dgr_params* prm, void* stream);
 
+/* Regrid (Alg. 1 line 3 construct_grid; refinement tolerance
+ * P:L465; the paper delegates it to DENDRO-GR without formulas: readings
+ * R30-R32 of DESIGN.md).
+ * dgr_regrid_indicator: w[e] (device, n_oct_local doubles) = the wavelet
+ *   indicator of owned octant e — the largest |P - prediction| over the interior
+ *   points of its 13^3 patches of the fields in field_mask (bit f = field f),
+ *   the prediction being the tensor degree-6 Lagrange interpolant from the
+ *   all-even patch points (spacing 2h).  0 up to rounding for data of degree
+ *   <= 6 per axis.  Ghost exchange + unzip + one kernel.
+ * dgr_regrid_octree: host; the regridded leaves from w (host, n_oct_global
+ *   doubles, global Morton order): a leaf with w > eps_refine and level <
+ *   level_max is split, a complete family of 8 sibling leaves with every w <
+ *   eps_coarsen and level > level_min (none split) is merged, then the minimal
+ *   2:1 vertex-balance closure and Morton order (every leaf changes by at most
+ *   one level).  out = NULL returns the count in *n_inout (as dgr_octree_build).
+ * dgr_regrid_transfer: u_new (the new mesh's state, owned DOFs) = the old
+ *   mesh's piecewise interpolant at every new DOF: the tensor Lagrange
+ *   interpolant of the finest old leaf containing it (lowest Morton on ties),
+ *   hanging nodes reconstructed; copies where a new DOF is an old node.  Both
+ *   meshes single-rank, same domain; synchronises `stream`. */
+dgr_status dgr_regrid_indicator(dgr_mesh m, double* u, uint32_t field_mask, double* w,
+                                void* stream);
+dgr_status dgr_regrid_octree(dgr_mesh m, const double* w, double eps_refine, double eps_coarsen,
+                             int level_min, int level_max, dgr_octant* out, int64_t* n_inout);
+dgr_status dgr_regrid_transfer(dgr_mesh old_m, double* u_old, dgr_mesh new_m, double* u_new,
+                               void* stream);
+
 /* In-process rank group: n meshes of one octree, meshes[r] = rank r of n,
  * each created with nccl_id = NULL (one per device, or several on one device),
  * driven by ONE process.  Their ghost exchange is libdgr's own (SURVEY §8e

@@ -173,6 +173,11 @@ class OracleMesh:
         self.zip_leaf, self.zip_node = zo_leaf, zo_node
         self._dofs_done = True
 
+    def dof_lattice(self):
+        """Lattice coordinates [n_dof, 3] of the DOFs (X = 6 anchor + i side)."""
+        self.build_dofs()
+        return self.node_X(self.zip_leaf, _local_ijk()[self.zip_node])
+
     def dof_coords(self):
         """Physical coordinates [3, n_dof] of the DOFs."""
         self.build_dofs()

@@ -82,7 +82,8 @@ EXPORTED = ["dgr_status_string", "dgr_last_error", "dgr_version", "dgr_octree_bu
             "dgr_last_launch_count",
             "dgr_profile_enable", "dgr_profile_read", "dgr_bench_dfma", "dgr_set_option",
             "dgr_group_create", "dgr_group_ghost_exchange", "dgr_group_rk4_step",
-            "dgr_group_destroy"]
+            "dgr_group_destroy", "dgr_rhs_inputs", "dgr_rhs_algebra", "dgr_regrid_indicator",
+            "dgr_regrid_octree", "dgr_regrid_transfer"]
 PROF_CLASSES = ["elements", "hanging", "unzip", "rhs", "zip_rk4", "exchange", "constraints",
                 "interp"]
 
@@ -125,12 +126,19 @@ def lib():
         L.dgr_group_ghost_exchange.argtypes = [vp, C.POINTER(vp), C.POINTER(vp)]
         L.dgr_group_rk4_step.argtypes = [vp, dp, C.POINTER(vp), C.POINTER(_Params), C.POINTER(vp)]
         L.dgr_group_destroy.argtypes = [vp]
+        L.dgr_rhs_inputs.argtypes = [vp, vp, vp, i64, C.POINTER(_Params), vp]
+        L.dgr_rhs_algebra.argtypes = [i32, i32, vp, vp, i64, i64, C.POINTER(_Params), vp]
+        L.dgr_regrid_indicator.argtypes = [vp, vp, C.c_uint32, vp, vp]
+        L.dgr_regrid_octree.argtypes = [vp, vp, dp, dp, i32, i32, vp, C.POINTER(i64)]
+        L.dgr_regrid_transfer.argtypes = [vp, vp, vp, vp, vp]
         for f in ["dgr_octree_build", "dgr_mesh_create", "dgr_mesh_info_get",
                   "dgr_mesh_export_maps", "dgr_mesh_destroy", "dgr_dof_coords", "dgr_unzip",
                   "dgr_ghost_exchange", "dgr_rhs_patches", "dgr_rhs", "dgr_rk4_stage",
                   "dgr_rk4_step", "dgr_rk4_step_host", "dgr_constraints", "dgr_profile_enable", "dgr_profile_read", "dgr_set_option",
                   "dgr_bench_dfma", "dgr_group_create", "dgr_group_ghost_exchange",
-                  "dgr_group_rk4_step", "dgr_group_destroy"]:
+                  "dgr_group_rk4_step", "dgr_group_destroy", "dgr_rhs_inputs",
+                  "dgr_rhs_algebra", "dgr_regrid_indicator", "dgr_regrid_octree",
+                  "dgr_regrid_transfer"]:
             getattr(L, f).restype = i32
         _lib = L
     return _lib
@@ -353,6 +361,51 @@ class Mesh:
                                      C.byref(p), _stream()))
         return out, norms.reshape(7, 2)
 
+    def rhs_inputs(self, u, prm=None, out=None):
+        """dgr_rhs_inputs: the 234 inputs of the RHS algebra at every interior point
+        of the owned octants, [234, n_oct_local * 343] (codegen/bssn_sym.py order)."""
+        import torch
+        n = self.info["n_oct_local"] * NPT
+        if out is None:
+            out = torch.empty((N_ALG_IN, n), dtype=torch.float64, device="cuda")
+        _dev(out, (N_ALG_IN, out.shape[1]), "out")
+        p = (prm or Params())._c()
+        _check(lib().dgr_rhs_inputs(self._h, self._state(u, "u"), _ptr(out), out.shape[1],
+                                    C.byref(p), _stream()))
+        return out
+
+    # ------------------------------------------------------------ regrid
+    def regrid_indicator(self, u, field_mask=0xFFFFFF, out=None):
+        """dgr_regrid_indicator: wavelet indicator per owned octant (device tensor)."""
+        import torch
+        n = self.info["n_oct_local"]
+        if out is None:
+            out = torch.empty(n, dtype=torch.float64, device="cuda")
+        _check(lib().dgr_regrid_indicator(self._h, self._state(u, "u"), int(field_mask),
+                                          _dev(out, (n,), "out"), _stream()))
+        return out
+
+    def regrid_octree(self, w, eps_refine, eps_coarsen, level_min, level_max):
+        """dgr_regrid_octree (host): the regridded leaves, uint32 [n, 4]."""
+        w = np.ascontiguousarray(np.asarray(w, dtype=np.float64))
+        if w.shape != (self.info["n_oct_global"],):
+            raise ValueError("w: one value per global octant")
+        n = C.c_int64(0)
+        args = (float(eps_refine), float(eps_coarsen), int(level_min), int(level_max))
+        _check(lib().dgr_regrid_octree(self._h, w.ctypes.data, *args, None, C.byref(n)))
+        out = np.zeros((n.value, 4), dtype=np.uint32)
+        _check(lib().dgr_regrid_octree(self._h, w.ctypes.data, *args, out.ctypes.data,
+                                       C.byref(n)))
+        return out
+
+    def regrid_transfer(self, u, new_mesh, out=None):
+        """dgr_regrid_transfer: the state on new_mesh interpolated from u on this mesh."""
+        if out is None:
+            out = new_mesh.new_state()
+        _check(lib().dgr_regrid_transfer(self._h, self._state(u, "u"), new_mesh._h,
+                                         new_mesh._state(out, "out"), _stream()))
+        return out
+
     def last_launch_count(self):
         return int(lib().dgr_last_launch_count(self._h))
 
@@ -396,6 +449,26 @@ class Mesh:
         n = np.zeros(8, dtype=np.int64)
         _check(lib().dgr_profile_read(self._h, ms.ctypes.data, n.ctypes.data, int(reset)))
         return {PROF_CLASSES[i]: (float(ms[i]), int(n[i])) for i in range(8) if n[i]}
+
+
+N_ALG_IN = 234
+ALG_VARIANTS = ["sympygr_cse", "binary_reduce", "staged_cse"]
+
+
+def rhs_algebra(variant, inp, prm=None, occ=False, out=None):
+    """dgr_rhs_algebra: the generated A kernel `variant` (name or 0..2) on
+    inp [234, n] -> [24, n] (algebra + KO)."""
+    import torch
+    v = ALG_VARIANTS.index(variant) if isinstance(variant, str) else int(variant)
+    n = inp.shape[1]
+    _dev(inp, (N_ALG_IN, n), "inp")
+    if out is None:
+        out = torch.empty((NF, n), dtype=torch.float64, device="cuda")
+    _dev(out, (NF, n), "out")
+    p = (prm or Params())._c()
+    _check(lib().dgr_rhs_algebra(v, int(bool(occ)), _ptr(inp), _ptr(out), n, n, C.byref(p),
+                                 _stream()))
+    return out
 
 
 class Group:

@@ -283,7 +283,7 @@ def kernel(variant, body, bounds):
     return "\n".join(lines)
 
 
-def main():
+def main(out_path=None):
     exprs, syms, prm = bssn_sym.rhs_exprs()
     parts = [HEADER]
     stats = {}
@@ -319,12 +319,14 @@ void launch_rhs_alg(int variant, int occ, const double* in, double* out, int64_t
 
 }  // namespace dgr
 """)
-    os.makedirs(os.path.dirname(OUT), exist_ok=True)
-    with open(OUT, "w") as f:
+    out_path = out_path or OUT
+    os.makedirs(os.path.dirname(out_path), exist_ok=True)
+    with open(out_path, "w") as f:
         f.write("\n".join(parts))
     for v in VARIANTS:
         print(f"{v}: {stats[v]}, {len(bodies[v])} statements")
-    print("wrote", OUT)
+    print("wrote", out_path)
+    return stats
 
 
 if __name__ == "__main__":

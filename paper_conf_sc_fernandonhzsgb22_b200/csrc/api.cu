@@ -590,6 +590,7 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
   lagrange_tables(w13, wext);
   upload_tables(w13, wext);
   upload_rhs_tables(wext);
+  upload_regrid_tables(w13);
   CUDA_TRY(cudaGetLastError());
   DevMesh& dm = m->dm;
   dm.n_owned = int32_t(no);
@@ -1267,6 +1268,108 @@ dgr_status dgr_rhs_algebra(int variant, int occ, const double* in, double* out, 
   const AlgParams ap{rp.eta, rp.lambda_f0, rp.lambda_f1, rp.chi_floor};
   launch_rhs_alg(variant, occ ? 1 : 0, in, out, n, ld, ap, static_cast<cudaStream_t>(stream));
   CUDA_TRY(cudaGetLastError());
+  return DGR_OK;
+}
+
+// ------------------------------------------------------------------ regrid
+dgr_status dgr_regrid_indicator(dgr_mesh m, double* u, uint32_t field_mask, double* w,
+                                void* stream) {
+  dgr_status s = need_device(m);
+  if (s) return s;
+  if (!u || !w || !(field_mask & 0xffffffu)) return fail(DGR_ERR_ARG, "bad regrid_indicator args");
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  m->launches = 0;
+  if ((s = exchange(m, u, st))) return s;
+  if ((s = do_unzip(m, u, NF, st))) return s;
+  PROF(m, 2, st, launch_wavelet(m->dm, m->d_patch, field_mask & 0xffffffu, w, st));
+  CUDA_TRY(cudaGetLastError());
+  return DGR_OK;
+}
+
+dgr_status dgr_regrid_octree(dgr_mesh m, const double* w, double eps_refine, double eps_coarsen,
+                             int level_min, int level_max, dgr_octant* out, int64_t* n_inout) {
+  if (!m || !w || !n_inout) return fail(DGR_ERR_ARG, "null argument");
+  const HostMesh& h = m->host;
+  if (level_min < 0 || level_max > h.D || level_min > level_max || !(eps_coarsen <= eps_refine))
+    return fail(DGR_ERR_ARG, "bad regrid levels or tolerances (eps_coarsen <= eps_refine)");
+  try {
+    std::vector<Oct> o = regrid_leaves(h.oct, w, eps_refine, eps_coarsen, level_min, level_max,
+                                       h.D, h.periodic);
+    if (!out) {
+      *n_inout = int64_t(o.size());
+      return DGR_OK;
+    }
+    if (*n_inout < int64_t(o.size())) return fail(DGR_ERR_ARG, "output buffer too small");
+    for (size_t i = 0; i < o.size(); ++i)
+      out[i] = {uint32_t(o[i].a[0]), uint32_t(o[i].a[1]), uint32_t(o[i].a[2]), uint32_t(o[i].l)};
+    *n_inout = int64_t(o.size());
+    return DGR_OK;
+  } catch (const std::bad_alloc&) {
+    return fail(DGR_ERR_OOM, "host allocation failed");
+  }
+}
+
+dgr_status dgr_regrid_transfer(dgr_mesh old_m, double* u_old, dgr_mesh new_m, double* u_new,
+                               void* stream) {
+  dgr_status s;
+  if ((s = need_device(old_m)) || (s = need_device(new_m))) return s;
+  if (!u_old || !u_new) return fail(DGR_ERR_ARG, "null state");
+  const HostMesh& ho = old_m->host;
+  const HostMesh& hn = new_m->host;
+  if (ho.nranks != 1 || hn.nranks != 1)
+    return fail(DGR_ERR_STATE, "dgr_regrid_transfer: single-rank meshes only");
+  if (ho.D != hn.D || ho.periodic != hn.periodic || ho.width != hn.width ||
+      ho.xmin[0] != hn.xmin[0] || ho.xmin[1] != hn.xmin[1] || ho.xmin[2] != hn.xmin[2])
+    return fail(DGR_ERR_ARG, "meshes of different domains");
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  // new DOF -> (finest old leaf containing it, lowest Morton index on ties;
+  // its half-grid coordinates t2), reading R32
+  const int64_t nd = hn.n_owned_dof;
+  std::vector<int4> map(size_t(std::max<int64_t>(nd, 1)));
+  const int64_t L = ho.L;
+  for (int64_t d = 0; d < nd; ++d) {
+    const int64_t g = hn.dof_gid[d];
+    const int32_t e = hn.zip_leaf[g], n = hn.zip_node[g];
+    const Oct& o = hn.oct[e];
+    const int64_t sn = hn.side(e);
+    const int64_t X[3] = {6 * o.a[0] + (n % 7) * sn, 6 * o.a[1] + ((n / 7) % 7) * sn,
+                          6 * o.a[2] + (n / 49) * sn};
+    int32_t best = -1;
+    for (int q = 0; q < 8; ++q) {
+      int64_t c[3];
+      for (int a = 0; a < 3; ++a) {
+        const int64_t v = 2 * X[a] + (((q >> a) & 1) ? 1 : -1);
+        c[a] = v >= 0 ? v / 12 : -((-v + 11) / 12);   // floor division
+      }
+      const int32_t leaf = ho.locate(c[0], c[1], c[2]);
+      if (leaf < 0) continue;
+      if (best < 0 || ho.oct[leaf].l > ho.oct[best].l ||
+          (ho.oct[leaf].l == ho.oct[best].l && leaf < best))
+        best = leaf;
+    }
+    if (best < 0) return fail(DGR_ERR_TREE, "new DOF outside the old mesh");
+    const int64_t so = ho.side(best);
+    int t2[3];
+    for (int a = 0; a < 3; ++a) {
+      int64_t off = X[a] - 6 * ho.oct[best].a[a];
+      if (ho.periodic) off = ((off % L) + L) % L;
+      if ((2 * off) % so != 0 || 2 * off / so > 12)
+        return fail(DGR_ERR_TREE, "new DOF not on the half-grid of its old element "
+                                  "(levels changed by more than one)");
+      t2[a] = int(2 * off / so);
+    }
+    const int32_t el = ho.g2l_oct[best];
+    map[size_t(d)] = make_int4(el, t2[0] | (t2[1] << 8) | (t2[2] << 16), 0, 0);
+  }
+  int4* d_map = nullptr;
+  CUDA_TRY(cudaMallocAsync(&d_map, map.size() * sizeof(int4), st));
+  CUDA_TRY(cudaMemcpyAsync(d_map, map.data(), map.size() * sizeof(int4), cudaMemcpyHostToDevice, st));
+  old_m->launches = 0;
+  if ((s = do_interp(old_m, u_old, NF, st))) return s;   // hanging-node slots of the old mesh
+  PROF(old_m, 2, st, launch_transfer(old_m->dm, u_old, d_map, nd, u_new, new_m->dm.dof_stride, st));
+  CUDA_TRY(cudaGetLastError());
+  CUDA_TRY(cudaFreeAsync(d_map, st));
+  CUDA_TRY(cudaStreamSynchronize(st));   // the host map is freed on return
   return DGR_OK;
 }
 

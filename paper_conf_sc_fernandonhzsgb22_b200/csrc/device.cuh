@@ -139,6 +139,15 @@ void launch_rhs_alg(int variant, int occ, const double* in, double* out, int64_t
 void launch_rhs_inputs(const DevMesh& m, const double* patches, double* in, int64_t ld,
                        double ko_sigma, cudaStream_t s);
 
+// regrid.cu (readings R30-R32): wavelet indicator per owned octant from the
+// patch buffer (fields in `mask`), and the intergrid transfer of the new
+// mesh's DOFs from the old mesh's element interpolants
+void upload_regrid_tables(const double* w13);
+void launch_wavelet(const DevMesh& m, const double* patches, uint32_t mask, double* w,
+                    cudaStream_t s);
+void launch_transfer(const DevMesh& old, const double* u_old, const int4* map, int64_t n,
+                     double* u_new, int64_t new_stride, cudaStream_t s);
+
 // constraints_kernel.cu
 void launch_constraints(const DevMesh& m, const double* patches, double* c_oct,
                         const RhsParams& p, cudaStream_t s);

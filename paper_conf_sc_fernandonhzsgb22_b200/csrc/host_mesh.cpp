@@ -66,6 +66,9 @@ struct Refiner {
 };
 }  // namespace
 
+std::vector<Oct> balance_internal(std::vector<std::unordered_set<uint64_t>>& I, int D,
+                                  bool periodic);
+
 std::vector<Oct> build_octree(const double xmin[3], double width, int D, bool periodic,
                               int level_min, const std::vector<PunctureDesc>& punct,
                               double rho) {
@@ -96,6 +99,14 @@ std::vector<Oct> build_octree(const double xmin[3], double width, int D, bool pe
       cur.swap(nxt);
     }
   }
+  return balance_internal(I, D, periodic);
+}
+
+// Minimal 2:1 vertex-balance closure of the tree whose internal nodes per
+// level are I, then its leaves in Morton order (shared by the builder and the
+// regrid).
+std::vector<Oct> balance_internal(std::vector<std::unordered_set<uint64_t>>& I, int D,
+                                  bool periodic) {
   int maxl = 0;
   for (int l = 0; l <= D; ++l)
     if (!I[l].empty()) maxl = l + 1;
@@ -156,6 +167,55 @@ std::vector<Oct> build_octree(const double xmin[3], double width, int D, bool pe
     }
   }
   return out;
+}
+
+std::vector<Oct> regrid_leaves(const std::vector<Oct>& leaves, const double* w, double eps_refine,
+                              double eps_coarsen, int level_min, int level_max, int D,
+                              bool periodic) {
+  // reading R31: split leaves above eps_refine (level < level_max),
+  // merge complete families of 8 sibling leaves all below eps_coarsen (level >
+  // level_min, none split), then the minimal balance closure
+  const size_t N = leaves.size();
+  std::vector<uint8_t> split(N, 0), merged(N, 0);
+  for (size_t e = 0; e < N; ++e) split[e] = w[e] > eps_refine && leaves[e].l < level_max;
+  std::vector<Oct> nl;
+  for (size_t e = 0; e < N;) {
+    const Oct& o = leaves[e];
+    const int64_t s = int64_t(1) << (D - o.l);
+    // a family starts at child 0 of its parent: 8 consecutive same-level
+    // leaves (Morton order) with one parent
+    bool fam = o.l > level_min && e + 8 <= N && o.l > 0 &&
+               (o.a[0] & (2 * s - 1)) == 0 && (o.a[1] & (2 * s - 1)) == 0 &&
+               (o.a[2] & (2 * s - 1)) == 0;
+    for (size_t c = 0; fam && c < 8; ++c) {
+      const Oct& q = leaves[e + c];
+      fam = q.l == o.l && q.a[0] == o.a[0] + int64_t(c & 1) * s &&
+            q.a[1] == o.a[1] + int64_t((c >> 1) & 1) * s &&
+            q.a[2] == o.a[2] + int64_t((c >> 2) & 1) * s && !split[e + c] &&
+            w[e + c] < eps_coarsen;
+    }
+    if (fam) {
+      nl.push_back({{o.a[0], o.a[1], o.a[2]}, o.l - 1});
+      e += 8;
+      continue;
+    }
+    if (split[e]) {
+      const int64_t h = s / 2;
+      for (int c = 0; c < 8; ++c)
+        nl.push_back({{o.a[0] + (c & 1) * h, o.a[1] + ((c >> 1) & 1) * h,
+                       o.a[2] + ((c >> 2) & 1) * h}, o.l + 1});
+    } else {
+      nl.push_back(o);
+    }
+    ++e;
+  }
+  std::vector<std::unordered_set<uint64_t>> I(D + 1);
+  for (const Oct& o : nl)
+    for (int l = 0; l < o.l; ++l) {
+      const int64_t s = int64_t(1) << (D - l);
+      I[l].insert(pack((o.a[0] / s) * s, (o.a[1] / s) * s, (o.a[2] / s) * s));
+    }
+  return balance_internal(I, D, periodic);
 }
 
 // --------------------------------------------------------------- HostMesh

@@ -134,4 +134,11 @@ struct PunctureDesc {
 std::vector<Oct> build_octree(const double xmin[3], double width, int D, bool periodic,
                               int level_min, const std::vector<PunctureDesc>& punct, double rho);
 
+// Regrid (readings R30-R32): new leaves from the per-leaf wavelet
+// indicator w (global Morton order) — split above eps_refine, merge complete
+// sibling families below eps_coarsen — then the minimal 2:1 balance closure.
+std::vector<Oct> regrid_leaves(const std::vector<Oct>& leaves, const double* w, double eps_refine,
+                              double eps_coarsen, int level_min, int level_max, int D,
+                              bool periodic);
+
 }  // namespace dgr

@@ -28,9 +28,9 @@ def test_symbolic_algebra_matches_oracle():
     assert err.max() < 1e-12, err
 
 
-def test_generated_file_is_current():
+def test_generated_file_is_current(tmp_path):
     with open(gen.OUT) as fh:
         committed = fh.read()
-    gen.main()
-    with open(gen.OUT) as fh:
-        assert fh.read() == committed, "csrc/gen/rhs_alg.cu differs from the generator's output"
+    out = tmp_path / "rhs_alg.cu"
+    gen.main(str(out))
+    assert out.read_text() == committed, "csrc/gen/rhs_alg.cu differs from the generator's output"

@@ -269,6 +269,41 @@ def test_100_steps_parity(name):
     assert_parity(got, v, 1e-8, f"100 steps {name}")
 
 
+def test_100_steps_amr_golden():
+    """north_star / BASELINE configs[1]: RK4 state after 100 steps on an
+    ADAPTIVE mesh within 1e-8 of the oracle.  small_bbh (q = 2 BBH, levels
+    2..6, 428 octants: hanging chains, coarse-fine interpolation, extrapolated
+    outer boundary), Brill-Lindquist data.  The oracle's 400 RHS evaluations
+    take ~10 min on 8 cores, so its state was computed once by
+    tools/make_golden_amr100.py (calls only oracle/ and synth/) and committed:
+    6,000 seeded sampled DOFs x 24 fields, plus per-field max |u| and RMS over
+    all DOFs.  A perturbation study (profiles/r2_growth_a.txt, bbh_small)
+    shows this setup amplifies a 1e-13 relative perturbation to ~1e-7 over 100
+    steps, so the last-bit differences of two correct implementations stay
+    within the bar; the GPU's per-field errors are printed."""
+    need_gpu()
+    import os as _os
+    g = np.load(_os.path.join(_os.path.dirname(__file__), "golden", "amr100_small_bbh_bl.npz"))
+    cfg = configs.small_bbh(lmax=6, rho=0.5)
+    m = dgr.Mesh(cfg)
+    assert m.info["n_oct_global"] == int(g["n_oct"]) and m.info["n_dof_owned"] == int(g["n_dof"])
+    xyz = m.dof_xyz_host()
+    u0 = initial.for_config(cfg, xyz, kind=str(g["kind"]), seed=int(g["seed"]))
+    ud = to_dev(u0, m.dof_stride)
+    dt = float(g["dt"])
+    for _ in range(int(g["steps"])):
+        m.rk4_step(ud, dt)
+    got = ud[:, :m.info["n_dof_owned"]].cpu().numpy()
+    fmax = g["fmax"]
+    err = np.abs(got[:, g["idx"]] - g["u"]).max(axis=1) / np.maximum(fmax, 1e-300)
+    print("100-step AMR per-field max-abs-relative errors (sampled DOFs):", err)
+    assert np.all(err <= 1e-8), err
+    assert np.all(np.abs(np.abs(got).max(axis=1) - fmax) <= 1e-8 * fmax)
+    rms = np.sqrt((got * got).mean(axis=1))
+    assert np.all(np.abs(rms - g["frms"]) <= 1e-8 * fmax)
+    assert float(g["moved"]) > 1e-3                  # the state really evolved
+
+
 @pytest.mark.parametrize("kind", ["bl", "random"])
 def test_rhs_sommerfeld_parity(kind):
     """Radiative outer boundary (reading R29): the CUDA RHS

@@ -76,7 +76,7 @@ def test_transfer_parity_and_identities():
     fa, fl = octree.sort_morton(fa, fl, om.D)
     fine = dgr.Mesh(cfg, np.concatenate([fa, fl[:, None]], axis=1).astype(np.uint32))
     uf = m.regrid_transfer(ud, fine)
-    back = fine.regrid_octree(np.zeros(fine.info["n_oct_global"]), 1.0, 0.5, 0, 20)
+    back = fine.regrid_octree(np.zeros(fine.info["n_oct_global"]), 1.0, 0.5, 0, 18)
     assert np.array_equal(back, m.octants)
     ub = fine.regrid_transfer(uf, dgr.Mesh(cfg, back))
     assert torch.equal(ub[:, :om.n_dof], ud[:, :om.n_dof])

@@ -183,6 +183,15 @@ def cpu_baseline_oracle(cfg, n_sample=None, reps=1, one_core=True):
     return res
 
 
+def _nccl_summary(path):
+    """Transport facts from NCCL_DEBUG=INFO (rank 0's log)."""
+    if not path or not os.path.exists(path):
+        return None
+    txt = open(path, errors="replace").read()
+    return {"log": path, "nvls": "NVLS" in txt and "NVLS multicast support is not available" not in txt,
+            "p2p_nvlink": "via P2P" in txt, "lines": txt.count("\n")}
+
+
 def run_reference(args, cfg):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
@@ -233,6 +242,13 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    nccl_log = None
+    if world > 1 and "NCCL_DEBUG" not in os.environ:
+        # NCCL's transport choices (NVLink P2P, NVLS) for the JSON line; the log
+        # goes to a file so rank 0's stdout stays one JSON line
+        nccl_log = f"/tmp/dgr_nccl_{os.getpid()}.log"
+        os.environ["NCCL_DEBUG"] = "INFO"
+        os.environ["NCCL_DEBUG_FILE"] = nccl_log
     torch.cuda.set_device(local)
     nccl_id = None
     if world > 1:
@@ -455,6 +471,7 @@ def main():
         "gpu_launches": launches_per_step * args.steps,
         "clocks": clk.summary(),
         "finite": finite,
+        "nccl": _nccl_summary(nccl_log) if world > 1 else None,
     }
     print(json.dumps(line), flush=True)
     if world > 1:

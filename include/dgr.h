@@ -113,7 +113,11 @@ typedef struct {
   int32_t sommerfeld; /* 1: radiative outer boundary at the DOFs on the faces of a
                          non-periodic domain, d_t f = -(x^i/r) d_i f - (f - f_inf)/r
                          (reading R29; PAPER.md is silent); 0: none (default) */
-  int32_t reserved;   /* 0 */
+  int32_t upwind;     /* 1: advective derivatives beta^k d_k f by the 4th-order lopsided
+                         stencil (-3 f_-1 - 10 f_0 + 18 f_1 - 6 f_2 + f_3)/(12 h) shifted
+                         towards +k where beta^k >= 0, mirrored where < 0 (reading R9u,
+                         for long moving-puncture evolutions); 0: centred D1 (R9,
+                         default; the paper's 72 first derivatives) */
 } dgr_params;
 
 typedef struct {

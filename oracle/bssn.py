@@ -10,6 +10,10 @@ readings of DESIGN.md §Readings:
   R6  f(alpha) = lambda_f0 + lambda_f1*alpha (default 1), eta = 2;
   R7  undifferentiated Gt^i in (8) and (17) is CalGt^i = gt^jk Gt^i_jk;
   R13 chi in every division is max(chi, chi_floor);
+  R9u (Params.upwind = 1, for long moving-puncture runs): every advective
+      derivative beta^k d_k f uses the 4th-order lopsided stencil on the side
+      beta^k points to (oracle/fd.py lop_plus / lop_minus) instead of the
+      centred D1 of R9;
   and the Kreiss-Oliger term (R8) is added to every field after the algebra.
 d_t Gt^i in eq (3) is the value of eq (8) before KO is added.
 
@@ -38,6 +42,7 @@ class Params:
     lambda_f1: float = 0.0
     chi_floor: float = 1e-4
     sommerfeld: int = 0        # 1: radiative outer boundary (oracle/boundary.py, R29)
+    upwind: int = 0            # 1: lopsided advective derivatives (R9u)
 
 
 def sym_to_full(v):
@@ -56,7 +61,7 @@ class PointData:
     """Values and FD derivatives of all fields at the interior points of a set
     of patches.  P: [24, n, 13, 13, 13]; h: [n]."""
 
-    def __init__(self, P, h):
+    def __init__(self, P, h, upwind=False):
         hh = np.asarray(h, dtype=np.float64)[:, None, None, None]
         I = fd.interior
         self.alpha = I(P[F_ALPHA])
@@ -87,6 +92,9 @@ class PointData:
         for k in range(3):
             for l in range(3):
                 self.dd_gt[k, l] = sym_to_full(ddg[k, l])                  # [k, l, i, j]
+        # R9u: lopsided advective derivatives beta^k d_k f of every field
+        if upwind:
+            self.adv = np.stack([fd.advect(P[f], self.beta, hh, True) for f in range(NF)])
 
 
 def geometry(d: PointData, prm: Params):
@@ -135,10 +143,17 @@ def algebra(d: PointData, prm: Params):
     ginv, chi, Gam, CalGt = G["ginv"], G["chi"], G["Gam"], G["CalGt"]
     a, K = d.alpha, d.K
     div_beta = np.einsum("kk...->...", d.d_beta)
-    adv = lambda grad_: np.einsum("k...,k...->...", d.beta, grad_)
-    # eq (10) Lie derivative, weight w = -2/3 (reading R5)
-    def lie(T, dT):
-        return (np.einsum("k...,kij...->ij...", d.beta, dT)
+
+    def adv(f, grad_):
+        """beta^k d_k of field f: centred (R9) from its gradient, or lopsided (R9u)"""
+        if prm.upwind:
+            return d.adv[f]
+        return np.einsum("k...,k...->...", d.beta, grad_)
+
+    # eq (10) Lie derivative, weight w = -2/3 (reading R5); f0: field of T_xx
+    def lie(T, dT, f0):
+        bdT = np.stack([adv(f0 + q, dT[:, i, j]) for q, (i, j) in enumerate(SYM)])
+        return (sym_to_full(bdT)
                 + np.einsum("ik...,jk...->ij...", T, d.d_beta)
                 + np.einsum("kj...,ik...->ij...", T, d.d_beta)
                 - (2.0 / 3.0) * T * div_beta)
@@ -148,22 +163,22 @@ def algebra(d: PointData, prm: Params):
     A_up = np.einsum("ik...,jl...,kl...->ij...", ginv, ginv, d.At)   # At^ij
     A_mix = np.einsum("kl...,lj...->kj...", ginv, d.At)               # At^k_j
     out = np.empty((NF,) + a.shape)
-    out[F_ALPHA] = adv(d.d_alpha) - 2.0 * a * K                                   # (1)
+    out[F_ALPHA] = adv(F_ALPHA, d.d_alpha) - 2.0 * a * K                          # (1)
     f_alpha = prm.lambda_f0 + prm.lambda_f1 * a
     for i in range(3):
-        out[F_BETA + i] = np.einsum("j...,j...->...", d.beta, d.d_beta[:, i]) \
+        out[F_BETA + i] = adv(F_BETA + i, d.d_beta[:, i]) \
             + 0.75 * f_alpha * d.B[i]                                             # (2)
-    rhs_gt = lie(d.gt, d.d_gt) - 2.0 * a * d.At                                   # (4)
-    out[F_CHI] = adv(d.d_chi) + (2.0 / 3.0) * d.chi * (a * K - div_beta)          # (5)
-    rhs_At = (lie(d.At, d.d_At) + d.chi * tf(-G["DDa"] + a * G["Ric"])
+    rhs_gt = lie(d.gt, d.d_gt, F_GAM) - 2.0 * a * d.At                            # (4)
+    out[F_CHI] = adv(F_CHI, d.d_chi) + (2.0 / 3.0) * d.chi * (a * K - div_beta)   # (5)
+    rhs_At = (lie(d.At, d.d_At, F_AT) + d.chi * tf(-G["DDa"] + a * G["Ric"])
               + a * (K * d.At - 2.0 * np.einsum("ik...,kj...->ij...", d.At, A_mix)))  # (6)
-    out[F_K] = adv(d.d_K) - G["DDa_tr"] + a * (np.einsum("ij...,ij...->...", d.At, A_up)
+    out[F_K] = adv(F_K, d.d_K) - G["DDa_tr"] + a * (np.einsum("ij...,ij...->...", d.At, A_up)
                                               + K * K / 3.0)                       # (7)
     # (8) from P:L117-119, reading R7
     dd_beta_div = np.einsum("jkk...->j...", d.dd_beta)                   # d_j d_k beta^k
     rhs_Gt = (np.einsum("jk...,jki...->i...", ginv, d.dd_beta)
               + np.einsum("ij...,j...->i...", ginv, dd_beta_div) / 3.0
-              + np.einsum("j...,ji...->i...", d.beta, d.d_Gt)
+              + np.stack([adv(F_GT + i, d.d_Gt[:, i]) for i in range(3)])
               - np.einsum("j...,ji...->i...", CalGt, d.d_beta)
               + (2.0 / 3.0) * CalGt * div_beta
               - 2.0 * np.einsum("ij...,j...->i...", A_up, d.d_alpha)
@@ -173,8 +188,8 @@ def algebra(d: PointData, prm: Params):
     for i in range(3):
         out[F_GT + i] = rhs_Gt[i]
         out[F_B + i] = (rhs_Gt[i] - prm.eta * d.B[i]                               # (3)
-                        + np.einsum("j...,j...->...", d.beta, d.d_B[:, i])
-                        - np.einsum("j...,j...->...", d.beta, d.d_Gt[:, i]))
+                        + adv(F_B + i, d.d_B[:, i])
+                        - adv(F_GT + i, d.d_Gt[:, i]))
     out[F_GAM:F_GAM + 6] = full_to_sym(rhs_gt)
     out[F_AT:F_AT + 6] = full_to_sym(rhs_At)
     return out
@@ -190,7 +205,7 @@ def rhs_patches(P, h, prm: Params, chunk=512):
     for i0 in range(0, n, chunk):
         i1 = min(n, i0 + chunk)
         Pc = P[:, i0:i1]
-        d = PointData(Pc, h[i0:i1])
+        d = PointData(Pc, h[i0:i1], upwind=bool(prm.upwind))
         r = algebra(d, prm)
         hh = h[i0:i1][:, None, None, None]
         for f in range(NF):

@@ -68,6 +68,32 @@ def ko(P, a, h, sigma):
                                    + 15.0 * u(1) - 6.0 * u(2) + u(3))
 
 
+def lop_plus(P, a, h):
+    """4th-order lopsided first derivative shifted towards +a (reading R9u):
+    (-3 u-1 - 10 u0 + 18 u1 - 6 u2 + u3) / (12 h)."""
+    u = lambda s: _sl(P, a, s)
+    return (-3.0 * u(-1) - 10.0 * u(0) + 18.0 * u(1) - 6.0 * u(2) + u(3)) / (12.0 * h)
+
+
+def lop_minus(P, a, h):
+    """Its mirror image, shifted towards -a: (3 u1 + 10 u0 - 18 u-1 + 6 u-2 - u-3) / (12 h)."""
+    u = lambda s: _sl(P, a, s)
+    return (3.0 * u(1) + 10.0 * u(0) - 18.0 * u(-1) + 6.0 * u(-2) - u(-3)) / (12.0 * h)
+
+
+def advect(P, beta, h, upwind):
+    """beta^k d_k u on the interior: centred D1 (reading R9) or, with upwind,
+    the lopsided stencil on the side beta^k points to (beta^k >= 0 -> +k)."""
+    out = 0.0
+    for a in range(3):
+        if upwind:
+            d = np.where(beta[a] >= 0.0, lop_plus(P, a, h), lop_minus(P, a, h))
+        else:
+            d = d1(P, a, h)
+        out = out + beta[a] * d
+    return out
+
+
 def interior(P):
     return P[..., K:K + R, K:K + R, K:K + R]
 

@@ -60,7 +60,7 @@ class _MeshDesc(C.Structure):
 class _Params(C.Structure):
     _fields_ = [("ko_sigma", C.c_double), ("eta", C.c_double), ("lambda_f0", C.c_double),
                 ("lambda_f1", C.c_double), ("chi_floor", C.c_double),
-                ("sommerfeld", C.c_int32), ("reserved", C.c_int32)]
+                ("sommerfeld", C.c_int32), ("upwind", C.c_int32)]
 
 
 class _Info(C.Structure):
@@ -159,10 +159,11 @@ class Params:
     lambda_f1: float = 0.0
     chi_floor: float = 1e-4
     sommerfeld: int = 0   # 1: radiative outer boundary (reading R29)
+    upwind: int = 0       # 1: lopsided advective derivatives (reading R9u)
 
     def _c(self):
         return _Params(self.ko_sigma, self.eta, self.lambda_f0, self.lambda_f1, self.chi_floor,
-                       int(self.sommerfeld), 0)
+                       int(self.sommerfeld), int(self.upwind))
 
 
 def octree_build(cfg) -> np.ndarray:

@@ -897,8 +897,10 @@ static dgr_status do_unzip(dgr_mesh m, const double* u, int nf, cudaStream_t st,
 }
 
 static RhsParams to_rp(const dgr_params* p) {
-  RhsParams r{0.4, 2.0, 1.0, 0.0, 1e-4, 0};
-  if (p) r = {p->ko_sigma, p->eta, p->lambda_f0, p->lambda_f1, p->chi_floor, p->sommerfeld != 0};
+  RhsParams r{0.4, 2.0, 1.0, 0.0, 1e-4, 0, 0};
+  if (p)
+    r = {p->ko_sigma, p->eta, p->lambda_f0, p->lambda_f1, p->chi_floor, p->sommerfeld != 0,
+         p->upwind != 0};
   return r;
 }
 

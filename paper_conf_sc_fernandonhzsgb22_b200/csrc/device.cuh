@@ -109,6 +109,7 @@ void launch_dfma(int blocks, int iters, double* out, cudaStream_t s);
 struct RhsParams {
   double ko_sigma, eta, lambda_f0, lambda_f1, chi_floor;
   int sommerfeld;   // radiative outer boundary (reading R29)
+  int upwind;       // lopsided advective derivatives (reading R9u)
 };
 // fused = false: read 13^3 patches ([24][n_owned][PATCH_PITCH], TMA bulk copies);
 // fused = true: `src` is the state u; every patch is gathered from u and the

@@ -194,6 +194,24 @@ __device__ __forceinline__ Derivs derivs(const double* __restrict__ s, int c, do
   return d;
 }
 
+// advective derivative beta^k d_k f at patch index c: reading R9, the centred
+// D1 (d1 = its values); with upw (dgr_params.upwind, reading R9u) the 4th-order
+// lopsided stencil (-3 f_-1 - 10 f_0 + 18 f_1 - 6 f_2 + f_3) / (12 h) shifted
+// towards +k where beta^k >= 0 and its mirror image where beta^k < 0
+__device__ __forceinline__ double advect(const double* __restrict__ s, int c, const double* beta,
+                                         const double* d1, double ih, int upw) {
+  if (!upw) return beta[0] * d1[0] + beta[1] * d1[1] + beta[2] * d1[2];
+  double a = 0.0;
+#pragma unroll
+  for (int k = 0; k < 3; ++k) {
+    const int st = k == 0 ? 1 : (k == 1 ? 13 : 169);
+    const int q = beta[k] >= 0.0 ? st : -st;
+    const double e = -3.0 * s[c - q] - 10.0 * s[c] + 18.0 * s[c + q] - 6.0 * s[c + 2 * q] + s[c + 3 * q];
+    a += beta[k] * ((beta[k] >= 0.0 ? e : -e) * (ih * (1.0 / 12.0)));
+  }
+  return a;
+}
+
 // D1 of a precomputed D1 field (raw numerators), at patch index c
 __device__ __forceinline__ double d1_of(const double* __restrict__ T, int c, int st) {
   return (T[c + st] - T[c - st]) * 45.0 - (T[c + 2 * st] - T[c - 2 * st]) * 9.0 +
@@ -711,7 +729,7 @@ __global__ void __launch_bounds__(RT, 1)
 #pragma unroll
         for (int k = 0; k < 3; ++k) SL(S0 + k * 6 + q) = d.d1[k];
         SL(A_AT + q) = trace6(gi, d.dd);   // (A_AT slot reused until the Christoffel block)
-        SL(A_GAM + q) += beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
+        SL(A_GAM + q) += advect(s, c0, beta, d.d1, ih, prm.upwind) + d.ko;
         if (q == 5) christoffel(gi);
       } else if (f == 1) {
         // ---------------- chi: advection, KO, R^chi (eq 18-19), eq (8) chi term
@@ -725,7 +743,7 @@ __global__ void __launch_bounds__(RT, 1)
         }
 #pragma unroll
         for (int k = 0; k < 3; ++k) dchi[k] = d.d1[k];
-        rC += beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
+        rC += advect(s, c0, beta, d.d1, ih, prm.upwind) + d.ko;
         double Rc[6];
 #pragma unroll
         for (int i = 0; i < 3; ++i)
@@ -764,7 +782,7 @@ __global__ void __launch_bounds__(RT, 1)
           gt[r] = SL(V_GAM + r);
         }
         const double* da = d.d1;
-        rA += beta[0] * da[0] + beta[1] * da[1] + beta[2] * da[2] + d.ko;
+        rA += advect(s, c0, beta, da, ih, prm.upwind) + d.ko;
         // gt^kl d_l chi d_k alpha
         double gdd = 0.0;
 #pragma unroll
@@ -802,7 +820,7 @@ __global__ void __launch_bounds__(RT, 1)
         // ---------------- Gt^k: Ricci d Gt term, advection + KO kept apart (eq 3)
         const int kk = f - 3;
         const Derivs d = derivs<false>(s, c0, ih, ko_scale);
-        SL(S0 + kk) = beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
+        SL(S0 + kk) = advect(s, c0, beta, d.d1, ih, prm.upwind) + d.ko;
         double gi[6], gt[6], Rg[6];
 #pragma unroll
         for (int r = 0; r < 6; ++r) {
@@ -829,7 +847,7 @@ __global__ void __launch_bounds__(RT, 1)
         const int kk = f - 6;
         const Derivs d = derivs2(s, Tx, Ty, c0, ih, ko_scale);
         const double* db = d.d1;   // d_j beta^kk
-        SL(A_BETA + kk) += beta[0] * db[0] + beta[1] * db[1] + beta[2] * db[2] + d.ko;
+        SL(A_BETA + kk) += advect(s, c0, beta, db, ih, prm.upwind) + d.ko;
         double gi[6], cal[3];
 #pragma unroll
         for (int r = 0; r < 6; ++r) gi[r] = SL(G_INV + r);
@@ -883,7 +901,7 @@ __global__ void __launch_bounds__(RT, 1)
       } else if (f == 2) {
         // ---------------- K: advection, KO, eq (8) -4/3 alpha gt^ij d_j K
         const Derivs d = derivs<false>(s, c0, ih, ko_scale);
-        rK += beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
+        rK += advect(s, c0, beta, d.d1, ih, prm.upwind) + d.ko;
         double gi[6];
 #pragma unroll
         for (int r = 0; r < 6; ++r) gi[r] = SL(G_INV + r);
@@ -895,11 +913,11 @@ __global__ void __launch_bounds__(RT, 1)
       } else if (f >= 18) {
         const int q = f - 18;
         const Derivs d = derivs<false>(s, c0, ih, ko_scale);
-        SL(A_AT + q) += beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
+        SL(A_AT + q) += advect(s, c0, beta, d.d1, ih, prm.upwind) + d.ko;
       } else {  // 9..11: B
         const int kk = f - 9;
         const Derivs d = derivs<false>(s, c0, ih, ko_scale);
-        SL(A_B + kk) = beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko;
+        SL(A_B + kk) = advect(s, c0, beta, d.d1, ih, prm.upwind) + d.ko;
       }
     }
     __syncthreads();  // everyone is done with this stage buffer
@@ -1204,7 +1222,7 @@ __global__ void __launch_bounds__(RT, 2)
 #pragma unroll
         for (int k = 0; k < 3; ++k) st_out(&out[(6 * k + q) * ostr], d.d1[k]);
         st_out(&out[(18 + q) * ostr], trace6(gi, d.dd));
-        st_out(&out[(24 + q) * ostr], beta[0] * d.d1[0] + beta[1] * d.d1[1] + beta[2] * d.d1[2] + d.ko);
+        st_out(&out[(24 + q) * ostr], advect(s, c0, beta, d.d1, ih, prm.upwind) + d.ko);
       }
     }
   }

@@ -174,3 +174,68 @@ def test_fd_weights_golden():
     assert w1 == g["d1_times_60"]
     assert w2 == g["d2_times_180"]
     assert wk == g["ko_times_64h_over_sigma"]
+
+
+# ------------------------------------------------ lopsided advection (R9u)
+
+def test_lopsided_stencils_exact_to_degree4_and_upwind_side():
+    """oracle.fd.lop_plus / lop_minus (reading R9u): exact first derivative of
+    polynomials of degree <= 4 (4th order), first error at x^5 with the
+    closed-form coefficient; the plus stencil reads offsets -1..3 only (a
+    perturbation at -2 or -3 leaves it unchanged), the minus one -3..1; and
+    fd.advect picks the side by the sign of beta^a."""
+    from oracle import fd as _fd
+    h = 0.125
+    z = np.arange(13) - 6.0                         # patch index -> x / h, interior centre at 0
+    X = np.broadcast_to((z * h)[None, None, :], (13, 13, 13)).copy()
+    for deg in range(5):
+        P = X ** deg
+        want = deg * X[3:10, 3:10, 3:10] ** max(deg - 1, 0) if deg else 0 * X[3:10, 3:10, 3:10]
+        assert np.abs(_fd.lop_plus(P, 0, h) - want).max() < 1e-12
+        assert np.abs(_fd.lop_minus(P, 0, h) - want).max() < 1e-12
+    # x^5 at x = 0: plus (-3(-1) - 0 + 18 - 6*32 + 243)/12 h^4 = 6 h^4; minus
+    # (3 + 0 + 18 - 6*32 + 243)/12 h^4 = 6 h^4 (odd function, mirrored stencil)
+    P = X ** 5
+    c = (6, 6)
+    assert abs(_fd.lop_plus(P, 0, h)[c + (3,)] - 6.0 * h ** 4) < 1e-12
+    assert abs(_fd.lop_minus(P, 0, h)[c + (3,)] - 6.0 * h ** 4) < 1e-12
+    Q = np.zeros((13, 13, 13))
+    Q[:, :, 6 - 2] = 1.0                            # offset -2 of interior point x = 3 (index 6)
+    assert _fd.lop_plus(Q, 0, h)[:, :, 3].max() == 0.0
+    assert _fd.lop_minus(Q, 0, h)[:, :, 3].max() != 0.0
+    rng = np.random.default_rng(0)
+    U = rng.standard_normal((13, 13, 13))
+    beta = np.stack([np.where(rng.uniform(size=(7, 7, 7)) > 0.5, 1.0, -1.0) * 0.3,
+                     np.zeros((7, 7, 7)), np.zeros((7, 7, 7))])
+    got = _fd.advect(U, beta, h, True)
+    want = beta[0] * np.where(beta[0] >= 0, _fd.lop_plus(U, 0, h), _fd.lop_minus(U, 0, h))
+    assert np.array_equal(got, want)
+    assert np.array_equal(_fd.advect(U, beta, h, False), beta[0] * _fd.d1(U, 0, h))
+
+
+def test_upwind_rhs_reduces_to_centred_where_fields_are_linear():
+    """With every field linear in x (lopsided and centred stencils are both exact
+    on degree <= 1, up to rounding), the upwind RHS equals the centred one; on
+    generic data they differ."""
+    from oracle import bssn as _b, rk4 as _rk4
+    from oracle.maps import OracleMesh
+    from oracle.unzip import unzip
+    from synth.configs import MeshConfig
+    cfg = MeshConfig(name="lin", xmin=(-1, -1, -1), width=2.0, periodic=False, level_min=1)
+    m = OracleMesh(cfg)
+    m.build_dofs()
+    x = m.dof_coords()
+    rng = np.random.default_rng(3)
+    a, b = rng.uniform(-0.1, 0.1, 24), rng.uniform(-0.05, 0.05, (24, 3))
+    base = np.zeros(24)
+    base[[0, 1, 12, 15, 17]] = 1.0
+    u = base[:, None] + a[:, None] + b @ x
+    P = unzip(m, u)
+    h = _rk4.octant_h(m)
+    r0 = _b.rhs_patches(P, h, _b.Params(ko_sigma=0.0))
+    r1 = _b.rhs_patches(P, h, _b.Params(ko_sigma=0.0, upwind=1))
+    assert np.abs(r1 - r0).max() < 1e-12 * (1 + np.abs(r0).max())
+    u2 = u + 0.05 * np.sin(3.0 * x[0])[None, :]
+    P2 = unzip(m, u2)
+    d = np.abs(_b.rhs_patches(P2, h, _b.Params(upwind=1)) - _b.rhs_patches(P2, h, _b.Params()))
+    assert d.max() > 1e-6

@@ -7,7 +7,8 @@ lapse minimum sampled along the run.
     python tools/long_run.py [t_end=100] [samples=20]
 Environment: DGR_SIGMA (KO strength, 0.4), DGR_ETA (2.0), DGR_CFL (0.25),
 DGR_BC ("both" | "somm" | "extrap"), DGR_LMAX (finest level, 8),
-DGR_PUNCT ("c2": offset h/4 in z as in synth.configs; "cell": at a cell centre).
+DGR_PUNCT ("c2": offset h/4 in z as in synth.configs; "cell": at a cell centre),
+DGR_UPWIND (1: lopsided advective derivatives, reading R9u).
 """
 import os
 import sys
@@ -44,7 +45,8 @@ far = torch.from_numpy(r > 24.0).cuda()           # outer region (boundary at 32
 print(f"C2: {m.info['n_oct_global']} octants, {n} DOFs, dt = {dt:.5f}, {steps} steps to t = {t_end}, "
       f"KO sigma {sigma}, eta {eta}")
 for somm in bcs:
-    prm = dgr.Params(sommerfeld=somm, ko_sigma=sigma, eta=eta)
+    prm = dgr.Params(sommerfeld=somm, ko_sigma=sigma, eta=eta,
+                     upwind=int(os.environ.get("DGR_UPWIND", "0")))
     u = torch.zeros((24, m.dof_stride), dtype=torch.float64, device="cuda")
     u[:, :n] = torch.from_numpy(u0)
     print(f"--- outer boundary: {'Sommerfeld (R29)' if somm else 'extrapolation (R12)'}")

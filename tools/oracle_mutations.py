@@ -19,23 +19,23 @@ B = "oracle/bssn.py"
 C = "oracle/constraints.py"
 MUTATIONS = [
     # eq (1)
-    (B, 'out[F_ALPHA] = adv(d.d_alpha) - 2.0 * a * K', 'out[F_ALPHA] = - 2.0 * a * K', "eq1 drop advection"),
-    (B, 'out[F_ALPHA] = adv(d.d_alpha) - 2.0 * a * K', 'out[F_ALPHA] = adv(d.d_alpha) + 2.0 * a * K', "eq1 sign of 2aK"),
+    (B, 'out[F_ALPHA] = adv(F_ALPHA, d.d_alpha) - 2.0 * a * K', 'out[F_ALPHA] = - 2.0 * a * K', "eq1 drop advection"),
+    (B, 'out[F_ALPHA] = adv(F_ALPHA, d.d_alpha) - 2.0 * a * K', 'out[F_ALPHA] = adv(F_ALPHA, d.d_alpha) + 2.0 * a * K', "eq1 sign of 2aK"),
     # eq (2)
-    (B, 'd.beta, d.d_beta[:, i])', 'd.beta, d.d_beta[i, :])', "eq2 transposed self-advection"),
+    (B, 'adv(F_BETA + i, d.d_beta[:, i])', 'adv(F_BETA + i, d.d_beta[i, :])', "eq2 transposed self-advection"),
     (B, '+ 0.75 * f_alpha * d.B[i]', '+ 0.5 * f_alpha * d.B[i]', "eq2 3/4 -> 1/2"),
     # eq (3)
     (B, 'out[F_B + i] = (rhs_Gt[i] - prm.eta', 'out[F_B + i] = (- prm.eta', "eq3 drop d_t Gt"),
-    (B, '- np.einsum("j...,j...->...", d.beta, d.d_Gt[:, i]))', ')', "eq3 drop -beta.grad Gt"),
-    (B, '+ np.einsum("j...,j...->...", d.beta, d.d_B[:, i])', '', "eq3 drop beta.grad B"),
-    (B, 'd.beta, d.d_B[:, i])', 'd.beta, d.d_B[i, :])', "eq3 transposed beta.grad B"),
+    (B, '- adv(F_GT + i, d.d_Gt[:, i]))', ')', "eq3 drop -beta.grad Gt"),
+    (B, '+ adv(F_B + i, d.d_B[:, i])', '', "eq3 drop beta.grad B"),
+    (B, 'adv(F_B + i, d.d_B[:, i])', 'adv(F_B + i, d.d_B[i, :])', "eq3 transposed beta.grad B"),
     # eq (4), Lie derivative
     (B, '- (2.0 / 3.0) * T * div_beta)', '- (0.0 / 3.0) * T * div_beta)', "eq10 weight 0"),
     (B, '+ np.einsum("ik...,jk...->ij...", T, d.d_beta)', '+ np.einsum("ik...,kj...->ij...", T, d.d_beta)', "eq10 transposed d beta"),
     (B, 'rhs_gt = lie(d.gt, d.d_gt) - 2.0 * a * d.At', 'rhs_gt = lie(d.gt, d.d_gt) + 2.0 * a * d.At', "eq4 sign of 2 a At"),
     # eq (5)
     (B, '(2.0 / 3.0) * d.chi * (a * K - div_beta)', '(2.0 / 3.0) * d.chi * (a * K + div_beta)', "eq5 sign div beta"),
-    (B, 'out[F_CHI] = adv(d.d_chi) +', 'out[F_CHI] = 0.0 +', "eq5 drop advection"),
+    (B, 'out[F_CHI] = adv(F_CHI, d.d_chi) +', 'out[F_CHI] = 0.0 +', "eq5 drop advection"),
     # eq (6)
     (B, 'd.chi * tf(-G["DDa"] + a * G["Ric"])', 'd.chi * tf(G["DDa"] + a * G["Ric"])', "eq6 sign DDa"),
     (B, 'd.chi * tf(-G["DDa"] + a * G["Ric"])', 'd.chi * (-G["DDa"] + a * G["Ric"])', "eq6 drop trace-free"),
@@ -43,12 +43,12 @@ MUTATIONS = [
         '+ a * (K * d.At - 1.0 * np.einsum("ik...,kj...->ij...", d.At, A_mix)))', "eq6 2 AA -> 1 AA"),
     (B, 'return T - d.gt * tr / 3.0', 'return T - d.gt * tr / 2.0', "eq11 1/3 -> 1/2"),
     # eq (7)
-    (B, 'out[F_K] = adv(d.d_K) - G["DDa_tr"]', 'out[F_K] = adv(d.d_K) + G["DDa_tr"]', "eq7 sign DDa_tr"),
+    (B, 'out[F_K] = adv(F_K, d.d_K) - G["DDa_tr"]', 'out[F_K] = adv(F_K, d.d_K) + G["DDa_tr"]', "eq7 sign DDa_tr"),
     (B, '+ K * K / 3.0)', '+ K * K / 2.0)', "eq7 K^2/3 -> K^2/2"),
     # eq (8)
     (B, 'rhs_Gt = (np.einsum("jk...,jki...->i...", ginv, d.dd_beta)', 'rhs_Gt = (0.0', "eq8 drop laplacian beta"),
     (B, '+ np.einsum("ij...,j...->i...", ginv, dd_beta_div) / 3.0', '+ np.einsum("ij...,j...->i...", ginv, dd_beta_div) / 6.0', "eq8 1/3 -> 1/6"),
-    (B, '+ np.einsum("j...,ji...->i...", d.beta, d.d_Gt)', '+ np.einsum("j...,ij...->i...", d.beta, d.d_Gt)', "eq8 transposed beta.grad Gt"),
+    (B, '+ np.stack([adv(F_GT + i, d.d_Gt[:, i]) for i in range(3)])', '+ np.stack([adv(F_GT + i, d.d_Gt[i, :]) for i in range(3)])', "eq8 transposed beta.grad Gt"),
     (B, '- np.einsum("j...,ji...->i...", CalGt, d.d_beta)', '+ np.einsum("j...,ji...->i...", CalGt, d.d_beta)', "eq8 sign CalGt d beta"),
     (B, '+ (2.0 / 3.0) * CalGt * div_beta', '- (2.0 / 3.0) * CalGt * div_beta', "eq8 sign CalGt div beta"),
     (B, '- 2.0 * np.einsum("ij...,j...->i...", A_up, d.d_alpha)', '+ 2.0 * np.einsum("ij...,j...->i...", A_up, d.d_alpha)', "eq8 sign At d alpha"),

@@ -198,9 +198,10 @@ __device__ __forceinline__ Derivs derivs(const double* __restrict__ s, int c, do
 // D1 (d1 = its values); with upw (dgr_params.upwind, reading R9u) the 4th-order
 // lopsided stencil (-3 f_-1 - 10 f_0 + 18 f_1 - 6 f_2 + f_3) / (12 h) shifted
 // towards +k where beta^k >= 0 and its mirror image where beta^k < 0
+template <bool UPW>
 __device__ __forceinline__ double advect(const double* __restrict__ s, int c, const double* beta,
-                                         const double* d1, double ih, int upw) {
-  if (!upw) return beta[0] * d1[0] + beta[1] * d1[1] + beta[2] * d1[2];
+                                         const double* d1, double ih) {
+  if (!UPW) return beta[0] * d1[0] + beta[1] * d1[1] + beta[2] * d1[2];
   double a = 0.0;
 #pragma unroll
   for (int k = 0; k < 3; ++k) {
@@ -295,7 +296,8 @@ __device__ __forceinline__ void at_up_w(const double* gi, const double* At, cons
 // the same arithmetic as k_unzip.
 // SOMM: radiative outer boundary (reading R29) compiled in (a separate
 // instantiation, so the default path carries none of its registers).
-template <bool FUSED, bool SOMM, bool PRE>
+// UPW: lopsided advective derivatives (reading R9u, dgr_params.upwind) compiled in
+template <bool FUSED, bool SOMM, bool PRE, bool UPW>
 __global__ void __launch_bounds__(RT, 1)
     k_rhs(DevMesh m, const double* __restrict__ patches, double* __restrict__ rhs_oct,
           RhsParams prm, int first, int count, const double* __restrict__ pre,
@@ -729,7 +731,7 @@ __global__ void __launch_bounds__(RT, 1)
 #pragma unroll
         for (int k = 0; k < 3; ++k) SL(S0 + k * 6 + q) = d.d1[k];
         SL(A_AT + q) = trace6(gi, d.dd);   // (A_AT slot reused until the Christoffel block)
-        SL(A_GAM + q) += advect(s, c0, beta, d.d1, ih, prm.upwind) + d.ko;
+        SL(A_GAM + q) += advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
         if (q == 5) christoffel(gi);
       } else if (f == 1) {
         // ---------------- chi: advection, KO, R^chi (eq 18-19), eq (8) chi term
@@ -743,7 +745,7 @@ __global__ void __launch_bounds__(RT, 1)
         }
 #pragma unroll
         for (int k = 0; k < 3; ++k) dchi[k] = d.d1[k];
-        rC += advect(s, c0, beta, d.d1, ih, prm.upwind) + d.ko;
+        rC += advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
         double Rc[6];
 #pragma unroll
         for (int i = 0; i < 3; ++i)
@@ -782,7 +784,7 @@ __global__ void __launch_bounds__(RT, 1)
           gt[r] = SL(V_GAM + r);
         }
         const double* da = d.d1;
-        rA += advect(s, c0, beta, da, ih, prm.upwind) + d.ko;
+        rA += advect<UPW>(s, c0, beta, da, ih) + d.ko;
         // gt^kl d_l chi d_k alpha
         double gdd = 0.0;
 #pragma unroll
@@ -820,7 +822,7 @@ __global__ void __launch_bounds__(RT, 1)
         // ---------------- Gt^k: Ricci d Gt term, advection + KO kept apart (eq 3)
         const int kk = f - 3;
         const Derivs d = derivs<false>(s, c0, ih, ko_scale);
-        SL(S0 + kk) = advect(s, c0, beta, d.d1, ih, prm.upwind) + d.ko;
+        SL(S0 + kk) = advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
         double gi[6], gt[6], Rg[6];
 #pragma unroll
         for (int r = 0; r < 6; ++r) {
@@ -847,7 +849,7 @@ __global__ void __launch_bounds__(RT, 1)
         const int kk = f - 6;
         const Derivs d = derivs2(s, Tx, Ty, c0, ih, ko_scale);
         const double* db = d.d1;   // d_j beta^kk
-        SL(A_BETA + kk) += advect(s, c0, beta, db, ih, prm.upwind) + d.ko;
+        SL(A_BETA + kk) += advect<UPW>(s, c0, beta, db, ih) + d.ko;
         double gi[6], cal[3];
 #pragma unroll
         for (int r = 0; r < 6; ++r) gi[r] = SL(G_INV + r);
@@ -901,7 +903,7 @@ __global__ void __launch_bounds__(RT, 1)
       } else if (f == 2) {
         // ---------------- K: advection, KO, eq (8) -4/3 alpha gt^ij d_j K
         const Derivs d = derivs<false>(s, c0, ih, ko_scale);
-        rK += advect(s, c0, beta, d.d1, ih, prm.upwind) + d.ko;
+        rK += advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
         double gi[6];
 #pragma unroll
         for (int r = 0; r < 6; ++r) gi[r] = SL(G_INV + r);
@@ -913,11 +915,11 @@ __global__ void __launch_bounds__(RT, 1)
       } else if (f >= 18) {
         const int q = f - 18;
         const Derivs d = derivs<false>(s, c0, ih, ko_scale);
-        SL(A_AT + q) += advect(s, c0, beta, d.d1, ih, prm.upwind) + d.ko;
+        SL(A_AT + q) += advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
       } else {  // 9..11: B
         const int kk = f - 9;
         const Derivs d = derivs<false>(s, c0, ih, ko_scale);
-        SL(A_B + kk) = advect(s, c0, beta, d.d1, ih, prm.upwind) + d.ko;
+        SL(A_B + kk) = advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
       }
     }
     __syncthreads();  // everyone is done with this stage buffer
@@ -1046,6 +1048,7 @@ constexpr size_t PRE_SMEM_BYTES = size_t(PRE_NBUF) * STAGE_DBL * 8 + size_t(TX_N
 // ring: the CTA barrier that releases stage g's data also proves every thread
 // is done with stage g-1, whose buffer then receives stage g+2 (two stages of
 // latency cover, two barriers per field).
+template <bool UPW>
 __global__ void __launch_bounds__(RT, 2)
     k_gt_pre(DevMesh m, const double* __restrict__ patches, double* __restrict__ pre,
              RhsParams prm, int first, int count) {
@@ -1222,7 +1225,7 @@ __global__ void __launch_bounds__(RT, 2)
 #pragma unroll
         for (int k = 0; k < 3; ++k) st_out(&out[(6 * k + q) * ostr], d.d1[k]);
         st_out(&out[(18 + q) * ostr], trace6(gi, d.dd));
-        st_out(&out[(24 + q) * ostr], advect(s, c0, beta, d.d1, ih, prm.upwind) + d.ko);
+        st_out(&out[(24 + q) * ostr], advect<UPW>(s, c0, beta, d.d1, ih) + d.ko);
       }
     }
   }
@@ -1262,6 +1265,26 @@ void upload_rhs_tables(const double* wext) {
   cudaMemcpyToSymbol(g_perm, perm, sizeof(perm));
 }
 
+template <bool U>
+static void launch_rhs_t(const DevMesh& m, const double* patches, double* rhs_oct,
+                         const RhsParams& p, bool fused, bool somm, int a, int c, int grid,
+                         int64_t cap, cudaStream_t s, double* pre, double* rhs_dof) {
+  if (fused && pre && !somm) {
+    // metric pre-pass (two CTAs per SM), then the 18 remaining fields
+    const int64_t cap2 = 2 * cap;
+    const int grid2 = int(c < cap2 ? c : cap2);
+    k_gt_pre<U><<<grid2, RT, PRE_SMEM_BYTES, s>>>(m, patches, pre, p, a, c);
+    k_rhs<true, false, true, U><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, pre, rhs_dof);
+  } else if (fused && !somm)
+    k_rhs<true, false, false, U><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr, rhs_dof);
+  else if (fused)
+    k_rhs<true, true, false, U><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr, nullptr);
+  else if (!somm)
+    k_rhs<false, false, false, U><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr, nullptr);
+  else
+    k_rhs<false, true, false, U><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr, nullptr);
+}
+
 void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const RhsParams& p,
                 bool fused, int64_t first, int64_t count, int leave_sm, cudaStream_t s,
                 double* pre, double* rhs_dof) {
@@ -1269,12 +1292,17 @@ void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const 
   static std::atomic<bool> done[MAX_DEVICES];
   if (first_on_device(done)) {
     const int sb = int(SMEM_BYTES);
-    cudaFuncSetAttribute(k_rhs<false, false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb);
-    cudaFuncSetAttribute(k_rhs<true, false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb);
-    cudaFuncSetAttribute(k_rhs<false, true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb);
-    cudaFuncSetAttribute(k_rhs<true, true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb);
-    cudaFuncSetAttribute(k_rhs<true, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb);
-    cudaFuncSetAttribute(k_gt_pre, cudaFuncAttributeMaxDynamicSharedMemorySize,
+#define DGR_ATTR(F, S, P, U) \
+    cudaFuncSetAttribute(k_rhs<F, S, P, U>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb);
+    DGR_ATTR(false, false, false, false) DGR_ATTR(true, false, false, false)
+    DGR_ATTR(false, true, false, false) DGR_ATTR(true, true, false, false)
+    DGR_ATTR(true, false, true, false) DGR_ATTR(false, false, false, true)
+    DGR_ATTR(true, false, false, true) DGR_ATTR(false, true, false, true)
+    DGR_ATTR(true, true, false, true) DGR_ATTR(true, false, true, true)
+#undef DGR_ATTR
+    cudaFuncSetAttribute(k_gt_pre<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         int(PRE_SMEM_BYTES));
+    cudaFuncSetAttribute(k_gt_pre<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          int(PRE_SMEM_BYTES));
   }
   const int n_sm = sm_count();
@@ -1283,20 +1311,10 @@ void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const 
   const int grid = int(count < cap ? count : cap);
   const bool somm = p.sommerfeld && !m.periodic;
   const int a = int(first), c = int(count);
-  if (fused && pre && !somm) {
-    // metric pre-pass (two CTAs per SM), then the 18 remaining fields
-    const int64_t cap2 = 2 * cap;
-    const int grid2 = int(count < cap2 ? count : cap2);
-    k_gt_pre<<<grid2, RT, PRE_SMEM_BYTES, s>>>(m, patches, pre, p, a, c);
-    k_rhs<true, false, true><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, pre, rhs_dof);
-  } else if (fused && !somm)
-    k_rhs<true, false, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr, rhs_dof);
-  else if (fused)
-    k_rhs<true, true, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr, nullptr);
-  else if (!somm)
-    k_rhs<false, false, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr, nullptr);
+  if (p.upwind)
+    launch_rhs_t<true>(m, patches, rhs_oct, p, fused, somm, a, c, grid, cap, s, pre, rhs_dof);
   else
-    k_rhs<false, true, false><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr, nullptr);
+    launch_rhs_t<false>(m, patches, rhs_oct, p, fused, somm, a, c, grid, cap, s, pre, rhs_dof);
 }
 
 }  // namespace dgr

@@ -280,9 +280,9 @@ def test_rhs_upwind_parity(kind):
     om = OracleMesh(cfg)
     om.build_dofs()
     u = initial.for_config(cfg, om.dof_coords(), kind=kind, seed=6)
-    if kind == "bl":      # give the shift both signs (BL data have beta = 0)
+    if kind == "bl":      # give the shift both signs and every gradient (BL: beta = 0)
         x = om.dof_coords()
-        u[6:9] = 0.2 * np.sin(x / 3.0 + np.arange(3)[:, None])
+        u[6:9] = 0.2 * np.sin((x[0] + 2.0 * x[1] - x[2]) / 3.0 + np.arange(3)[:, None])
     m = dgr.Mesh(cfg)
     ud = to_dev(u, m.dof_stride)
     prm = obssn.Params(upwind=1)

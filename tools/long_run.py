@@ -8,7 +8,8 @@ lapse minimum sampled along the run.
 Environment: DGR_SIGMA (KO strength, 0.4), DGR_ETA (2.0), DGR_CFL (0.25),
 DGR_BC ("both" | "somm" | "extrap"), DGR_LMAX (finest level, 8),
 DGR_PUNCT ("c2": offset h/4 in z as in synth.configs; "cell": at a cell centre),
-DGR_UPWIND (1: lopsided advective derivatives, reading R9u).
+DGR_UPWIND (1: lopsided advective derivatives, reading R9u), DGR_RHO (refinement
+radius factor of the mesh rule, 1.0).
 """
 import os
 import sys
@@ -26,7 +27,7 @@ samples = int(sys.argv[2]) if len(sys.argv) > 2 else 20
 import dataclasses
 from synth.configs import Puncture
 lmax = int(os.environ.get("DGR_LMAX", "8"))
-cfg = configs.c2_schwarzschild(lmax=lmax)
+cfg = configs.c2_schwarzschild(rho=float(os.environ.get("DGR_RHO", "1.0")), lmax=lmax)
 if os.environ.get("DGR_PUNCT", "c2") == "cell":
     hh = cfg.width / (6.0 * (1 << lmax))
     cfg = dataclasses.replace(cfg, punctures=(Puncture(hh / 2, hh / 2, hh / 2, 1.0, lmax),))

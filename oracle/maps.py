@@ -15,7 +15,14 @@ neighbour map; readings R14-R17 in DESIGN.md):
   sight.  Since a DOF is a node of every leaf containing it, the first leaf
   that sees it is the lowest-index leaf containing it.
 * Hanging source: the coarser leaf containing X, lowest Morton index on ties.
-* Zip owner of a DOF: the finest leaf containing it, lowest index on ties.
+* Zip owner of a DOF: the COARSEST leaf containing it, lowest index on ties
+  (reading R17, round 2: with the finest leaf as owner, the value of a node
+  shared by a coarse and a fine leaf is updated from the fine leaf's
+  stencil, whose padding is interpolated from the coarse leaf's values at
+  that node, a feedback loop that makes moving-puncture runs blow up at
+  every refinement interface the gauge pulse crosses; with the coarsest
+  leaf the shared node is updated from the coarse stencil, which reads the
+  fine side by injection: DESIGN.md §8b, profiles/r2_long_run_*).
 * Padding source of patch point x of octant b: the finest leaf TOUCHING b whose
   closed box contains x, lowest index on ties; kind = copy (same level),
   inject (source finer), interp (source coarser); points outside a
@@ -127,7 +134,7 @@ class OracleMesh:
             fst = np.full(M, np.iinfo(np.int64).max)
             hs = np.full(M, np.iinfo(np.int64).max)
             own = np.full(M, -1, dtype=np.int64)
-            own_lvl = np.full(M, -1, dtype=np.int64)
+            own_lvl = np.full(M, np.iinfo(np.int64).max, dtype=np.int64)
             for q in range(8):
                 c = cont[:, q]
                 ok = c >= 0
@@ -138,7 +145,7 @@ class OracleMesh:
                 coarser = ok & (self.levels[cc] < self.levels[ee])
                 hs = np.where(coarser, np.minimum(hs, cc), hs)
                 lv = self.levels[cc]
-                better = ok & ((lv > own_lvl) | ((lv == own_lvl) & (cc < own)))
+                better = ok & ((lv < own_lvl) | ((lv == own_lvl) & (cc < own)))
                 own = np.where(better, cc, own)
                 own_lvl = np.where(better, lv, own_lvl)
             sl = (slice(e0, e1), bidx)

@@ -201,7 +201,7 @@ def _extrapolate(mesh: OracleMesh, P, octs):
 
 def zip_rhs(mesh: OracleMesh, rhs_oct: np.ndarray) -> np.ndarray:
     """Patch-to-octant: DOF value = the owner octant's interior value
-    (zip owner: finest containing leaf, lowest index; reading R17).
+    (zip owner: coarsest containing leaf, lowest index; reading R17).
     rhs_oct: [nf, n_oct, 343] -> [nf, n_dof]."""
     mesh.build_dofs()
     return rhs_oct[:, mesh.zip_leaf, mesh.zip_node]

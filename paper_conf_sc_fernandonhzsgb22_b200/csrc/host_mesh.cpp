@@ -357,6 +357,7 @@ struct NodeInfo {
 // the node grid of every leaf whose closed box contains it.
 void HostMesh::classify_nodes() {
   const int64_t N = int64_t(oct.size());
+
   std::vector<NodeInfo> info(size_t(N) * NPT);
   std::vector<int32_t> n_new(N, 0);
   int bad = 0;
@@ -405,7 +406,11 @@ void HostMesh::classify_nodes() {
           hsrc = t.leaf;
           std::memcpy(hsh, t.sh, sizeof(hsh));
         }
-        if (c.l > own_l || (c.l == own_l && t.leaf < own)) {
+        // zip owner (reading R17): the coarsest containing leaf, lowest index
+        // on ties — a shared coarse/fine node is updated from the coarse
+        // stencil (the finest-owner rule feeds the coarse->fine padding
+        // interpolation back into the node and is unstable)
+        if (c.l < own_l || (c.l == own_l && t.leaf < own)) {
           own = t.leaf;
           own_l = c.l;
         }

@@ -115,6 +115,21 @@ def small_bbh(lmax: int = 6, rho: float = 0.5) -> MeshConfig:
     return _bbh("small_bbh", 2.0, lmax - 1, lmax, rho, "small q=2 BBH", level_min=2, width=32.0)
 
 
+def c3_large() -> MeshConfig:
+    """configs[2] at the Fig. 17 caption size: BL q=1, levels 3..12, rho = 3.4
+    (~257M unknowns; reading R22)."""
+    c = c3_bbh_q1(rho=3.4)
+    return MeshConfig(**{**c.__dict__, "name": "c3big"})
+
+
+def table3_mesh(k: int) -> MeshConfig:
+    """m1..m5 of PAPER.md Table III: BL q=1 puncture meshes of
+    decreasing adaptivity, finest level 12, 10, 8, 6, 4 (levels 3..L, rho 2.5)."""
+    L = [12, 10, 8, 6, 4][k - 1]
+    c = _bbh("m%d" % k, 1.0, L, L, 2.5, "Table III m%d: BL q=1, levels 3..%d" % (k, L))
+    return c
+
+
 CONFIGS = {
     "c1": c1_uniform,
     "c2": c2_schwarzschild,
@@ -123,6 +138,9 @@ CONFIGS = {
     "c5": c5_bbh_q8,
     "small": small_adaptive,
     "small_bbh": small_bbh,
+    "c3big": c3_large,
+    "m1": lambda: table3_mesh(1), "m2": lambda: table3_mesh(2), "m3": lambda: table3_mesh(3),
+    "m4": lambda: table3_mesh(4), "m5": lambda: table3_mesh(5),
 }
 
 

@@ -158,8 +158,8 @@ def test_dofs_bruteforce(periodic):
                 if key not in ids:
                     ids[key] = len(ids)
                 o2n[e, n] = ids[key]
-                # zip owner: finest, then lowest index
-                own = min(cont, key=lambda cs: (-m.levels[cs[0]], cs[0]))[0]
+                # zip owner (R17): coarsest, then lowest index
+                own = min(cont, key=lambda cs: (m.levels[cs[0]], cs[0]))[0]
                 assert m.zip_leaf[ids[key]] == own
             else:
                 n_hang += 1

@@ -9,7 +9,8 @@ Environment: DGR_SIGMA (KO strength, 0.4), DGR_ETA (2.0), DGR_CFL (0.25),
 DGR_BC ("both" | "somm" | "extrap"), DGR_LMAX (finest level, 8),
 DGR_PUNCT ("c2": offset h/4 in z as in synth.configs; "cell": at a cell centre),
 DGR_UPWIND (1: lopsided advective derivatives, reading R9u), DGR_RHO (refinement
-radius factor of the mesh rule, 1.0).
+radius factor of the mesh rule, 1.0), DGR_CFG (c2 default; any synth config
+name, e.g. c3 for the BL q=1 BBH).
 """
 import os
 import sys
@@ -27,7 +28,10 @@ samples = int(sys.argv[2]) if len(sys.argv) > 2 else 20
 import dataclasses
 from synth.configs import Puncture
 lmax = int(os.environ.get("DGR_LMAX", "8"))
-cfg = configs.c2_schwarzschild(rho=float(os.environ.get("DGR_RHO", "1.0")), lmax=lmax)
+if os.environ.get("DGR_CFG", "c2") == "c2":
+    cfg = configs.c2_schwarzschild(rho=float(os.environ.get("DGR_RHO", "1.0")), lmax=lmax)
+else:
+    cfg = configs.get(os.environ["DGR_CFG"])
 if os.environ.get("DGR_PUNCT", "c2") == "cell":
     hh = cfg.width / (6.0 * (1 << lmax))
     cfg = dataclasses.replace(cfg, punctures=(Puncture(hh / 2, hh / 2, hh / 2, 1.0, lmax),))
@@ -42,8 +46,8 @@ bcs = {"both": (0, 1), "somm": (1,), "extrap": (0,)}[os.environ.get("DGR_BC", "b
 steps = int(round(t_end / dt))
 every = max(1, steps // samples)
 r = np.sqrt((xyz ** 2).sum(axis=0))
-far = torch.from_numpy(r > 24.0).cuda()           # outer region (boundary at 32)
-print(f"C2: {m.info['n_oct_global']} octants, {n} DOFs, dt = {dt:.5f}, {steps} steps to t = {t_end}, "
+far = torch.from_numpy(r > 0.75 * cfg.width / 2).cuda()   # outer region (near the boundary)
+print(f"{cfg.name}: {m.info['n_oct_global']} octants, {n} DOFs, dt = {dt:.5f}, {steps} steps to t = {t_end}, "
       f"KO sigma {sigma}, eta {eta}")
 for somm in bcs:
     prm = dgr.Params(sommerfeld=somm, ko_sigma=sigma, eta=eta,
@@ -52,7 +56,7 @@ for somm in bcs:
     u[:, :n] = torch.from_numpy(u0)
     print(f"--- outer boundary: {'Sommerfeld (R29)' if somm else 'extrapolation (R12)'}")
     print(f"{'t':>7s} {'H_L2':>10s} {'H_max':>10s} {'M_L2':>10s} {'G_L2':>10s} "
-          f"{'H_max(r>24)':>12s} {'alpha_min':>10s} {'finite':>6s}")
+          f"{'H_max(outer)':>12s} {'alpha_min':>10s} {'finite':>6s}")
     t0 = time.time()
     for k in range(steps + 1):
         if k % every == 0 or k == steps:

@@ -46,8 +46,10 @@ constexpr int NSLOT = 57;
 // index c = x + 13y + 169z minus an offset so thread reads stay conflict-free
 constexpr int TX_OFF = 3, TX_N = 2191;    // x in 3..9, y, z in 0..12
 constexpr int TY_OFF = 42, TY_N = 2113;   // x, y in 3..9, z in 0..12
+constexpr int T_N = 2 * STAGE_DBL;        // Tx + Ty, or two light-field stage halves
+static_assert(TX_N + TY_N <= T_N, "Tx/Ty fit the two pair halves");
 constexpr size_t SMEM_BYTES = size_t(NSLOT) * NPP * 8 + size_t(2) * STAGE_DBL * 8 +
-                              size_t(TX_N + TY_N) * 8 + 16 + size_t(2) * RT * 2;
+                              size_t(T_N) * 8 + 16 + size_t(2) * RT * 2;
 
 // thread -> interior point map (filled by upload_rhs_tables): every warp holds
 // at most two points per residue of their stage-buffer index mod 16, so its
@@ -63,11 +65,25 @@ __device__ long long g_stage_cycles[NF + 2];
 constexpr int N_TXL = 13 * 7 + 7 * 6, N_TYL = 7 * 13;
 static_assert(N_TXL + N_TYL <= RT, "one pencil per thread");
 
-// field processing order
-__constant__ int c_order[NF] = {12, 13, 14, 15, 16, 17, 1, 0, 3, 4, 5, 6,
-                                7,  8,  2,  18, 19, 20, 21, 22, 23, 9, 10, 11};
-// field order after the metric pre-pass (k_gt_pre): the same without gt_ij
-__constant__ int c_order_pre[NF - 6] = {1, 0, 3, 4, 5, 6, 7, 8, 2, 18, 19, 20, 21, 22, 23, 9, 10, 11};
+// field processing order: the metric gt_ij (skipped after the pre-pass), then
+// the other fields with second derivatives (chi, alpha, beta^i: "heavy"),
+// then the first-derivative-only ("light") fields Gt^i, K, At_ij, B^i
+__constant__ int c_order[NF] = {12, 13, 14, 15, 16, 17, 1, 0, 6, 7, 8, 3,
+                                4,  5,  2,  18, 19, 20, 21, 22, 23, 9, 10, 11};
+__constant__ int c_order_pre[NF - 6] = {1, 0, 6, 7, 8, 3, 4, 5, 2, 18, 19, 20, 21, 22, 23, 9, 10, 11};
+// fused path: the same order in stages of one or two fields — the light
+// fields after the first go in pairs, the pair's second field staged in the
+// Tx/Ty region (free once the last heavy stage's D1 pass is done: the first
+// light stage is single, so a pair's gather, issued two stages ahead, never
+// lands while a heavy stage still uses Tx/Ty).  Same per-point arithmetic in
+// the same order as single stages (bit-identical to the two-pass path).
+constexpr int NST_FULL = 18, NST_PRE = 12;
+__constant__ int2 c_stg[NST_FULL] = {{12, -1}, {13, -1}, {14, -1}, {15, -1}, {16, -1}, {17, -1},
+                                     {1, -1},  {0, -1},  {6, -1},  {7, -1},  {8, -1},  {3, -1},
+                                     {4, 5},   {2, 18},  {19, 20}, {21, 22}, {23, 9},  {10, 11}};
+__constant__ int2 c_stg_pre[NST_PRE] = {{1, -1},  {0, -1},  {6, -1},  {7, -1},
+                                        {8, -1},  {3, -1},  {4, 5},   {2, 18},
+                                        {19, 20}, {21, 22}, {23, 9},  {10, 11}};
 
 __device__ __forceinline__ int sidx(int i, int j) {
   // (0,0)0 (0,1)1 (0,2)2 (1,1)3 (1,2)4 (2,2)5
@@ -306,12 +322,17 @@ __global__ void __launch_bounds__(RT, 1)
   // read in the prologue); the stream holds the 18 other fields
   constexpr int NS = PRE ? NF - 6 : NF;
   const int* ORD = PRE ? c_order_pre : c_order;
+  // stages: FUSED in one- or two-field stages (c_stg*), else one field each
+  constexpr int NST = FUSED ? (PRE ? NST_PRE : NST_FULL) : NS;
+  const int2* STG = PRE ? c_stg_pre : c_stg;
+  auto stA = [&](int k) { return FUSED ? STG[k].x : ORD[k]; };
+  auto stB = [&](int k) { return FUSED ? STG[k].y : -1; };
   extern __shared__ __align__(128) double smem[];
   double* slots = smem;                           // [NSLOT][NPP]
   double* stage = smem + NSLOT * NPP;             // [2][STAGE_DBL]
-  double* Tx = stage + 2 * STAGE_DBL;             // [TX_N]
+  double* Tx = stage + 2 * STAGE_DBL;             // [TX_N] (T region: [T_N])
   double* Ty = Tx + TX_N;                         // [TY_N]
-  uint64_t* bars = reinterpret_cast<uint64_t*>(Ty + TY_N);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(Tx + T_N);
   // this thread's point: patch index c0 (-1: no point) and interior index p, kept
   // in shared memory and re-read where needed (cheaper than a register spill)
   int16_t* tab_c0 = reinterpret_cast<int16_t*>(bars + 2);
@@ -352,6 +373,12 @@ __global__ void __launch_bounds__(RT, 1)
 #pragma unroll
     for (int j = 0; j < GJ; ++j)
       if (tid + RT * j < n) cp_async8(d0 + 8 * gdst[j], uf, af, gidx[j], ds);
+  };
+  // FUSED: stage k's field(s) into stage buffer b (and T-region half b), one
+  // cp.async group per stage
+  auto gather_stage = [&](int b, int k) {
+    gather(stage + b * STAGE_DBL, stA(k));
+    if (stB(k) >= 0) gather(Tx + b * STAGE_DBL, stB(k));
     cp_async_commit();
   };
   // FUSED: the value of field f at element node (e, p), through o2s
@@ -383,8 +410,8 @@ __global__ void __launch_bounds__(RT, 1)
   __syncthreads();
   if (FUSED) {
     load_gidx(e);
-    gather(stage, ORD[0]);
-    gather(stage + STAGE_DBL, ORD[1]);
+    gather_stage(0, 0);
+    gather_stage(1, 1);
   } else if (tid == 0) {
     const double* pb = patches + int64_t(e) * PATCH_PITCH;
     bulk_load(stage, pb + ORD[0] * fstride, STAGE_DBL * 8, &bars[0]);
@@ -603,7 +630,7 @@ __global__ void __launch_bounds__(RT, 1)
     for (int r = 0; r < 6; ++r) gi[r] = SL(G_INV + r);
     christoffel(gi);
   }
-  for (int st = 0; st < NS; ++st, ++g) {
+  for (int st = 0; st < NST; ++st, ++g) {
     const int buf = g & 1;
 #ifdef DGR_RHS_TIMING
     if (tid == 0) {   // per-stage cycle profile (experiment builds only)
@@ -618,8 +645,9 @@ __global__ void __launch_bounds__(RT, 1)
       __syncthreads();    // ... and everyone else's
       if (bnd) {
         // outer-boundary extrapolation along x, then y, then z (reading R12),
-        // the arithmetic of k_unzip, in shared memory
-        double* sw = stage + buf * STAGE_DBL;
+        // the arithmetic of k_unzip, in shared memory (both fields of a pair)
+        for (int hb = 0; hb < (stB(st) >= 0 ? 2 : 1); ++hb) {
+        double* sw = (hb ? Tx : stage) + buf * STAGE_DBL;
         for (int a = 0; a < 3; ++a) {
           const int sa = a == 0 ? 1 : (a == 1 ? 13 : 169);
           const int sb = a == 0 ? 13 : 1, sc = a == 2 ? 13 : 169;
@@ -650,12 +678,13 @@ __global__ void __launch_bounds__(RT, 1)
           }
           __syncthreads();
         }
+        }
       }
     } else {
       mbar_wait(&bars[buf], (g >> 1) & 1);
     }
     const double* s = stage + buf * STAGE_DBL;
-    const int f = ORD[st];
+    const int f = stA(st);
     const bool second = f <= 1 || (f >= 6 && f <= 8) || (f >= 12 && f <= 17);
     if (second) {
       // cooperative first derivatives along x (and y) of the staged field on
@@ -698,6 +727,9 @@ __global__ void __launch_bounds__(RT, 1)
       }
       __syncthreads();
     }
+    // the per-point work of one staged field f (patch in s); a pair stage runs
+    // it for both fields, in order
+    auto point_work = [&](const double* __restrict__ s, const int f) {
     const int c0 = tab_c0[tid];
     if (SOMM && bpt) {
       // radiative condition d_t f = -(x^i/r) d_i f - (f - f_inf)/r replaces the
@@ -922,15 +954,17 @@ __global__ void __launch_bounds__(RT, 1)
         SL(A_B + kk) = advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
       }
     }
+    };
+    point_work(s, f);
+    if (FUSED && stB(st) >= 0) point_work(Tx + buf * STAGE_DBL, stB(st));
     __syncthreads();  // everyone is done with this stage buffer
     if (FUSED) {
-      double* dst = stage + buf * STAGE_DBL;
-      if (st + 2 < NS) {
-        gather(dst, ORD[st + 2]);
+      if (st + 2 < NST) {
+        gather_stage(buf, st + 2);
       } else {
-        if (st + 2 == NS && en >= 0) load_gidx(en);   // the current octant's gathers are issued
-        if (en >= 0) gather(dst, ORD[st + 2 - NS]);
-        else cp_async_commit();                        // (empty group keeps the count uniform)
+        if (st + 2 == NST && en >= 0) load_gidx(en);   // the current octant's gathers are issued
+        if (en >= 0) gather_stage(buf, st + 2 - NST);
+        else cp_async_commit();                         // (empty group keeps the count uniform)
       }
       continue;
     }

@@ -107,60 +107,55 @@ __global__ void __launch_bounds__(IP_THREADS)
   const int es2 = a2 == 0 ? 1 : (a2 == 1 ? 7 : 49);
   const int es3 = a3 == 0 ? 1 : (a3 == 1 ? 7 : 49);
   const int lo1 = lo[a1], lo2 = lo[a2];
-  const float rn1 = 1.0f / float(n1);
-  // T1[g][r3][r2][i1] = sum_m W[lo1+i1][m] E_g[m, r2, r3]: one thread per
-  // (field, node row): the row's 7 values are loaded once and reused from
-  // registers for all n1 outputs (same sums in the same order as evaluating
-  // each output on its own, so results are bitwise unchanged)
-  for (int idx = tid; idx < IP_FG * 49; idx += IP_THREADS) {
-    const int g = idx / 49, r = idx - g * 49;   // r = r3 * 7 + r2
+  const float rn1 = 1.0f / float(n1), rn2 = 1.0f / float(n2);
+  // T1[g][r3][r2][i1] = sum_m W[lo1+i1][m] E_g[m, r2, r3]
+  for (int idx = tid; idx < 49 * n1; idx += IP_THREADS) {
+    const int r = fdiv(idx, rn1), i1 = idx - r * n1;   // r = r3 * 7 + r2
     const int r3 = r / 7, r2 = r - r3 * 7;
-    const double* src = Es + g * NPT + r2 * es2 + r3 * es3;
-    double v[7];
+    const int row = r2 * es2 + r3 * es3;
+    const int tt = lo1 + i1;
+    double v[IP_FG];
+    if (tt & 1) {
+      const double* w = W + tt * 7;
 #pragma unroll
-    for (int q = 0; q < 7; ++q) v[q] = src[q * es1];
-    double* dst = T1 + g * IP_T1 + r * n1;
+      for (int g = 0; g < IP_FG; ++g) v[g] = 0.0;
 #pragma unroll
-    for (int i1 = 0; i1 < IP_N1; ++i1) {
-      if (i1 >= n1) break;
-      const int tt = lo1 + i1;
-      double acc;
-      if (tt & 1) {
-        const double* w = W + tt * 7;
-        acc = 0.0;
+      for (int q = 0; q < 7; ++q) {
+        const double wq = w[q];
 #pragma unroll
-        for (int q = 0; q < 7; ++q) acc = fma(w[q], v[q], acc);
-      } else {
-        acc = src[(tt >> 1) * es1];   // a node: copy (re-read, so v stays in registers)
+        for (int g = 0; g < IP_FG; ++g) v[g] = fma(wq, Es[g * NPT + row + q * es1], v[g]);
       }
-      dst[i1] = acc;
+    } else {
+#pragma unroll
+      for (int g = 0; g < IP_FG; ++g) v[g] = Es[g * NPT + row + (tt >> 1) * es1];
     }
+#pragma unroll
+    for (int g = 0; g < IP_FG; ++g) T1[g * IP_T1 + r * n1 + i1] = v[g];
   }
   __syncthreads();
-  // T2[g][r3][i2][i1] = sum_m W[lo2+i2][m] T1[g][r3][m][i1]: one thread per
-  // (field, r3, i1) column, its 7 values reused for all n2 outputs
-  for (int idx = tid; idx < IP_FG * 7 * n1; idx += IP_THREADS) {
-    const int g = idx / (7 * n1);
-    const int rem = idx - g * 7 * n1;
-    const int r3 = fdiv(rem, rn1), i1 = rem - r3 * n1;
-    const double* src = T1 + g * IP_T1 + r3 * 7 * n1 + i1;
-    double v[7];
+  // T2[g][r3][i2][i1] = sum_m W[lo2+i2][m] T1[g][r3][m][i1]
+  for (int idx = tid; idx < 7 * n2 * n1; idx += IP_THREADS) {
+    const int q12 = fdiv(idx, rn1), i1 = idx - q12 * n1;
+    const int r3 = fdiv(q12, rn2), i2 = q12 - r3 * n2;
+    const int tt = lo2 + i2;
+    const int col = r3 * 7 * n1 + i1;
+    double v[IP_FG];
+    if (tt & 1) {
+      const double* w = W + tt * 7;
 #pragma unroll
-    for (int q = 0; q < 7; ++q) v[q] = src[q * n1];
-    double* dst = T2 + g * IP_T2 + r3 * n2 * n1 + i1;
-    for (int i2 = 0; i2 < n2; ++i2) {
-      const int tt = lo2 + i2;
-      double acc;
-      if (tt & 1) {
-        const double* w = W + tt * 7;
-        acc = 0.0;
+      for (int g = 0; g < IP_FG; ++g) v[g] = 0.0;
 #pragma unroll
-        for (int q = 0; q < 7; ++q) acc = fma(w[q], v[q], acc);
-      } else {
-        acc = src[(tt >> 1) * n1];
+      for (int q = 0; q < 7; ++q) {
+        const double wq = w[q];
+#pragma unroll
+        for (int g = 0; g < IP_FG; ++g) v[g] = fma(wq, T1[g * IP_T1 + col + q * n1], v[g]);
       }
-      dst[i2 * n1] = acc;
+    } else {
+#pragma unroll
+      for (int g = 0; g < IP_FG; ++g) v[g] = T1[g * IP_T1 + col + (tt >> 1) * n1];
     }
+#pragma unroll
+    for (int g = 0; g < IP_FG; ++g) T2[g * IP_T2 + (r3 * n2 + i2) * n1 + i1] = v[g];
   }
   __syncthreads();
   // slot value = sum_m W[t2_a3][m] T2[g][m][i2][i1]
@@ -228,35 +223,25 @@ __global__ void __launch_bounds__(UZ_THREADS, 3)
   const double* af = m.aux + f * m.aux_stride - ds;   // slot i - ds
   double* dst = patches + (int64_t(f) * m.n_owned + e) * PATCH_PITCH;
 
-  // ---- gather: 16 loads in flight per lane (two adjacent patch points per
-  // lane, 8 pairs); coalesced streaming (evict-first) 16-byte stores, so the
-  // 10-GB patch stream does not evict the element values and slots the
-  // neighbouring patches still gather from L2 (patch rows are 16-B aligned)
-  constexpr int U2 = 8;
-  for (int p0 = 0; p0 < NPATCH; p0 += 64 * U2) {
-    double v0[U2], v1[U2];
-    int o0[U2], o1[U2];
+  // ---- gather: 16 loads in flight per lane; coalesced streaming (evict-first)
+  // stores, so the 10-GB patch stream does not evict the element values and
+  // slots the neighbouring patches still gather from L2
+  constexpr int U = 16;
+  for (int p0 = 0; p0 < NPATCH; p0 += 32 * U) {
+    double v[U];
+    int o[U];
 #pragma unroll
-    for (int u = 0; u < U2; ++u) {
-      const int p = p0 + 2 * (u * 32 + lane);
-      o0[u] = p < NPATCH ? soff[p] : -3;
-      o1[u] = p + 1 < NPATCH ? soff[p + 1] : -3;
-      // (volatile asm keeps all loads ahead of the stores; invalid points load
+    for (int u = 0; u < U; ++u) {
+      const int p = p0 + u * 32 + lane;
+      o[u] = p < NPATCH ? soff[p] : -3;
+      // (volatile asm keeps all U loads ahead of the stores; invalid points load
       // element value 0 and are not stored)
-      const int x0 = max(o0[u], 0), x1 = max(o1[u], 0);
-      asm volatile("ld.global.nc.f64 %0, [%1];" : "=d"(v0[u]) : "l"((x0 < ds ? uf : af) + x0));
-      asm volatile("ld.global.nc.f64 %0, [%1];" : "=d"(v1[u]) : "l"((x1 < ds ? uf : af) + x1));
+      const int x = max(o[u], 0);
+      asm volatile("ld.global.nc.f64 %0, [%1];" : "=d"(v[u]) : "l"((x < ds ? uf : af) + x));
     }
 #pragma unroll
-    for (int u = 0; u < U2; ++u) {
-      const int p = p0 + 2 * (u * 32 + lane);
-      if (o0[u] >= 0 && o1[u] >= 0) {
-        __stcs(reinterpret_cast<double2*>(dst + p), make_double2(v0[u], v1[u]));
-      } else {
-        if (o0[u] >= 0) __stcs(dst + p, v0[u]);
-        if (o1[u] >= 0) __stcs(dst + p + 1, v1[u]);
-      }
-    }
+    for (int u = 0; u < U; ++u)
+      if (o[u] >= 0) __stcs(dst + p0 + u * 32 + lane, v[u]);
   }
 
   // ---- outer-boundary extrapolation along x, then y, then z (reading R12)

@@ -305,6 +305,31 @@ dgr_status dgr_regrid_octree(dgr_mesh m, const double* w, double eps_refine, dou
 dgr_status dgr_regrid_transfer(dgr_mesh old_m, double* u_old, dgr_mesh new_m, double* u_new,
                                void* stream);
 
+/* Gravitational-wave extraction ("the Penrose scalar Psi_4 ... expanded
+ * in spin-weighted spherical harmonics (l, m modes) on spherical shells";
+ * readings R33-R36 of DESIGN.md).
+ * dgr_psi4: psi[c * ld + e * 343 + node] (device, ld = n_oct_local * 343, c = 0
+ *   Re, 1 Im) = Psi_4 = (E_ij - i B_ij) mbar^i mbar^j at every node of every
+ *   owned octant, from that octant's own patch (E, B the electric / magnetic
+ *   Weyl parts in vacuum; tetrad r^, theta^, phi^ about center[3],
+ *   Gram-Schmidt in the physical metric).  Ghost exchange + unzip + the
+ *   234-input derivative kernel + the generated k_psi4.
+ * dgr_psi4_sphere: host points xyz[3][npts] (physical) -> out[2][npts] (host):
+ *   the degree-6 interpolant of psi over the finest octant containing each
+ *   point (single-rank meshes; synchronises).
+ * dgr_psi4_modes: the whole extraction on a sphere of `radius` about center:
+ *   Gauss-Legendre (n_theta) x uniform (n_phi) quadrature (reading R35, in
+ *   place of Lebedev's), modes[2 q], [2 q + 1] = Re, Im of C_lm = sum_k w_k
+ *   Psi_4(x_k) conj(-2Y_lm(x_k)), q over l = 2..l_max, m = -l..l; `sphere`
+ *   (host [2][n_theta * n_phi], optional) receives the point values. */
+dgr_status dgr_psi4(dgr_mesh m, double* u, const double* center, double* psi,
+                    const dgr_params* prm, void* stream);
+dgr_status dgr_psi4_sphere(dgr_mesh m, const double* psi, int64_t npts, const double* xyz,
+                           double* out, void* stream);
+dgr_status dgr_psi4_modes(dgr_mesh m, double* u, const double* center, double radius, int n_theta,
+                          int n_phi, int l_max, double* modes, double* sphere,
+                          const dgr_params* prm, void* stream);
+
 /* In-process rank group: n meshes of one octree, meshes[r] = rank r of n,
  * each created with nccl_id = NULL (one per device, or several on one device),
  * driven by ONE process.  Their ghost exchange is libdgr's own (SURVEY §8e

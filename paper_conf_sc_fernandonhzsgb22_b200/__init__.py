@@ -83,7 +83,8 @@ EXPORTED = ["dgr_status_string", "dgr_last_error", "dgr_version", "dgr_octree_bu
             "dgr_profile_enable", "dgr_profile_read", "dgr_bench_dfma", "dgr_set_option",
             "dgr_group_create", "dgr_group_ghost_exchange", "dgr_group_rk4_step",
             "dgr_group_destroy", "dgr_rhs_inputs", "dgr_rhs_algebra", "dgr_regrid_indicator",
-            "dgr_regrid_octree", "dgr_regrid_transfer"]
+            "dgr_regrid_octree", "dgr_regrid_transfer", "dgr_psi4", "dgr_psi4_sphere",
+            "dgr_psi4_modes"]
 PROF_CLASSES = ["elements", "hanging", "unzip", "rhs", "zip_rk4", "exchange", "constraints",
                 "interp"]
 
@@ -131,6 +132,9 @@ def lib():
         L.dgr_regrid_indicator.argtypes = [vp, vp, C.c_uint32, vp, vp]
         L.dgr_regrid_octree.argtypes = [vp, vp, dp, dp, i32, i32, vp, C.POINTER(i64)]
         L.dgr_regrid_transfer.argtypes = [vp, vp, vp, vp, vp]
+        L.dgr_psi4.argtypes = [vp, vp, vp, vp, C.POINTER(_Params), vp]
+        L.dgr_psi4_sphere.argtypes = [vp, vp, i64, vp, vp, vp]
+        L.dgr_psi4_modes.argtypes = [vp, vp, vp, dp, i32, i32, i32, vp, vp, C.POINTER(_Params), vp]
         for f in ["dgr_octree_build", "dgr_mesh_create", "dgr_mesh_info_get",
                   "dgr_mesh_export_maps", "dgr_mesh_destroy", "dgr_dof_coords", "dgr_unzip",
                   "dgr_ghost_exchange", "dgr_rhs_patches", "dgr_rhs", "dgr_rk4_stage",
@@ -138,7 +142,7 @@ def lib():
                   "dgr_bench_dfma", "dgr_group_create", "dgr_group_ghost_exchange",
                   "dgr_group_rk4_step", "dgr_group_destroy", "dgr_rhs_inputs",
                   "dgr_rhs_algebra", "dgr_regrid_indicator", "dgr_regrid_octree",
-                  "dgr_regrid_transfer"]:
+                  "dgr_regrid_transfer", "dgr_psi4", "dgr_psi4_sphere", "dgr_psi4_modes"]:
             getattr(L, f).restype = i32
         _lib = L
     return _lib
@@ -406,6 +410,47 @@ class Mesh:
         _check(lib().dgr_regrid_transfer(self._h, self._state(u, "u"), new_mesh._h,
                                          new_mesh._state(out, "out"), _stream()))
         return out
+
+    # ------------------------------------------------- gravitational waves
+    def psi4(self, u, center=(0.0, 0.0, 0.0), prm=None, out=None):
+        """dgr_psi4: Psi_4 (Re, Im) at every node of every owned octant,
+        [2, n_oct_local * 343] device tensor (column e * 343 + node)."""
+        import torch
+        n = self.info["n_oct_local"] * NPT
+        if out is None:
+            out = torch.empty((2, n), dtype=torch.float64, device="cuda")
+        c = (C.c_double * 3)(*center)
+        p = (prm or Params())._c()
+        _check(lib().dgr_psi4(self._h, self._state(u, "u"), c, _dev(out, (2, n), "out"),
+                              C.byref(p), _stream()))
+        return out
+
+    def psi4_sphere(self, psi, xyz):
+        """dgr_psi4_sphere: psi (from psi4()) at host points xyz [3, n] -> [2, n]."""
+        xyz = np.ascontiguousarray(np.asarray(xyz, dtype=np.float64))
+        n = xyz.shape[1]
+        out = np.zeros((2, n))
+        _check(lib().dgr_psi4_sphere(self._h, _dev(psi, (2, psi.shape[1]), "psi"), n,
+                                     xyz.ctypes.data, out.ctypes.data, _stream()))
+        return out
+
+    def psi4_modes(self, u, center=(0.0, 0.0, 0.0), radius=50.0, n_theta=16, n_phi=32,
+                   l_max=4, prm=None):
+        """dgr_psi4_modes: {(l, m): C_lm} on a sphere (and the sphere values [2, n])."""
+        nm = sum(2 * l + 1 for l in range(2, l_max + 1))
+        modes = np.zeros(2 * nm)
+        sph = np.zeros((2, n_theta * n_phi))
+        c = (C.c_double * 3)(*center)
+        p = (prm or Params())._c()
+        _check(lib().dgr_psi4_modes(self._h, self._state(u, "u"), c, float(radius), int(n_theta),
+                                    int(n_phi), int(l_max), modes.ctypes.data, sph.ctypes.data,
+                                    C.byref(p), _stream()))
+        out, q = {}, 0
+        for l in range(2, l_max + 1):
+            for m in range(-l, l + 1):
+                out[(l, m)] = complex(modes[2 * q], modes[2 * q + 1])
+                q += 1
+        return out, sph
 
     def last_launch_count(self):
         return int(lib().dgr_last_launch_count(self._h))

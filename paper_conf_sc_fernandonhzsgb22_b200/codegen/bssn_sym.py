@@ -46,8 +46,9 @@ def inputs():
     return syms, prm
 
 
-def rhs_exprs():
-    """The 24 output expressions (field order) and the input symbols."""
+def rhs_exprs(want_geometry=False):
+    """The 24 output expressions (field order) and the input symbols (and, with
+    want_geometry, the geometric intermediates for other generated kernels)."""
     syms, prm = inputs()
     val = syms[:24]
     D = lambda f, k: syms[24 + 3 * f + k]
@@ -157,4 +158,8 @@ def rhs_exprs():
         out[18 + q] = rhs_At[i, j]
     algebra = list(out)
     with_ko = [algebra[f] + KO(f) for f in range(NF)]
+    if want_geometry:
+        geo = dict(gi=gi, gt=gt, At=At, K=K, chi_e=chi_e, Gphys=Gphys, Ric=Ric, D=D,
+                   dgt=dgt, dAt=dAt, dchi=dchi, dK=dK)
+        return with_ko, syms, prm, geo
     return with_ko, syms, prm

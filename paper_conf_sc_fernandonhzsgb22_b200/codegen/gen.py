@@ -35,6 +35,7 @@ from . import bssn_sym
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 OUT = os.path.join(os.path.dirname(HERE), "csrc", "gen", "rhs_alg.cu")
+OUT_PSI4 = os.path.join(os.path.dirname(HERE), "csrc", "gen", "psi4.cu")
 VARIANTS = ["sympygr_cse", "binary_reduce", "staged_cse"]
 STAGES = [[0], [1], [2], [6, 7, 8], [9, 10, 11], [3, 4, 5], list(range(12, 18)),
           list(range(18, 24))]
@@ -82,6 +83,11 @@ class Emitter:
             if x.is_Integer and x < 0:
                 bs = self(b)
                 return "(1.0 / (" + " * ".join([bs] * int(-x)) + "))"
+            if x.is_Rational and x.q == 2:          # half-integer powers: sqrt
+                k = int(x.p)
+                bs = f"sqrt({self(b)})"
+                prod = " * ".join([bs] * abs(k))
+                return f"({prod})" if k > 0 else f"(1.0 / ({prod}))"
         raise ValueError(f"cannot emit {e!r}")
 
 
@@ -329,5 +335,65 @@ void launch_rhs_alg(int variant, int occ, const double* in, double* out, int64_t
     return stats
 
 
+PSI4_HEADER = """// GENERATED by paper_conf_sc_fernandonhzsgb22_b200/codegen/gen.py — do not edit.
+// The Weyl scalar Psi_4 (PAPER.md P:L159; readings R33-R34, codegen/psi4_sym.py)
+// at n points: in [234][ld] (the inputs of dgr_rhs_inputs), xyz [3][ld] the
+// points' positions relative to the extraction centre -> out [2][ld] (Re, Im).
+// SymPy CSE over both outputs (the generator's second workload).
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../device.cuh"
+
+namespace dgr {
+"""
+
+
+def gen_psi4(out_path=None):
+    from . import psi4_sym
+    exprs, syms, prm, (px, py, pz) = psi4_sym.psi4_exprs()
+    names = _sym_names(syms, prm)
+    names.update({px: "v_px", py: "v_py", pz: "v_pz"})
+    rep, red = sp.cse(exprs, symbols=sp.numbered_symbols("t"), optimizations=None, order="none")
+    for t, _ in rep:
+        names[t] = t.name
+    em = Emitter(names.get)
+    need = set()
+    for _, x in rep:
+        need |= x.free_symbols
+    for x in red:
+        need |= x.free_symbols
+    idx = {s_: k for k, s_ in enumerate(syms)}
+    body = [_load(s_, idx[s_]) for s_ in sorted(need & set(syms), key=idx.get)]
+    if syms[1] not in need:
+        body.append(_load(syms[1], 1))
+    body += ["const double v_px = xyz[0 * ld + i];", "const double v_py = xyz[1 * ld + i];",
+             "const double v_pz = xyz[2 * ld + i];",
+             "const double chi_e = fmax(v_chi, p.chi_floor);"]
+    body += [f"const double {t.name} = {em(x)};" for t, x in rep]
+    body += [f"out[{f} * ld + i] = {em(x)};" for f, x in enumerate(red)]
+    lines = [PSI4_HEADER, f"// {len(rep)} CSE temporaries",
+             "__global__ void __launch_bounds__(128)",
+             "k_psi4(const double* __restrict__ in, const double* __restrict__ xyz, "
+             "double* __restrict__ out, int64_t n, int64_t ld, AlgParams p) {",
+             "  for (int64_t i = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; i < n;",
+             "       i += int64_t(gridDim.x) * blockDim.x) {"]
+    lines += ["    " + l for l in body]
+    lines += ["  }", "}", "",
+              "void launch_psi4(const double* in, const double* xyz, double* out, int64_t n, "
+              "int64_t ld, const AlgParams& p, cudaStream_t s) {",
+              "  if (n <= 0) return;",
+              "  int64_t blocks = (n + 127) / 128;",
+              "  const int64_t cap = int64_t(sm_count()) * 8;",
+              "  if (blocks > cap) blocks = cap;",
+              "  k_psi4<<<int(blocks), 128, 0, s>>>(in, xyz, out, n, ld, p);",
+              "}", "", "}  // namespace dgr", ""]
+    out_path = out_path or OUT_PSI4
+    with open(out_path, "w") as f:
+        f.write("\n".join(lines))
+    print(f"psi4: {len(rep)} CSE temporaries; wrote {out_path}")
+
+
 if __name__ == "__main__":
-    sys.exit(main())
+    main()
+    gen_psi4()

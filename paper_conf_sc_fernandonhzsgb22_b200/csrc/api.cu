@@ -128,6 +128,11 @@ struct dgr_mesh_s {
   double* d_us = nullptr;       // RK4 stage state [24][dof_stride]
   double* d_acc = nullptr;      // RK4 accumulator
   double* d_cnorm = nullptr;    // constraint norm partials
+  // Psi_4 extraction (allocated on first use): inputs [234][n], positions [3][n],
+  // Psi_4 at the octant nodes [2][n], n = n_owned * 343
+  double* d_psi_in = nullptr;
+  double* d_psi_xyz = nullptr;
+  double* d_psi = nullptr;
   // dgr_rk4_step_host: three device state slots, copy streams and events
   // (allocated on first use)
   double* d_hbuf[3] = {nullptr, nullptr, nullptr};
@@ -1372,6 +1377,172 @@ dgr_status dgr_regrid_transfer(dgr_mesh old_m, double* u_old, dgr_mesh new_m, do
   CUDA_TRY(cudaGetLastError());
   CUDA_TRY(cudaFreeAsync(d_map, st));
   CUDA_TRY(cudaStreamSynchronize(st));   // the host map is freed on return
+  return DGR_OK;
+}
+
+// ---------------------------------------------------------- Psi_4 extraction
+dgr_status dgr_psi4(dgr_mesh m, double* u, const double* center, double* psi,
+                    const dgr_params* prm, void* stream) {
+  dgr_status s = need_device(m);
+  if (s) return s;
+  if (!u || !center || !psi) return fail(DGR_ERR_ARG, "null argument");
+  const int64_t n = int64_t(m->dm.n_owned) * NPT;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (!m->d_psi_in) CUDA_TRY(m->alloc(&m->d_psi_in, size_t(234) * std::max<int64_t>(n, 1)));
+  if (!m->d_psi_xyz) CUDA_TRY(m->alloc(&m->d_psi_xyz, size_t(3) * std::max<int64_t>(n, 1)));
+  m->launches = 0;
+  if ((s = exchange(m, u, st))) return s;
+  if ((s = do_unzip(m, u, NF, st))) return s;
+  const RhsParams rp = to_rp(prm);
+  const AlgParams ap{rp.eta, rp.lambda_f0, rp.lambda_f1, rp.chi_floor};
+  PROF(m, 6, st, launch_rhs_inputs(m->dm, m->d_patch, m->d_psi_in, n, rp.ko_sigma, st));
+  PROF(m, 6, st, launch_octant_xyz(m->dm, center, m->d_psi_xyz, n, st));
+  PROF(m, 6, st, launch_psi4(m->d_psi_in, m->d_psi_xyz, psi, n, n, ap, st));
+  CUDA_TRY(cudaGetLastError());
+  return DGR_OK;
+}
+
+dgr_status dgr_psi4_sphere(dgr_mesh m, const double* psi, int64_t npts, const double* xyz,
+                           double* out, void* stream) {
+  dgr_status s = need_device(m);
+  if (s) return s;
+  if (!psi || npts < 0 || (npts > 0 && (!xyz || !out))) return fail(DGR_ERR_ARG, "bad psi4_sphere args");
+  const HostMesh& h = m->host;
+  if (h.nranks != 1) return fail(DGR_ERR_STATE, "dgr_psi4_sphere: single-rank meshes only");
+  if (npts == 0) return DGR_OK;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  const double unit = h.width / double(h.L);
+  std::vector<int32_t> oc(static_cast<size_t>(npts));
+  std::vector<double> t(static_cast<size_t>(3 * npts));
+  for (int64_t k = 0; k < npts; ++k) {
+    double X[3];
+    int64_t lo[3];
+    bool on[3];
+    for (int a = 0; a < 3; ++a) {
+      X[a] = (xyz[a * npts + k] - h.xmin[a]) / unit;
+      lo[a] = int64_t(std::floor(X[a] / 6.0));
+      on[a] = double(lo[a]) * 6.0 == X[a];
+    }
+    // finest leaf whose closed box contains X, lowest Morton index on ties (R36)
+    int32_t best = -1;
+    for (int q = 0; q < 8; ++q) {
+      int64_t c[3];
+      for (int a = 0; a < 3; ++a) c[a] = (on[a] && ((q >> a) & 1)) ? lo[a] - 1 : lo[a];
+      const int32_t leaf = h.locate(c[0], c[1], c[2]);
+      if (leaf < 0) continue;
+      if (best < 0 || h.oct[leaf].l > h.oct[best].l ||
+          (h.oct[leaf].l == h.oct[best].l && leaf < best))
+        best = leaf;
+    }
+    if (best < 0) return fail(DGR_ERR_ARG, "extraction point outside the domain");
+    oc[size_t(k)] = best;
+    const double sd = double(h.side(best));
+    for (int a = 0; a < 3; ++a) t[size_t(a * npts + k)] = (X[a] - 6.0 * double(h.oct[best].a[a])) / sd;
+  }
+  int32_t* d_oc = nullptr;
+  double *d_t = nullptr, *d_out = nullptr;
+  CUDA_TRY(cudaMallocAsync(&d_oc, size_t(npts) * 4, st));
+  CUDA_TRY(cudaMallocAsync(&d_t, size_t(3 * npts) * 8, st));
+  CUDA_TRY(cudaMallocAsync(&d_out, size_t(2 * npts) * 8, st));
+  CUDA_TRY(cudaMemcpyAsync(d_oc, oc.data(), size_t(npts) * 4, cudaMemcpyHostToDevice, st));
+  CUDA_TRY(cudaMemcpyAsync(d_t, t.data(), size_t(3 * npts) * 8, cudaMemcpyHostToDevice, st));
+  PROF(m, 6, st, launch_sphere_interp(psi, int64_t(m->dm.n_owned) * NPT, d_oc, d_t, npts, d_out, st));
+  CUDA_TRY(cudaGetLastError());
+  CUDA_TRY(cudaMemcpyAsync(out, d_out, size_t(2 * npts) * 8, cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(cudaFreeAsync(d_oc, st));
+  CUDA_TRY(cudaFreeAsync(d_t, st));
+  CUDA_TRY(cudaFreeAsync(d_out, st));
+  CUDA_TRY(cudaStreamSynchronize(st));
+  return DGR_OK;
+}
+
+// Gauss-Legendre nodes (ascending) and weights by Newton iteration on P_n
+static void gauss_legendre(int n, std::vector<double>& x, std::vector<double>& w) {
+  x.assign(size_t(n), 0.0);
+  w.assign(size_t(n), 0.0);
+  for (int i = 0; i < n; ++i) {
+    double z = std::cos(M_PI * (i + 0.75) / (n + 0.5)), dp = 0.0;
+    for (int it = 0; it < 100; ++it) {
+      double p0 = 1.0, p1 = z;
+      for (int k = 2; k <= n; ++k) {
+        const double p2 = ((2.0 * k - 1.0) * z * p1 - (k - 1.0) * p0) / k;
+        p0 = p1;
+        p1 = p2;
+      }
+      if (n == 1) { p1 = z; p0 = 1.0; }
+      dp = n * (z * p1 - p0) / (z * z - 1.0);
+      const double dz = p1 / dp;
+      z -= dz;
+      if (std::fabs(dz) < 1e-16) break;
+    }
+    x[size_t(n - 1 - i)] = z;
+    w[size_t(n - 1 - i)] = 2.0 / ((1.0 - z * z) * dp * dp);
+  }
+}
+
+// spin-weighted spherical harmonic sY_lm (Goldberg et al. 1967), real and
+// imaginary parts
+static void swsh(int sw, int l, int mm, double th, double ph, double* re, double* im) {
+  auto fact = [](int k) { double f = 1.0; for (int i = 2; i <= k; ++i) f *= i; return f; };
+  auto comb = [&](int a, int b) { return (b < 0 || b > a) ? 0.0 : fact(a) / (fact(b) * fact(a - b)); };
+  if (l < std::abs(sw) || l < std::abs(mm)) { *re = *im = 0.0; return; }
+  const double pre = ((mm & 1) ? -1.0 : 1.0) *
+                     std::sqrt((2 * l + 1) / (4 * M_PI) * fact(l + mm) * fact(l - mm) /
+                               (fact(l + sw) * fact(l - sw)));
+  double tot = 0.0;
+  for (int r = 0; r <= l - sw; ++r) {
+    const int k = r + sw - mm;
+    if (k < 0 || k > l + sw) continue;
+    tot += comb(l - sw, r) * comb(l + sw, k) * (((l - r - sw) & 1) ? -1.0 : 1.0) *
+           std::pow(std::cos(th / 2), 2 * r + sw - mm) * std::pow(std::sin(th / 2), 2 * l - 2 * r - sw + mm);
+  }
+  *re = pre * tot * std::cos(mm * ph);
+  *im = pre * tot * std::sin(mm * ph);
+}
+
+dgr_status dgr_psi4_modes(dgr_mesh m, double* u, const double* center, double radius, int n_theta,
+                          int n_phi, int l_max, double* modes, double* sphere,
+                          const dgr_params* prm, void* stream) {
+  dgr_status s = need_device(m);
+  if (s) return s;
+  if (!u || !center || !modes || radius <= 0 || n_theta < 1 || n_phi < 1 || l_max < 2 || l_max > 12)
+    return fail(DGR_ERR_ARG, "bad psi4_modes args (radius > 0, l_max in 2..12)");
+  const int64_t n = int64_t(m->dm.n_owned) * NPT;
+  if (!m->d_psi) CUDA_TRY(m->alloc(&m->d_psi, size_t(2) * std::max<int64_t>(n, 1)));
+  if ((s = dgr_psi4(m, u, center, m->d_psi, prm, stream))) return s;
+  std::vector<double> gx, gw;
+  gauss_legendre(n_theta, gx, gw);
+  const int64_t np = int64_t(n_theta) * n_phi;
+  std::vector<double> xyz(static_cast<size_t>(3 * np)), th(static_cast<size_t>(np)),
+      ph(static_cast<size_t>(np)), wt(static_cast<size_t>(np));
+  for (int i = 0; i < n_theta; ++i)
+    for (int j = 0; j < n_phi; ++j) {
+      const int64_t k = int64_t(i) * n_phi + j;
+      th[size_t(k)] = std::acos(gx[size_t(i)]);
+      ph[size_t(k)] = 2.0 * M_PI * j / n_phi;
+      wt[size_t(k)] = gw[size_t(i)] * (2.0 * M_PI / n_phi);
+      xyz[size_t(k)] = radius * std::sin(th[size_t(k)]) * std::cos(ph[size_t(k)]) + center[0];
+      xyz[size_t(np + k)] = radius * std::sin(th[size_t(k)]) * std::sin(ph[size_t(k)]) + center[1];
+      xyz[size_t(2 * np + k)] = radius * std::cos(th[size_t(k)]) + center[2];
+    }
+  std::vector<double> val(static_cast<size_t>(2 * np));
+  if ((s = dgr_psi4_sphere(m, m->d_psi, np, xyz.data(), val.data(), stream))) return s;
+  if (sphere) std::memcpy(sphere, val.data(), val.size() * 8);
+  int q = 0;
+  for (int l = 2; l <= l_max; ++l)
+    for (int mm = -l; mm <= l; ++mm, ++q) {
+      double cr = 0.0, ci = 0.0;
+      for (int64_t k = 0; k < np; ++k) {
+        double yr, yi;
+        swsh(-2, l, mm, th[size_t(k)], ph[size_t(k)], &yr, &yi);
+        const double pr = val[size_t(k)], pi_ = val[size_t(np + k)];
+        // psi * conj(Y)
+        cr += wt[size_t(k)] * (pr * yr + pi_ * yi);
+        ci += wt[size_t(k)] * (pi_ * yr - pr * yi);
+      }
+      modes[2 * q] = cr;
+      modes[2 * q + 1] = ci;
+    }
   return DGR_OK;
 }
 

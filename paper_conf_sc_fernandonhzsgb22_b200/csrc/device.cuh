@@ -149,6 +149,14 @@ void launch_wavelet(const DevMesh& m, const double* patches, uint32_t mask, doub
 void launch_transfer(const DevMesh& old, const double* u_old, const int4* map, int64_t n,
                      double* u_new, int64_t new_stride, cudaStream_t s);
 
+// gen/psi4.cu (generated) + psi4.cu: gravitational-wave extraction (R33-R36)
+void launch_psi4(const double* in, const double* xyz, double* out, int64_t n, int64_t ld,
+                 const AlgParams& p, cudaStream_t s);
+void launch_octant_xyz(const DevMesh& m, const double c[3], double* xyz, int64_t ld,
+                       cudaStream_t s);
+void launch_sphere_interp(const double* psi, int64_t ld, const int32_t* oct, const double* t,
+                          int64_t n, double* out, cudaStream_t s);
+
 // constraints_kernel.cu
 void launch_constraints(const DevMesh& m, const double* patches, double* c_oct,
                         const RhsParams& p, cudaStream_t s);

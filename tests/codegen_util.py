@@ -61,3 +61,19 @@ def oracle_rhs(x, prm=None):
 def relerr(got, want):
     scale = np.maximum(np.abs(want).max(axis=1), 1e-300)
     return np.abs(got - want).max(axis=1) / scale
+
+
+def eval_cse(exprs, values):
+    """Evaluate SymPy expressions numerically through their CSE (fast for the
+    large generated algebras): values maps input symbols to numpy arrays."""
+    import sympy as sp
+    rep, red = sp.cse(exprs, optimizations=None, order="none")
+    env = dict(values)
+    for t, e in rep + [(None, r) for r in red]:
+        fs = sorted(e.free_symbols, key=lambda s: s.name)
+        v = sp.lambdify(fs, e, modules="numpy")(*[env[s] for s in fs])
+        if t is None:
+            env.setdefault("__out__", []).append(v)
+        else:
+            env[t] = v
+    return env["__out__"]

@@ -38,4 +38,16 @@ g = dgr.Group(meshes)
 g.rk4_step(sts, dt)
 torch.cuda.synchronize()
 g.close()
+# regrid (k_wavelet, k_transfer) and Psi_4 extraction (k_rhs_inputs, k_psi4,
+# k_sphere_interp), lopsided advection, generated algebra kernels
+w = m.regrid_indicator(ud).cpu().numpy()
+octs = m.regrid_octree(w, float(np.quantile(w, 0.8)), float(np.quantile(w, 0.3)), 1, lmax + 1)
+m2 = dgr.Mesh(cfg, octs)
+m.regrid_transfer(ud, m2)
+m.psi4_modes(ud, (0.013, -0.021, 0.007), 5.0, 6, 12, l_max=3)
+m.rk4_step(ud, dt, prm=dgr.Params(upwind=1))
+inp = m.rhs_inputs(ud)
+for v in dgr.ALG_VARIANTS:
+    dgr.rhs_algebra(v, inp)
+torch.cuda.synchronize()
 print("sanitize case done", flush=True)

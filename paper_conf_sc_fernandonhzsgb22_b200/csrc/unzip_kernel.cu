@@ -36,7 +36,10 @@ constexpr int UZ_THREADS = 32 * UZ_WARPS;
 #define DGR_IP_FG 4
 #endif
 constexpr int IP_FG = DGR_IP_FG;            // fields per k_interp CTA
-constexpr int IP_THREADS = 256;
+#ifndef DGR_IP_THREADS
+#define DGR_IP_THREADS 256
+#endif
+constexpr int IP_THREADS = DGR_IP_THREADS;   // (experiment builds: -DDGR_IP_THREADS=...)
 // sweep scratch per field: a face group's box is at most IP_N1 = 4 points thick
 // along its first sweep axis (host-checked in api.cu), so T1 = 49 x n1 and
 // T2 = 7 x n2 x n1 <= 7 x 13 x 4 (29 KB per 4-field CTA: 6 CTAs per SM)
@@ -203,7 +206,13 @@ void launch_interp(const DevMesh& m, const double* u, int nf, int64_t first, int
 // copies with 8 loads in flight per lane and coalesced stores, then the
 // outer-boundary extrapolation along x, y, z (boundary octants only) in three
 // warp-synchronous passes over the patch just written.
-__global__ void __launch_bounds__(UZ_THREADS, 3)
+#ifndef DGR_UZ_MINB
+#define DGR_UZ_MINB 3
+#endif
+#ifndef DGR_UZ_U
+#define DGR_UZ_U 16
+#endif
+__global__ void __launch_bounds__(UZ_THREADS, DGR_UZ_MINB)
     k_unzip(DevMesh m, const double* __restrict__ u, double* __restrict__ patches, int nf) {
   __shared__ int32_t soff[NPATCH];
   __shared__ double WX[21];
@@ -226,7 +235,7 @@ __global__ void __launch_bounds__(UZ_THREADS, 3)
   // ---- gather: 16 loads in flight per lane; coalesced streaming (evict-first)
   // stores, so the 10-GB patch stream does not evict the element values and
   // slots the neighbouring patches still gather from L2
-  constexpr int U = 16;
+  constexpr int U = DGR_UZ_U;   // loads in flight per lane (experiment builds: -DDGR_UZ_U=...)
   for (int p0 = 0; p0 < NPATCH; p0 += 32 * U) {
     double v[U];
     int o[U];

@@ -158,3 +158,37 @@ def test_host_only_mesh_refuses_device_calls():
         m.rk4_step_host([h], [], 1e-3)
     with pytest.raises(ValueError):
         m.rk4_step_host([h[:, :-1].contiguous()], [h], 1e-3)
+
+
+def test_round2_entry_points_validate_without_gpu():
+    """The round-2 C ABI (group, regrid, Psi_4, code-generation study) rejects
+    null / host-only arguments synchronously, before any CUDA call."""
+    L = dgr.lib()
+    cfg = configs.c1_uniform()
+    m = dgr.Mesh(cfg, device=False)
+    vp = C.c_void_p
+    p16 = vp(16)
+    c3 = (C.c_double * 3)(0.0, 0.0, 0.0)
+    # host-only mesh -> DGR_ERR_STATE
+    assert L.dgr_regrid_indicator(m._h, p16, 0xFFFFFF, p16, None) == -6
+    assert L.dgr_regrid_transfer(m._h, p16, m._h, p16, None) == -6
+    assert L.dgr_psi4(m._h, p16, c3, p16, None, None) == -6
+    assert L.dgr_psi4_modes(m._h, p16, c3, C.c_double(1.0), 4, 8, 2, p16, None, None, None) == -6
+    assert L.dgr_rhs_inputs(m._h, p16, p16, 10, None, None) == -6
+    # null / out-of-range arguments -> DGR_ERR_ARG
+    assert L.dgr_rhs_algebra(3, 0, p16, p16, 1, 1, None, None) == -1
+    assert L.dgr_rhs_algebra(0, 0, p16, p16, 5, 4, None, None) == -1
+    n = C.c_int64(0)
+    assert L.dgr_regrid_octree(None, None, C.c_double(1.0), C.c_double(0.5), 0, 3, None,
+                               C.byref(n)) == -1
+    arr = (vp * 1)(m._h.value)
+    g = vp()
+    assert L.dgr_group_create(arr, 1, C.byref(g)) == -1        # host-only mesh in a group
+    assert L.dgr_group_create(None, 2, C.byref(g)) == -1
+    # regrid octree works on host-only meshes: eps between all w -> the same tree
+    w = np.full(m.info["n_oct_global"], 0.5)
+    octs = m.regrid_octree(w, 1.0, 0.1, 0, 18)
+    assert np.array_equal(octs, m.octants)
+    # with every octant above eps_refine: one level finer everywhere
+    octs = m.regrid_octree(w, 0.25, 0.1, 0, 18)
+    assert len(octs) == 8 * m.info["n_oct_global"] and np.all(octs[:, 3] == m.octants[0, 3] + 1)

@@ -13,9 +13,10 @@ run() {
 {
 run exp0
 run exp1 -DDGR_UZ_U=12 -DDGR_UZ_MINB=4
-run exp2 -DDGR_UZ_U=8 -DDGR_UZ_MINB=5
-run exp3 -DDGR_IP_THREADS=128
-run exp4 -DDGR_IP_THREADS=512
-run exp5 -DDGR_UZ_U=24 -DDGR_UZ_MINB=2
+run exp6 -DDGR_UZ_U=12 -DDGR_UZ_MINB=5
+run exp7 -DDGR_UZ_U=14 -DDGR_UZ_MINB=4
+run exp8 -DDGR_UZ_U=10 -DDGR_UZ_MINB=5
+run exp9 -DDGR_IP_THREADS=128 -DDGR_IP_FG=2
+run exp10 -DDGR_IP_THREADS=192
 } > gpurun_out/${TAG}.txt 2>&1
 cat gpurun_out/${TAG}.txt

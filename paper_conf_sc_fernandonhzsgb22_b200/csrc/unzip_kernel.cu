@@ -37,7 +37,7 @@ constexpr int UZ_THREADS = 32 * UZ_WARPS;
 #endif
 constexpr int IP_FG = DGR_IP_FG;            // fields per k_interp CTA
 #ifndef DGR_IP_THREADS
-#define DGR_IP_THREADS 256
+#define DGR_IP_THREADS 128   // (A/B: 0.493 -> 0.488 ms on C3; 512: 0.675)
 #endif
 constexpr int IP_THREADS = DGR_IP_THREADS;   // (experiment builds: -DDGR_IP_THREADS=...)
 // sweep scratch per field: a face group's box is at most IP_N1 = 4 points thick
@@ -207,10 +207,10 @@ void launch_interp(const DevMesh& m, const double* u, int nf, int64_t first, int
 // outer-boundary extrapolation along x, y, z (boundary octants only) in three
 // warp-synchronous passes over the patch just written.
 #ifndef DGR_UZ_MINB
-#define DGR_UZ_MINB 3
+#define DGR_UZ_MINB 4   // (A/B, profiles/r2ab_*, r2ac_*: 14 loads in flight x 4 CTAs per SM: 2.51 -> 2.45 ms on C3)
 #endif
 #ifndef DGR_UZ_U
-#define DGR_UZ_U 16
+#define DGR_UZ_U 14
 #endif
 __global__ void __launch_bounds__(UZ_THREADS, DGR_UZ_MINB)
     k_unzip(DevMesh m, const double* __restrict__ u, double* __restrict__ patches, int nf) {

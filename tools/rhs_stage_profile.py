@@ -15,12 +15,16 @@ buf = (C.c_longlong * 25)()
 dgr.lib().dgr_debug_rhs_stage_cycles(buf)
 m.rhs(u); torch.cuda.synchronize()
 dgr.lib().dgr_debug_rhs_stage_cycles(buf)
-order = [12, 13, 14, 15, 16, 17, 1, 0, 3, 4, 5, 6, 7, 8, 2, 18, 19, 20, 21, 22, 23, 9, 10, 11]
-names = ["alpha", "chi", "K", "Gt0", "Gt1", "Gt2", "b0", "b1", "b2", "B0", "B1", "B2",
-         "gxx", "gxy", "gxz", "gyy", "gyz", "gzz", "Axx", "Axy", "Axz", "Ayy", "Ayz", "Azz"]
 v = np.array(buf[:], dtype=np.float64)
 tot = v.sum()
-print("slot 0 = epilogue-to-prologue gap; slot k = stage k-1; slot 24 = stage 23")
-lab = ["(prologue)"] + [names[order[k]] + (" +CH" if k == 5 else "") for k in range(24)]
-for k in range(25):
-    print(f"{k:3d} {lab[k]:12s} {100 * v[k] / tot:6.2f}%")
+# default path (fused, metric pre-pass, light-field pairs; rhs_kernel.cu c_stg_pre):
+# slot 0 = epilogue of the previous octant + prologue (values, pre-pass rows,
+# Christoffel block); slot k = stage k-1; slot 24 = the last stage
+stages = ["chi", "alpha", "b0", "b1", "b2", "Gt0", "Gt1+Gt2", "K+Axx", "Axy+Axz", "Ayy+Ayz",
+          "Azz+B0", "B1+B2"]
+print("slot 0 = epilogue-to-prologue (incl. Christoffel block); slot k = stage k-1")
+for k in range(len(stages) + 1):
+    lab = "(prologue)" if k == 0 else stages[k - 1]
+    val = v[k] if k < len(stages) else v[k] + v[24]
+    print(f"{k:3d} {lab:12s} {100 * val / tot:6.2f}%")
+print(f"cycles total {tot:.3e} (CTA thread 0, summed over octants)")

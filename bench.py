@@ -454,6 +454,7 @@ def main():
                           + (", 10 GB patch buffer per stage)" if args.path == "two-pass" else ")")),
                    "parallelism": f"morton-partition x{world}"},
         "rhs_gflops": (kern.get("rhs", {}).get("achieved", 0) * 1e3) or None,
+        "octant_points_per_s": info["n_oct_global"] * 343 / (ms_max * 1e-3),
         "roofline": roof,
         "kernels": kern,
         "kernel_timing": ("CUDA events around every libdgr launch on its stream, over a second "

@@ -39,7 +39,8 @@ lmin, lmax = m.info["level_min"], m.info["level_max"]
 steps = int(round(t_end / dt))
 print(f"{name}: {m.info['n_oct_global']} octants, dt {dt:.5f}, {steps} steps, regrid every {fr}, "
       f"extract every {every} at r = {radius}", flush=True)
-print(f"{'t':>7s} {'Re C22':>11s} {'Im C22':>11s} {'|C20|':>10s} {'H_L2':>10s} {'octants':>8s}")
+print(f"{'t':>7s} {'Re C22':>11s} {'Im C22':>11s} {'|C20|':>10s} {'H_L2':>10s} {'octants':>8s} "
+      f"{'Re C20':>11s}")
 t0 = time.time()
 t_regrid = 0.0
 for k in range(steps + 1):
@@ -48,7 +49,7 @@ for k in range(steps + 1):
         _, nm = m.constraints(u, prm=prm)
         c22, c20 = modes[(2, 2)], modes[(2, 0)]
         print(f"{k * dt:7.2f} {c22.real: .4e} {c22.imag: .4e} {abs(c20):.4e} {nm[0, 0]:.4e} "
-              f"{m.info['n_oct_global']:8d}", flush=True)
+              f"{m.info['n_oct_global']:8d} {c20.real: .4e}", flush=True)
         if not np.isfinite(nm[0, 0]):
             break
     if k > 0 and k % fr == 0 and k < steps:

@@ -81,9 +81,9 @@ __device__ __forceinline__ double trace6(const double* gi, const double* X) {
 
 }  // namespace
 
-// (__maxnreg__: the full 184-register budget of a 352-thread CTA — with
-// __launch_bounds__(352, 1) ptxas settled on 168 registers and 564 B of spills)
-__global__ void __maxnreg__(184)
+// (__maxnreg__(184) removes half the spills but the launch then fails with
+// "too many resources requested": kept at __launch_bounds__(352, 1))
+__global__ void __launch_bounds__(CT, 1)
     k_constraints(DevMesh m, const double* __restrict__ patches, double* __restrict__ c_oct,
                   RhsParams prm) {
   extern __shared__ __align__(128) double smem[];

@@ -543,9 +543,6 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
       std::vector<int32_t> gs(gm.size(), -1);
       std::vector<int16_t> gd(gm.size(), 0);
       std::vector<int> idx(NPATCH);
-      // (DGR_GATHER_SORT_ONLY=1: the round-1 order, source-sorted only — A/B switch)
-      const char* so = std::getenv("DGR_GATHER_SORT_ONLY");
-      const bool interleave_banks = !(so && so[0] == '1');
       for (int64_t e = 0; e < no; ++e) {
         const int32_t* row = gm.data() + size_t(e) * GM_PITCH;
         // groups: cross points (at most one coordinate in the padding: all a
@@ -564,35 +561,10 @@ static dgr_status upload(dgr_mesh m, cudaStream_t st) {
           const int ga = grp(a), gb = grp(b);
           return ga != gb ? ga < gb : row[a] < row[b];
         });
-        // shared-memory banks: 8-byte cp.async are written half a warp at a
-        // time, patch point p in bank pair p mod 16, so 16 consecutive entries
-        // are conflict-free iff their residues differ.  Inside each group,
-        // interleave the source-sorted entries by bank pair — cycles
-        // (0, 1, ..., 15), each taking the next smallest source of every
-        // residue — so any 16 consecutive entries hit distinct pairs (while
-        // the residue buckets last) and a warp's sources stay close together.
-        if (interleave_banks) {
-          std::vector<int> out;
-          out.reserve(NPATCH);
-          size_t g0 = 0;
-          while (g0 < size_t(NPATCH)) {
-            size_t g1 = g0;
-            while (g1 < size_t(NPATCH) && grp(idx[g1]) == grp(idx[g0])) ++g1;
-            std::vector<int> bucket[16];
-            for (size_t k = g0; k < g1; ++k) bucket[idx[k] % 16].push_back(idx[k]);
-            size_t pos[16] = {0};
-            size_t left = g1 - g0;
-            while (left) {
-              for (int r = 0; r < 16; ++r)
-                if (pos[r] < bucket[r].size()) {
-                  out.push_back(bucket[r][pos[r]++]);
-                  --left;
-                }
-            }
-            g0 = g1;
-          }
-          idx.assign(out.begin(), out.end());
-        }
+        // (interleaving the entries by shared-memory bank pair to remove the
+        // cp.async write conflicts measured slower — k_rhs 5.58 -> 5.97 ms:
+        // the data-pipe wavefronts follow the number of global lines a warp's
+        // 32 copies touch, which the source order minimises)
         for (int k = 0; k < NPATCH; ++k) {
           gs[size_t(e) * GM_PITCH + k] = row[idx[k]];
           gd[size_t(e) * GM_PITCH + k] = int16_t(idx[k]);

@@ -727,6 +727,54 @@ __global__ void __launch_bounds__(RT, 1)
       }
       __syncthreads();
     }
+    // the per-point work of a first-derivative-only ("light") field f from its
+    // derivatives d (s: its staged patch, which the lopsided advection reads)
+    auto light_apply = [&](const double* __restrict__ s, const int f, const Derivs& d) {
+      const int c0 = tab_c0[tid];
+      if (f >= 3 && f <= 5) {
+        // ---------------- Gt^k: Ricci d Gt term, advection + KO kept apart (eq 3)
+        const int kk = f - 3;
+        SL(S0 + kk) = advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
+        double gi[6], gt[6], Rg[6];
+#pragma unroll
+        for (int r = 0; r < 6; ++r) {
+          gi[r] = SL(G_INV + r);
+          gt[r] = SL(V_GAM + r);
+        }
+#pragma unroll
+        for (int i = 0; i < 3; ++i)
+#pragma unroll
+          for (int j = i; j < 3; ++j)
+            Rg[sidx(i, j)] = 0.5 * (gt[sidx(kk, i)] * d.d1[j] + gt[sidx(kk, j)] * d.d1[i]);
+        const double trR = trace6(gi, Rg);
+        const double ca = chi * alpha;
+        if (TF_ONCE) {
+#pragma unroll
+          for (int r = 0; r < 6; ++r) SL(A_AT + r) += ca * Rg[r];
+          ttr += ca * trR;
+        } else {
+#pragma unroll
+          for (int r = 0; r < 6; ++r) SL(A_AT + r) += ca * (Rg[r] - gt[r] * trR * (1.0 / 3.0));
+        }
+      } else if (f == 2) {
+        // ---------------- K: advection, KO, eq (8) -4/3 alpha gt^ij d_j K
+        rK += advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
+        double gi[6];
+#pragma unroll
+        for (int r = 0; r < 6; ++r) gi[r] = SL(G_INV + r);
+#pragma unroll
+        for (int i = 0; i < 3; ++i)
+          SL(A_GT + i) += -(4.0 / 3.0) * alpha *
+                          (gi[sidx(i, 0)] * d.d1[0] + gi[sidx(i, 1)] * d.d1[1] +
+                           gi[sidx(i, 2)] * d.d1[2]);
+      } else if (f >= 18) {
+        const int q = f - 18;
+        SL(A_AT + q) += advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
+      } else {  // 9..11: B
+        const int kk = f - 9;
+        SL(A_B + kk) = advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
+      }
+    };
     // the per-point work of one staged field f (patch in s); a pair stage runs
     // it for both fields, in order
     auto point_work = [&](const double* __restrict__ s, const int f) {
@@ -850,32 +898,6 @@ __global__ void __launch_bounds__(RT, 1)
 #pragma unroll
           for (int i = 0; i < 3; ++i) SL(A_GT + i) += -2.0 * v[i];
         }
-      } else if (f >= 3 && f <= 5) {
-        // ---------------- Gt^k: Ricci d Gt term, advection + KO kept apart (eq 3)
-        const int kk = f - 3;
-        const Derivs d = derivs<false>(s, c0, ih, ko_scale);
-        SL(S0 + kk) = advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
-        double gi[6], gt[6], Rg[6];
-#pragma unroll
-        for (int r = 0; r < 6; ++r) {
-          gi[r] = SL(G_INV + r);
-          gt[r] = SL(V_GAM + r);
-        }
-#pragma unroll
-        for (int i = 0; i < 3; ++i)
-#pragma unroll
-          for (int j = i; j < 3; ++j)
-            Rg[sidx(i, j)] = 0.5 * (gt[sidx(kk, i)] * d.d1[j] + gt[sidx(kk, j)] * d.d1[i]);
-        const double trR = trace6(gi, Rg);
-        const double ca = chi * alpha;
-        if (TF_ONCE) {
-#pragma unroll
-          for (int r = 0; r < 6; ++r) SL(A_AT + r) += ca * Rg[r];
-          ttr += ca * trR;
-        } else {
-#pragma unroll
-          for (int r = 0; r < 6; ++r) SL(A_AT + r) += ca * (Rg[r] - gt[r] * trR * (1.0 / 3.0));
-        }
       } else if (f >= 6 && f <= 8) {
         // ---------------- beta^kk: Lie derivative terms, eq (2), eq (8) shift terms
         const int kk = f - 6;
@@ -932,31 +954,28 @@ __global__ void __launch_bounds__(RT, 1)
                                          gi[sidx(i, 1)] * d.dd[sidx(1, kk)] +
                                          gi[sidx(i, 2)] * d.dd[sidx(2, kk)]) +
                           (2.0 / 3.0) * cal[i] * db[kk];
-      } else if (f == 2) {
-        // ---------------- K: advection, KO, eq (8) -4/3 alpha gt^ij d_j K
-        const Derivs d = derivs<false>(s, c0, ih, ko_scale);
-        rK += advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
-        double gi[6];
-#pragma unroll
-        for (int r = 0; r < 6; ++r) gi[r] = SL(G_INV + r);
-#pragma unroll
-        for (int i = 0; i < 3; ++i)
-          SL(A_GT + i) += -(4.0 / 3.0) * alpha *
-                          (gi[sidx(i, 0)] * d.d1[0] + gi[sidx(i, 1)] * d.d1[1] +
-                           gi[sidx(i, 2)] * d.d1[2]);
-      } else if (f >= 18) {
-        const int q = f - 18;
-        const Derivs d = derivs<false>(s, c0, ih, ko_scale);
-        SL(A_AT + q) += advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
-      } else {  // 9..11: B
-        const int kk = f - 9;
-        const Derivs d = derivs<false>(s, c0, ih, ko_scale);
-        SL(A_B + kk) = advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
+      } else {
+        light_apply(s, f, derivs<false>(s, c0, ih, ko_scale));
       }
     }
     };
-    point_work(s, f);
-    if (FUSED && stB(st) >= 0) point_work(Tx + buf * STAGE_DBL, stB(st));
+    if (FUSED && !SOMM && stB(st) >= 0) {
+      // a pair of light fields: both fields' derivatives first (one straight
+      // line of 2 x 19 independent shared-memory loads, so the two fields'
+      // latency chains overlap), then each field's algebra in the pair order
+      // — the same arithmetic as two single stages
+      const int c0 = tab_c0[tid];
+      if (c0 >= 0) {
+        const double* sB = Tx + buf * STAGE_DBL;
+        const Derivs dA = derivs<false>(s, c0, ih, ko_scale);
+        const Derivs dB = derivs<false>(sB, c0, ih, ko_scale);
+        light_apply(s, f, dA);
+        light_apply(sB, stB(st), dB);
+      }
+    } else {
+      point_work(s, f);
+      if (FUSED && stB(st) >= 0) point_work(Tx + buf * STAGE_DBL, stB(st));
+    }
     __syncthreads();  // everyone is done with this stage buffer
     if (FUSED) {
       if (st + 2 < NST) {

@@ -36,11 +36,24 @@ constexpr int NPP = RT;   // slot stride in doubles: slots are indexed by thread
 // stages the A_AT slots hold gt^lm d_lm gt_ij (A_AT is first written by the
 // Christoffel block) and from the Christoffel block to the beta stages the A_B
 // slots hold CalGt^k (A_B is first written by the B stage).
+// DGR_TMEM_VALS (default): the point's read-only values gt_ij, At_ij and gt^ij
+// live in tensor memory (tm_* below) instead of 18 shared-memory slots.
+#ifndef DGR_TMEM_VALS
+#define DGR_TMEM_VALS 1
+#endif
+#if DGR_TMEM_VALS
+constexpr int A_GT = 0, A_BETA = 3, A_B = 6, A_GAM = 9, A_AT = 15;             // accumulators (21)
+constexpr int S0 = 21;                                                         // scratch (18)
+constexpr int NSLOT = 39;
+#else
 constexpr int V_GAM = 0, V_AT = 6;                                             // values (12)
 constexpr int A_GT = 12, A_BETA = 15, A_B = 18, A_GAM = 21, A_AT = 27;         // accumulators (21)
 constexpr int G_INV = 33;                                                      // gt^ij (6)
 constexpr int S0 = 39;                                                         // scratch (18)
 constexpr int NSLOT = 57;
+#endif
+// the point values' store: TV_GT gt_ij, TV_AT At_ij, TV_GI gt^ij (6 doubles each)
+enum { TV_GT = 0, TV_AT = 1, TV_GI = 2 };
 // first x-/y-derivatives of the staged field for the mixed second derivatives
 // (D_xy = D1_y D1_x, D_xz = D1_z D1_x, D_yz = D1_z D1_y), stored at the patch
 // index c = x + 13y + 169z minus an offset so thread reads stay conflict-free
@@ -49,7 +62,60 @@ constexpr int TY_OFF = 42, TY_N = 2113;   // x, y in 3..9, z in 0..12
 constexpr int T_N = 2 * STAGE_DBL;        // Tx + Ty, or two light-field stage halves
 static_assert(TX_N + TY_N <= T_N, "Tx/Ty fit the two pair halves");
 constexpr size_t SMEM_BYTES = size_t(NSLOT) * NPP * 8 + size_t(2) * STAGE_DBL * 8 +
-                              size_t(T_N) * 8 + 16 + size_t(2) * RT * 2;
+                              size_t(T_N) * 8 + 16 + size_t(2) * RT * 2 + 16;
+
+// Tensor memory as per-thread storage (tcgen05.ld / tcgen05.st, 32x32b shape:
+// each thread moves 32-bit columns of its own TMEM lane).  Warp w reaches lanes
+// 32 (w % 4) .. + 31 only, so the 11 warps share the 4 lane quarters and take
+// column blocks of TM_WCOLS by w / 4 (3 x 36 = 108 of TM_COLS allocated).
+// A double is two columns (low word first).  Loads complete at tcgen05.wait::ld
+// (its register operands tie the loaded values to the wait).
+constexpr int TM_COLS = 128, TM_WCOLS = 36;
+__device__ __forceinline__ void tm_ld6(uint32_t ta, double* v) {
+  uint32_t r[12];
+  asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+               : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]),
+                 "=r"(r[6]), "=r"(r[7])
+               : "r"(ta));
+  asm volatile("tcgen05.ld.sync.aligned.32x32b.x4.b32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11])
+               : "r"(ta + 8));
+  asm volatile("tcgen05.wait::ld.sync.aligned;"
+               : "+r"(r[0]), "+r"(r[1]), "+r"(r[2]), "+r"(r[3]), "+r"(r[4]), "+r"(r[5]),
+                 "+r"(r[6]), "+r"(r[7]), "+r"(r[8]), "+r"(r[9]), "+r"(r[10]), "+r"(r[11])
+               :
+               : "memory");
+#pragma unroll
+  for (int i = 0; i < 6; ++i) v[i] = __hiloint2double(int(r[2 * i + 1]), int(r[2 * i]));
+}
+__device__ __forceinline__ void tm_st6(uint32_t ta, const double* v) {
+  uint32_t r[12];
+#pragma unroll
+  for (int i = 0; i < 6; ++i) {
+    r[2 * i] = uint32_t(__double2loint(v[i]));
+    r[2 * i + 1] = uint32_t(__double2hiint(v[i]));
+  }
+  asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"r"(ta),
+               "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7])
+               : "memory");
+  asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1, %2, %3, %4};" ::"r"(ta + 8),
+               "r"(r[8]), "r"(r[9]), "r"(r[10]), "r"(r[11])
+               : "memory");
+}
+#if !DGR_TMEM_VALS
+__device__ __forceinline__ int vslot(int w) { return w == TV_GT ? V_GAM : (w == TV_AT ? V_AT : G_INV); }
+__device__ __forceinline__ void slots_ld6(const double* p, double* v) {
+#pragma unroll
+  for (int r = 0; r < 6; ++r) v[r] = p[r * NPP];
+}
+__device__ __forceinline__ void slots_st6(double* p, const double* v) {
+#pragma unroll
+  for (int r = 0; r < 6; ++r) p[r * NPP] = v[r];
+}
+#endif
+__device__ __forceinline__ void tm_st_wait() {
+  asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+}
 
 // thread -> interior point map (filled by upload_rhs_tables): every warp holds
 // at most two points per residue of their stage-buffer index mod 16, so its
@@ -138,6 +204,7 @@ __device__ __forceinline__ void cp_async_wait1() {
 // extrapolation rows l_m(-(t+1)), t = 0..2 (reading R12; host-computed, api.cu)
 __constant__ double c_rWEXT[3 * 7];
 constexpr int GJ = (NPATCH + RT - 1) / RT;   // gather points per thread (7)
+constexpr int C_CENTRE = 6 + 13 * 6 + 169 * 6;   // patch centre (threads without a point)
 
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   uint32_t ok = 0;
@@ -337,6 +404,7 @@ __global__ void __launch_bounds__(RT, 1)
   // in shared memory and re-read where needed (cheaper than a register spill)
   int16_t* tab_c0 = reinterpret_cast<int16_t*>(bars + 2);
   int16_t* tab_p = tab_c0 + RT;
+  uint32_t* tm_base = reinterpret_cast<uint32_t*>(tab_p + RT);   // TMEM allocation address
 
   const int tid = threadIdx.x;
   {
@@ -407,7 +475,25 @@ __global__ void __launch_bounds__(RT, 1)
     mbar_init(&bars[0], 1);
     mbar_init(&bars[1], 1);
   }
+#if DGR_TMEM_VALS
+  if (tid < 32) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tm_base)),
+                 "n"(TM_COLS)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
   __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  // this thread's TMEM address (lane quarter of its warp, column block)
+  const uint32_t tma = *tm_base + (uint32_t(32 * ((tid >> 5) & 3)) << 16) + TM_WCOLS * (tid >> 7);
+#define VALS_LD(w, v) tm_ld6(tma + 12 * (w), v)
+#define VALS_ST(w, v) tm_st6(tma + 12 * (w), v)
+#else
+  __syncthreads();
+#define VALS_LD(w, v) slots_ld6(slots + vslot(w) * NPP + tid, v)
+#define VALS_ST(w, v) slots_st6(slots + vslot(w) * NPP + tid, v)
+#endif
   if (FUSED) {
     load_gidx(e);
     gather_stage(0, 0);
@@ -424,10 +510,13 @@ __global__ void __launch_bounds__(RT, 1)
   e = ol[li];
   const int en = li + int(gridDim.x) < count ? ol[li + gridDim.x] : -1;   // next octant of this CTA
   const double* pbase = patches + int64_t(e) * (FUSED ? NPT : PATCH_PITCH);
+  // (threads without a point — 9 of 352 — run the same code on the patch
+  // centre / element node 0 and store nothing: TMEM accesses are warp-wide)
   const bool active = tab_c0[tid] >= 0;
   // the point's own values: patch index c0 of the staged patches, or (FUSED)
   // element node p of u / a hanging-node slot through o2s
-  const int cv = FUSED ? __ldg(m.o2s + int64_t(e) * NPT + max(int(tab_p[tid]), 0)) : tab_c0[tid];
+  const int cv = FUSED ? __ldg(m.o2s + int64_t(e) * NPT + max(int(tab_p[tid]), 0))
+                       : (active ? int(tab_c0[tid]) : C_CENTRE);
   auto own = [&](int f) -> double {
     if (!FUSED) return __ldg(pbase + f * fstride + cv);
     return cv < ds ? __ldg(patches + f * fstride + cv) : __ldg(m.aux + f * m.aux_stride + (cv - ds));
@@ -460,7 +549,7 @@ __global__ void __launch_bounds__(RT, 1)
   }
 
   // ---- values at the point (patch interior) -------------------------------
-  if (PRE && active) {
+  if (PRE) {
     // metric pre-pass results -> d gt (S0), gt^lm d_lm gt (A_AT), adv + KO of gt
     // (A_GAM) slots, asynchronously, in flight while the values are read
     // (pre rows are indexed by thread, [c][n_owned][RT]: coalesced)
@@ -475,32 +564,38 @@ __global__ void __launch_bounds__(RT, 1)
     }
     cp_async_commit();
   }
-  double alpha = 0, chi = 0, Kv = 0, beta[3] = {0, 0, 0};
-  if (active) {
+  double alpha, chi, Kv, beta[3];
+  {
     alpha = own(0);
     chi = own(1);
     Kv = own(2);
 #pragma unroll
     for (int i = 0; i < 3; ++i) beta[i] = own(6 + i);
-    double g[6];
+    double g[6], at[6];
 #pragma unroll
     for (int q = 0; q < 6; ++q) {
       g[q] = own(12 + q);
-      SL(V_GAM + q) = g[q];
-      SL(V_AT + q) = own(18 + q);
+      at[q] = own(18 + q);
     }
+    VALS_ST(TV_GT, g);
+    VALS_ST(TV_AT, at);
     // inverse metric by adjugate / determinant
     const double a00 = g[3] * g[5] - g[4] * g[4];
     const double a01 = g[2] * g[4] - g[1] * g[5];
     const double a02 = g[1] * g[4] - g[2] * g[3];
     const double det = g[0] * a00 + g[1] * a01 + g[2] * a02;
     const double idet = 1.0 / det;
-    SL(G_INV + 0) = a00 * idet;
-    SL(G_INV + 1) = a01 * idet;
-    SL(G_INV + 2) = a02 * idet;
-    SL(G_INV + 3) = (g[0] * g[5] - g[2] * g[2]) * idet;
-    SL(G_INV + 4) = (g[1] * g[2] - g[0] * g[4]) * idet;
-    SL(G_INV + 5) = (g[0] * g[3] - g[1] * g[1]) * idet;
+    double gi[6];
+    gi[0] = a00 * idet;
+    gi[1] = a01 * idet;
+    gi[2] = a02 * idet;
+    gi[3] = (g[0] * g[5] - g[2] * g[2]) * idet;
+    gi[4] = (g[1] * g[2] - g[0] * g[4]) * idet;
+    gi[5] = (g[0] * g[3] - g[1] * g[1]) * idet;
+    VALS_ST(TV_GI, gi);
+#if DGR_TMEM_VALS
+    tm_st_wait();
+#endif
 #pragma unroll
     for (int q = 0; q < 6; ++q) SL(A_GT + q) = 0.0;     // A_GT, A_BETA
     if (!PRE) {
@@ -520,11 +615,8 @@ __global__ void __launch_bounds__(RT, 1)
   auto christoffel = [&](const double* gi) {
       // ---------------- Christoffel block (eqs 12, 17; readings R1, R7)
       double gt[6], At[6];
-#pragma unroll
-      for (int r = 0; r < 6; ++r) {
-        gt[r] = SL(V_GAM + r);
-        At[r] = SL(V_AT + r);
-      }
+      VALS_LD(TV_GT, gt);
+      VALS_LD(TV_AT, At);
       double C[3][6];  // first kind C_k,ij = 1/2 (d_i g_kj + d_j g_ki - d_k g_ij)
 #pragma unroll
       for (int k = 0; k < 3; ++k)
@@ -621,13 +713,12 @@ __global__ void __launch_bounds__(RT, 1)
 #ifdef DGR_RHS_TIMING
   long long t_last = clock64();
 #endif
-  if (PRE && active) {
+  if (PRE) {
     // the metric pre-pass results for this point (copies issued before the
     // point's values were read), then the Christoffel block
     asm volatile("cp.async.wait_all;" ::: "memory");
     double gi[6];
-#pragma unroll
-    for (int r = 0; r < 6; ++r) gi[r] = SL(G_INV + r);
+    VALS_LD(TV_GI, gi);
     christoffel(gi);
   }
   for (int st = 0; st < NST; ++st, ++g) {
@@ -730,17 +821,14 @@ __global__ void __launch_bounds__(RT, 1)
     // the per-point work of a first-derivative-only ("light") field f from its
     // derivatives d (s: its staged patch, which the lopsided advection reads)
     auto light_apply = [&](const double* __restrict__ s, const int f, const Derivs& d) {
-      const int c0 = tab_c0[tid];
+      const int c0 = active ? int(tab_c0[tid]) : C_CENTRE;
       if (f >= 3 && f <= 5) {
         // ---------------- Gt^k: Ricci d Gt term, advection + KO kept apart (eq 3)
         const int kk = f - 3;
         SL(S0 + kk) = advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
         double gi[6], gt[6], Rg[6];
-#pragma unroll
-        for (int r = 0; r < 6; ++r) {
-          gi[r] = SL(G_INV + r);
-          gt[r] = SL(V_GAM + r);
-        }
+        VALS_LD(TV_GI, gi);
+        VALS_LD(TV_GT, gt);
 #pragma unroll
         for (int i = 0; i < 3; ++i)
 #pragma unroll
@@ -760,8 +848,7 @@ __global__ void __launch_bounds__(RT, 1)
         // ---------------- K: advection, KO, eq (8) -4/3 alpha gt^ij d_j K
         rK += advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
         double gi[6];
-#pragma unroll
-        for (int r = 0; r < 6; ++r) gi[r] = SL(G_INV + r);
+        VALS_LD(TV_GI, gi);
 #pragma unroll
         for (int i = 0; i < 3; ++i)
           SL(A_GT + i) += -(4.0 / 3.0) * alpha *
@@ -778,7 +865,7 @@ __global__ void __launch_bounds__(RT, 1)
     // the per-point work of one staged field f (patch in s); a pair stage runs
     // it for both fields, in order
     auto point_work = [&](const double* __restrict__ s, const int f) {
-    const int c0 = tab_c0[tid];
+    const int c0 = active ? int(tab_c0[tid]) : C_CENTRE;
     if (SOMM && bpt) {
       // radiative condition d_t f = -(x^i/r) d_i f - (f - f_inf)/r replaces the
       // whole right-hand side of field f here (the epilogue skips this point)
@@ -800,14 +887,13 @@ __global__ void __launch_bounds__(RT, 1)
       const double ir = 1.0 / sqrt(r2);
       rhs_oct[int64_t(f) * no * NPT + int64_t(e) * NPT + q] = -xr * ir - (s[c0] - finf) * ir;
     }
-    if (c0 >= 0) {
+    {
       if (!PRE && f >= 12 && f <= 17) {
         // ---------------- conformal metric gt_q: d gt, gt^lm d_lm gt, adv, KO
         const int q = f - 12;
         const Derivs d = derivs2(s, Tx, Ty, c0, ih, ko_scale);
         double gi[6];
-#pragma unroll
-        for (int r = 0; r < 6; ++r) gi[r] = SL(G_INV + r);
+        VALS_LD(TV_GI, gi);
 #pragma unroll
         for (int k = 0; k < 3; ++k) SL(S0 + k * 6 + q) = d.d1[k];
         SL(A_AT + q) = trace6(gi, d.dd);   // (A_AT slot reused until the Christoffel block)
@@ -817,12 +903,9 @@ __global__ void __launch_bounds__(RT, 1)
         // ---------------- chi: advection, KO, R^chi (eq 18-19), eq (8) chi term
         const Derivs d = derivs2(s, Tx, Ty, c0, ih, ko_scale);
         double gi[6], At[6], gt[6];
-#pragma unroll
-        for (int r = 0; r < 6; ++r) {
-          gi[r] = SL(G_INV + r);
-          At[r] = SL(V_AT + r);
-          gt[r] = SL(V_GAM + r);
-        }
+        VALS_LD(TV_GI, gi);
+        VALS_LD(TV_AT, At);
+        VALS_LD(TV_GT, gt);
 #pragma unroll
         for (int k = 0; k < 3; ++k) dchi[k] = d.d1[k];
         rC += advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
@@ -857,12 +940,9 @@ __global__ void __launch_bounds__(RT, 1)
         // ---------------- alpha: advection, KO, D_i D_j alpha (eqs 13-15)
         const Derivs d = derivs2(s, Tx, Ty, c0, ih, ko_scale);
         double gi[6], At[6], gt[6];
-#pragma unroll
-        for (int r = 0; r < 6; ++r) {
-          gi[r] = SL(G_INV + r);
-          At[r] = SL(V_AT + r);
-          gt[r] = SL(V_GAM + r);
-        }
+        VALS_LD(TV_GI, gi);
+        VALS_LD(TV_AT, At);
+        VALS_LD(TV_GT, gt);
         const double* da = d.d1;
         rA += advect<UPW>(s, c0, beta, da, ih) + d.ko;
         // gt^kl d_l chi d_k alpha
@@ -905,8 +985,7 @@ __global__ void __launch_bounds__(RT, 1)
         const double* db = d.d1;   // d_j beta^kk
         SL(A_BETA + kk) += advect<UPW>(s, c0, beta, db, ih) + d.ko;
         double gi[6], cal[3];
-#pragma unroll
-        for (int r = 0; r < 6; ++r) gi[r] = SL(G_INV + r);
+        VALS_LD(TV_GI, gi);
 #pragma unroll
         for (int k = 0; k < 3; ++k) cal[k] = SL(A_B + k);
         // Lie derivative terms of gt and At (eq 10, w = -2/3) need all of d_j beta^k:
@@ -926,11 +1005,9 @@ __global__ void __launch_bounds__(RT, 1)
           const double div = DB[0][0] + DB[1][1] + DB[2][2];
 #pragma unroll
           for (int t = 0; t < 2; ++t) {
-            const int vb = t == 0 ? V_GAM : V_AT;
             const int ab = t == 0 ? A_GAM : A_AT;
             double T[6];
-#pragma unroll
-            for (int r = 0; r < 6; ++r) T[r] = SL(vb + r);
+            VALS_LD(t == 0 ? TV_GT : TV_AT, T);
 #pragma unroll
             for (int i = 0; i < 3; ++i)
 #pragma unroll
@@ -964,8 +1041,8 @@ __global__ void __launch_bounds__(RT, 1)
       // line of 2 x 19 independent shared-memory loads, so the two fields'
       // latency chains overlap), then each field's algebra in the pair order
       // — the same arithmetic as two single stages
-      const int c0 = tab_c0[tid];
-      if (c0 >= 0) {
+      const int c0 = active ? int(tab_c0[tid]) : C_CENTRE;
+      {
         const double* sB = Tx + buf * STAGE_DBL;
         const Derivs dA = derivs<false>(s, c0, ih, ko_scale);
         const Derivs dB = derivs<false>(sB, c0, ih, ko_scale);
@@ -1013,16 +1090,14 @@ __global__ void __launch_bounds__(RT, 1)
 #endif
   // ---- epilogue: undifferentiated terms, combine, store ----------------------
   const int p = tab_p[tid];
-  if (tab_c0[tid] >= 0) {
-    double gi[6], At[6], B[3];
-#pragma unroll
-    for (int r = 0; r < 6; ++r) {
-      gi[r] = SL(G_INV + r);
-      At[r] = SL(V_AT + r);
-    }
-    const int cb = FUSED ? __ldg(m.o2s + int64_t(e) * NPT + p) : tab_c0[tid];
+  {
+    double gi[6], At[6], gtv[6], B[3];
+    VALS_LD(TV_GI, gi);
+    VALS_LD(TV_AT, At);
+    if (TF_ONCE) VALS_LD(TV_GT, gtv);
+    const int cb = FUSED ? __ldg(m.o2s + int64_t(e) * NPT + p) : (active ? int(tab_c0[tid]) : C_CENTRE);
     // (zip by the store: the DOF this point is the zip owner of, or -1)
-    const int dz = rhs_dof ? __ldg(m.own + int64_t(e) * NPT + p) : -1;
+    const int dz = rhs_dof && active ? __ldg(m.own + int64_t(e) * NPT + p) : -1;
 #pragma unroll
     for (int i = 0; i < 3; ++i)
       B[i] = !FUSED ? __ldg(pbase + (9 + i) * fstride + cb)
@@ -1061,7 +1136,7 @@ __global__ void __launch_bounds__(RT, 1)
         r[12 + q] = SL(A_GAM + q) - 2.0 * alpha * At[q];                          // (4)
         const double AAij = At[sidx(i, 0)] * Am[0][j] + At[sidx(i, 1)] * Am[1][j] +
                             At[sidx(i, 2)] * Am[2][j];
-        const double atf = TF_ONCE ? SL(A_AT + q) - SL(V_GAM + q) * ttr * (1.0 / 3.0) : SL(A_AT + q);
+        const double atf = TF_ONCE ? SL(A_AT + q) - gtv[q] * ttr * (1.0 / 3.0) : SL(A_AT + q);
         r[18 + q] = atf + alpha * (Kv * At[q] - 2.0 * AAij);                        // (6)
       }
     double* out = rhs_oct + int64_t(e) * NPT + p;
@@ -1071,13 +1146,22 @@ __global__ void __launch_bounds__(RT, 1)
 #pragma unroll
         for (int f = 0; f < NF; ++f) st_out(&rhs_dof[f * int64_t(m.dof_stride) + dz], r[f]);
       }
-    } else if (!SOMM || !bpt) {
+    } else if (active && (!SOMM || !bpt)) {
 #pragma unroll
       for (int f = 0; f < NF; ++f) out[f * ostr] = r[f];
     }
   }
   }  // octant loop
+#if DGR_TMEM_VALS
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  if (tid < 32)
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tm_base), "n"(TM_COLS)
+                 : "memory");
+#endif
 #undef SL
+#undef VALS_LD
+#undef VALS_ST
 }
 
 // ---------------------------------------------------------------------------

@@ -156,6 +156,16 @@ __device__ __forceinline__ int sidx(int i, int j) {
   return i <= j ? (i == 0 ? j : (i == 1 ? 2 + j : 5)) : (j == 0 ? i : (j == 1 ? 2 + i : 5));
 }
 
+// runtime-selected entries with compile-time array indices (a dynamically
+// indexed local array would live in local memory, i.e. in the L1 the gathers need)
+__device__ __forceinline__ double sel3(int k, double a, double b, double c) {
+  return k == 0 ? a : (k == 1 ? b : c);
+}
+// X_{k i} of a symmetric 3x3 matrix in sidx storage, k runtime, i compile-time
+__device__ __forceinline__ double row3(const double* X, int k, int i) {
+  return sel3(k, X[sidx(0, i)], X[sidx(1, i)], X[sidx(2, i)]);
+}
+
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
@@ -833,7 +843,7 @@ __global__ void __launch_bounds__(RT, 1)
         for (int i = 0; i < 3; ++i)
 #pragma unroll
           for (int j = i; j < 3; ++j)
-            Rg[sidx(i, j)] = 0.5 * (gt[sidx(kk, i)] * d.d1[j] + gt[sidx(kk, j)] * d.d1[i]);
+            Rg[sidx(i, j)] = 0.5 * (row3(gt, kk, i) * d.d1[j] + row3(gt, kk, j) * d.d1[i]);
         const double trR = trace6(gi, Rg);
         const double ca = chi * alpha;
         if (TF_ONCE) {
@@ -983,6 +993,7 @@ __global__ void __launch_bounds__(RT, 1)
         const int kk = f - 6;
         const Derivs d = derivs2(s, Tx, Ty, c0, ih, ko_scale);
         const double* db = d.d1;   // d_j beta^kk
+        const double dbk = sel3(kk, db[0], db[1], db[2]);   // d_kk beta^kk
         SL(A_BETA + kk) += advect<UPW>(s, c0, beta, db, ih) + d.ko;
         double gi[6], cal[3];
         VALS_LD(TV_GI, gi);
@@ -1021,16 +1032,16 @@ __global__ void __launch_bounds__(RT, 1)
               }
           }
         }
-        rC += -(2.0 / 3.0) * chi * db[kk];
+        rC += -(2.0 / 3.0) * chi * dbk;
         // Gt^kk += gt^jl d_jl beta^kk - CalGt^j d_j beta^kk
         SL(A_GT + kk) += trace6(gi, d.dd) - (cal[0] * db[0] + cal[1] * db[1] + cal[2] * db[2]);
         // Gt^i += 1/3 gt^ij d_j d_kk beta^kk + 2/3 CalGt^i d_kk beta^kk
 #pragma unroll
         for (int i = 0; i < 3; ++i)
-          SL(A_GT + i) += (1.0 / 3.0) * (gi[sidx(i, 0)] * d.dd[sidx(0, kk)] +
-                                         gi[sidx(i, 1)] * d.dd[sidx(1, kk)] +
-                                         gi[sidx(i, 2)] * d.dd[sidx(2, kk)]) +
-                          (2.0 / 3.0) * cal[i] * db[kk];
+          SL(A_GT + i) += (1.0 / 3.0) * (gi[sidx(i, 0)] * row3(d.dd, kk, 0) +
+                                         gi[sidx(i, 1)] * row3(d.dd, kk, 1) +
+                                         gi[sidx(i, 2)] * row3(d.dd, kk, 2)) +
+                          (2.0 / 3.0) * cal[i] * dbk;
       } else {
         light_apply(s, f, derivs<false>(s, c0, ih, ko_scale));
       }

@@ -157,7 +157,10 @@ __device__ __forceinline__ int sidx(int i, int j) {
 }
 
 // runtime-selected entries with compile-time array indices (a dynamically
-// indexed local array would live in local memory, i.e. in the L1 the gathers need)
+// indexed local array would live in local memory, i.e. in the L1 the gathers
+// need); products of selected entries are rounded explicitly (__dmul_rn /
+// __fma_rn) where they are used, so every kernel instantiation contracts them
+// the same way (fused == two-pass bit for bit)
 __device__ __forceinline__ double sel3(int k, double a, double b, double c) {
   return k == 0 ? a : (k == 1 ? b : c);
 }
@@ -273,7 +276,7 @@ __device__ __forceinline__ Derivs derivs(const double* __restrict__ s, int c, do
   d.d1[0] = lx.d1 * f1;
   d.d1[1] = ly.d1 * f1;
   d.d1[2] = lz.d1 * f1;
-  d.ko = (lx.ko + ly.ko + lz.ko) * ko_scale;
+  d.ko = __dmul_rn(lx.ko + ly.ko + lz.ko, ko_scale);
   if (SECOND) {
     const double f2 = ih * ih * (1.0 / 180.0);
     const double fm = ih * ih * (1.0 / 3600.0);
@@ -287,6 +290,8 @@ __device__ __forceinline__ Derivs derivs(const double* __restrict__ s, int c, do
   return d;
 }
 
+// (callers add the KO term with __dadd_rn and derivs* round it with __dmul_rn,
+// so no kernel instantiation fuses the two: fused == two-pass bit for bit)
 // advective derivative beta^k d_k f at patch index c: reading R9, the centred
 // D1 (d1 = its values); with upw (dgr_params.upwind, reading R9u) the 4th-order
 // lopsided stencil (-3 f_-1 - 10 f_0 + 18 f_1 - 6 f_2 + f_3) / (12 h) shifted
@@ -295,13 +300,17 @@ template <bool UPW>
 __device__ __forceinline__ double advect(const double* __restrict__ s, int c, const double* beta,
                                          const double* d1, double ih) {
   if (!UPW) return beta[0] * d1[0] + beta[1] * d1[1] + beta[2] * d1[2];
+  // (rounding pinned by explicit fma / mul: the sign selects would otherwise let
+  // different kernel instantiations contract differently)
   double a = 0.0;
 #pragma unroll
   for (int k = 0; k < 3; ++k) {
     const int st = k == 0 ? 1 : (k == 1 ? 13 : 169);
     const int q = beta[k] >= 0.0 ? st : -st;
-    const double e = -3.0 * s[c - q] - 10.0 * s[c] + 18.0 * s[c + q] - 6.0 * s[c + 2 * q] + s[c + 3 * q];
-    a += beta[k] * ((beta[k] >= 0.0 ? e : -e) * (ih * (1.0 / 12.0)));
+    const double e =
+        __fma_rn(-3.0, s[c - q],
+                 __fma_rn(-10.0, s[c], __fma_rn(18.0, s[c + q], __fma_rn(-6.0, s[c + 2 * q], s[c + 3 * q]))));
+    a = __fma_rn(beta[k], __dmul_rn(beta[k] >= 0.0 ? e : -e, ih * (1.0 / 12.0)), a);
   }
   return a;
 }
@@ -324,7 +333,7 @@ __device__ __forceinline__ Derivs derivs2(const double* __restrict__ s,
   d.d1[0] = lx.d1 * f1;
   d.d1[1] = ly.d1 * f1;
   d.d1[2] = lz.d1 * f1;
-  d.ko = (lx.ko + ly.ko + lz.ko) * ko_scale;
+  d.ko = __dmul_rn(lx.ko + ly.ko + lz.ko, ko_scale);
   const double f2 = ih * ih * (1.0 / 180.0);
   const double fm = ih * ih * (1.0 / 3600.0);
   d.dd[0] = lx.d2 * f2;
@@ -835,7 +844,7 @@ __global__ void __launch_bounds__(RT, 1)
       if (f >= 3 && f <= 5) {
         // ---------------- Gt^k: Ricci d Gt term, advection + KO kept apart (eq 3)
         const int kk = f - 3;
-        SL(S0 + kk) = advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
+        SL(S0 + kk) = __dadd_rn(advect<UPW>(s, c0, beta, d.d1, ih), d.ko);
         double gi[6], gt[6], Rg[6];
         VALS_LD(TV_GI, gi);
         VALS_LD(TV_GT, gt);
@@ -843,7 +852,7 @@ __global__ void __launch_bounds__(RT, 1)
         for (int i = 0; i < 3; ++i)
 #pragma unroll
           for (int j = i; j < 3; ++j)
-            Rg[sidx(i, j)] = 0.5 * (row3(gt, kk, i) * d.d1[j] + row3(gt, kk, j) * d.d1[i]);
+            Rg[sidx(i, j)] = 0.5 * (__dmul_rn(row3(gt, kk, i), d.d1[j]) + __dmul_rn(row3(gt, kk, j), d.d1[i]));
         const double trR = trace6(gi, Rg);
         const double ca = chi * alpha;
         if (TF_ONCE) {
@@ -856,7 +865,7 @@ __global__ void __launch_bounds__(RT, 1)
         }
       } else if (f == 2) {
         // ---------------- K: advection, KO, eq (8) -4/3 alpha gt^ij d_j K
-        rK += advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
+        rK += __dadd_rn(advect<UPW>(s, c0, beta, d.d1, ih), d.ko);
         double gi[6];
         VALS_LD(TV_GI, gi);
 #pragma unroll
@@ -866,10 +875,10 @@ __global__ void __launch_bounds__(RT, 1)
                            gi[sidx(i, 2)] * d.d1[2]);
       } else if (f >= 18) {
         const int q = f - 18;
-        SL(A_AT + q) += advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
+        SL(A_AT + q) += __dadd_rn(advect<UPW>(s, c0, beta, d.d1, ih), d.ko);
       } else {  // 9..11: B
         const int kk = f - 9;
-        SL(A_B + kk) = advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
+        SL(A_B + kk) = __dadd_rn(advect<UPW>(s, c0, beta, d.d1, ih), d.ko);
       }
     };
     // the per-point work of one staged field f (patch in s); a pair stage runs
@@ -907,7 +916,7 @@ __global__ void __launch_bounds__(RT, 1)
 #pragma unroll
         for (int k = 0; k < 3; ++k) SL(S0 + k * 6 + q) = d.d1[k];
         SL(A_AT + q) = trace6(gi, d.dd);   // (A_AT slot reused until the Christoffel block)
-        SL(A_GAM + q) += advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
+        SL(A_GAM + q) += __dadd_rn(advect<UPW>(s, c0, beta, d.d1, ih), d.ko);
         if (q == 5) christoffel(gi);
       } else if (f == 1) {
         // ---------------- chi: advection, KO, R^chi (eq 18-19), eq (8) chi term
@@ -918,7 +927,7 @@ __global__ void __launch_bounds__(RT, 1)
         VALS_LD(TV_GT, gt);
 #pragma unroll
         for (int k = 0; k < 3; ++k) dchi[k] = d.d1[k];
-        rC += advect<UPW>(s, c0, beta, d.d1, ih) + d.ko;
+        rC += __dadd_rn(advect<UPW>(s, c0, beta, d.d1, ih), d.ko);
         double Rc[6];
 #pragma unroll
         for (int i = 0; i < 3; ++i)
@@ -954,7 +963,7 @@ __global__ void __launch_bounds__(RT, 1)
         VALS_LD(TV_AT, At);
         VALS_LD(TV_GT, gt);
         const double* da = d.d1;
-        rA += advect<UPW>(s, c0, beta, da, ih) + d.ko;
+        rA += __dadd_rn(advect<UPW>(s, c0, beta, da, ih), d.ko);
         // gt^kl d_l chi d_k alpha
         double gdd = 0.0;
 #pragma unroll
@@ -994,7 +1003,7 @@ __global__ void __launch_bounds__(RT, 1)
         const Derivs d = derivs2(s, Tx, Ty, c0, ih, ko_scale);
         const double* db = d.d1;   // d_j beta^kk
         const double dbk = sel3(kk, db[0], db[1], db[2]);   // d_kk beta^kk
-        SL(A_BETA + kk) += advect<UPW>(s, c0, beta, db, ih) + d.ko;
+        SL(A_BETA + kk) += __dadd_rn(advect<UPW>(s, c0, beta, db, ih), d.ko);
         double gi[6], cal[3];
         VALS_LD(TV_GI, gi);
 #pragma unroll
@@ -1032,16 +1041,17 @@ __global__ void __launch_bounds__(RT, 1)
               }
           }
         }
-        rC += -(2.0 / 3.0) * chi * dbk;
+        rC = __fma_rn(-(2.0 / 3.0) * chi, dbk, rC);
         // Gt^kk += gt^jl d_jl beta^kk - CalGt^j d_j beta^kk
         SL(A_GT + kk) += trace6(gi, d.dd) - (cal[0] * db[0] + cal[1] * db[1] + cal[2] * db[2]);
         // Gt^i += 1/3 gt^ij d_j d_kk beta^kk + 2/3 CalGt^i d_kk beta^kk
 #pragma unroll
         for (int i = 0; i < 3; ++i)
-          SL(A_GT + i) += (1.0 / 3.0) * (gi[sidx(i, 0)] * row3(d.dd, kk, 0) +
-                                         gi[sidx(i, 1)] * row3(d.dd, kk, 1) +
-                                         gi[sidx(i, 2)] * row3(d.dd, kk, 2)) +
-                          (2.0 / 3.0) * cal[i] * dbk;
+          SL(A_GT + i) += __fma_rn(1.0 / 3.0,
+                                   __fma_rn(gi[sidx(i, 2)], row3(d.dd, kk, 2),
+                                            __fma_rn(gi[sidx(i, 1)], row3(d.dd, kk, 1),
+                                                     __dmul_rn(gi[sidx(i, 0)], row3(d.dd, kk, 0)))),
+                                   __dmul_rn((2.0 / 3.0) * cal[i], dbk));
       } else {
         light_apply(s, f, derivs<false>(s, c0, ih, ko_scale));
       }
@@ -1373,7 +1383,7 @@ __global__ void __launch_bounds__(RT, 2)
 #pragma unroll
         for (int k = 0; k < 3; ++k) st_out(&out[(6 * k + q) * ostr], d.d1[k]);
         st_out(&out[(18 + q) * ostr], trace6(gi, d.dd));
-        st_out(&out[(24 + q) * ostr], advect<UPW>(s, c0, beta, d.d1, ih) + d.ko);
+        st_out(&out[(24 + q) * ostr], __dadd_rn(advect<UPW>(s, c0, beta, d.d1, ih), d.ko));
       }
     }
   }

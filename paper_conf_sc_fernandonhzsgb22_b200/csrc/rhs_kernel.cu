@@ -21,6 +21,7 @@
 // first-kind symbol C_ijk itself (gt_il gt^lm C_mjk = C_ijk).
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <vector>
 
 #include "device.cuh"
@@ -62,7 +63,7 @@ constexpr int TY_OFF = 42, TY_N = 2113;   // x, y in 3..9, z in 0..12
 constexpr int T_N = 2 * STAGE_DBL;        // Tx + Ty, or two light-field stage halves
 static_assert(TX_N + TY_N <= T_N, "Tx/Ty fit the two pair halves");
 constexpr size_t SMEM_BYTES = size_t(NSLOT) * NPP * 8 + size_t(2) * STAGE_DBL * 8 +
-                              size_t(T_N) * 8 + 16 + size_t(2) * RT * 2 + 16;
+                              size_t(T_N) * 8 + 16 + size_t(3) * RT * 2 + 16;
 
 // Tensor memory as per-thread storage (tcgen05.ld / tcgen05.st, 32x32b shape:
 // each thread moves 32-bit columns of its own TMEM lane).  Warp w reaches lanes
@@ -127,9 +128,41 @@ __device__ int16_t g_perm[RT];
 __device__ long long g_stage_cycles[NF + 2];
 #endif
 
-// Lines of the cooperative D1 pass (register pencils, see the stage loop)
+// Lines of the cooperative D1 pass (register pencils): threads < N_TXL take
+// the x-lines of Tx (at the 133 (y, z) rows of the cross-shaped region: z in
+// 3..9 with all y, or y in 3..9 with z in {0,1,2,10,11,12}), the next N_TYL the
+// y-lines of Ty (x in 3..9, all z).  g_d1b[tid] is the line's first patch
+// index b, assigned on the host so that the lanes of every half-warp start in
+// distinct 8-byte bank pairs (b mod 16): each line's 13 loads and 7 stores are
+// then conflict-free (filled by upload_rhs_tables; -1: no line)
 constexpr int N_TXL = 13 * 7 + 7 * 6, N_TYL = 7 * 13;
 static_assert(N_TXL + N_TYL <= RT, "one pencil per thread");
+__device__ int16_t g_d1b[RT];
+
+// the D1 pass of the staged field s: Tx = D1_x s, Ty = D1_y s (raw numerators)
+// on the region the mixed stencils read (one 13-point line per thread, 20
+// shared-memory accesses per 7 values)
+__device__ __forceinline__ void d1_pass(const double* __restrict__ s, double* __restrict__ Tx,
+                                        double* __restrict__ Ty, int tid, const int16_t* tab_d1b) {
+  if (tid >= N_TXL + N_TYL) return;
+  const int b = tab_d1b[tid];
+  double v[13];
+  if (tid < N_TXL) {
+#pragma unroll
+    for (int k = 0; k < 13; ++k) v[k] = s[b + k];
+#pragma unroll
+    for (int x = 3; x <= 9; ++x)
+      Tx[b + x - TX_OFF] = (v[x + 1] - v[x - 1]) * 45.0 - (v[x + 2] - v[x - 2]) * 9.0 +
+                           (v[x + 3] - v[x - 3]);
+  } else {
+#pragma unroll
+    for (int k = 0; k < 13; ++k) v[k] = s[b + 13 * k];
+#pragma unroll
+    for (int y = 3; y <= 9; ++y)
+      Ty[b + 13 * y - TY_OFF] = (v[y + 1] - v[y - 1]) * 45.0 - (v[y + 2] - v[y - 2]) * 9.0 +
+                                (v[y + 3] - v[y - 3]);
+  }
+}
 
 // field processing order: the metric gt_ij (skipped after the pre-pass), then
 // the other fields with second derivatives (chi, alpha, beta^i: "heavy"),
@@ -423,7 +456,8 @@ __global__ void __launch_bounds__(RT, 1)
   // in shared memory and re-read where needed (cheaper than a register spill)
   int16_t* tab_c0 = reinterpret_cast<int16_t*>(bars + 2);
   int16_t* tab_p = tab_c0 + RT;
-  uint32_t* tm_base = reinterpret_cast<uint32_t*>(tab_p + RT);   // TMEM allocation address
+  int16_t* tab_d1b = tab_p + RT;                                  // D1-pass line (g_d1b)
+  uint32_t* tm_base = reinterpret_cast<uint32_t*>(tab_d1b + RT);  // TMEM allocation address
 
   const int tid = threadIdx.x;
   {
@@ -431,6 +465,7 @@ __global__ void __launch_bounds__(RT, 1)
     const int q = pp >= 0 ? pp : 0;
     tab_c0[tid] = pp >= 0 ? int16_t((q % 7 + 3) + 13 * ((q / 7) % 7 + 3) + 169 * (q / 49 + 3)) : -1;
     tab_p[tid] = int16_t(q);
+    tab_d1b[tid] = g_d1b[tid];
   }
   const int64_t no = m.n_owned;
   const int64_t fstride = FUSED ? m.dof_stride : no * PATCH_PITCH;
@@ -798,43 +833,9 @@ __global__ void __launch_bounds__(RT, 1)
     const bool second = f <= 1 || (f >= 6 && f <= 8) || (f >= 12 && f <= 17);
     if (second) {
       // cooperative first derivatives along x (and y) of the staged field on
-      // the extended region the mixed stencils need, by register pencils: each
-      // thread loads one 13-point line once and writes D1 at its 7 interior
-      // points (20 shared-memory accesses per 7 values instead of 49).
-      // Tx: lines along x at the 133 (y, z) rows of the cross-shaped region
-      // (z in 3..9 with all y, or y in 3..9 with z in {0,1,2,10,11,12});
-      // Ty: lines along y at x in 3..9, all z.  Consecutive lanes take rows
-      // 13 apart (Tx) or consecutive x (Ty), so loads and stores stay within
-      // two wavefronts per warp.
-      if (tid < N_TXL) {
-        int y, z;
-        if (tid < 91) {
-          z = 3 + tid / 13;
-          y = tid % 13;
-        } else {
-          const int r2 = tid - 91, zz = r2 / 7;
-          z = zz < 3 ? zz : zz + 7;
-          y = 3 + r2 % 7;
-        }
-        const int b = 13 * y + 169 * z;
-        double v[13];
-#pragma unroll
-        for (int k = 0; k < 13; ++k) v[k] = s[b + k];
-#pragma unroll
-        for (int x = 3; x <= 9; ++x)
-          Tx[b + x - TX_OFF] = (v[x + 1] - v[x - 1]) * 45.0 - (v[x + 2] - v[x - 2]) * 9.0 +
-                               (v[x + 3] - v[x - 3]);
-      } else if (tid < N_TXL + N_TYL) {
-        const int q = tid - N_TXL;
-        const int b = (3 + q % 7) + 169 * (q / 7);
-        double v[13];
-#pragma unroll
-        for (int k = 0; k < 13; ++k) v[k] = s[b + 13 * k];
-#pragma unroll
-        for (int y = 3; y <= 9; ++y)
-          Ty[b + 13 * y - TY_OFF] = (v[y + 1] - v[y - 1]) * 45.0 - (v[y + 2] - v[y - 2]) * 9.0 +
-                                    (v[y + 3] - v[y - 3]);
-      }
+      // the extended region the mixed stencils need (d1_pass: register
+      // pencils, one conflict-free 13-point line per thread)
+      d1_pass(s, Tx, Ty, tid, tab_d1b);
       __syncthreads();
     }
     // the per-point work of a first-derivative-only ("light") field f from its
@@ -1200,7 +1201,7 @@ __global__ void __launch_bounds__(RT, 1)
 constexpr int NPRE = 30;
 constexpr int PRE_NBUF = 3;   // stage ring depth of the pre-pass
 constexpr size_t PRE_SMEM_BYTES = size_t(PRE_NBUF) * STAGE_DBL * 8 + size_t(TX_N + TY_N) * 8 +
-                                  size_t(2) * RT * 2;
+                                  size_t(3) * RT * 2;
 
 // Fused path only (patches gathered from u and the slots).  Three-deep stage
 // ring: the CTA barrier that releases stage g's data also proves every thread
@@ -1216,12 +1217,14 @@ __global__ void __launch_bounds__(RT, 2)
   double* Ty = Tx + TX_N;                         // [TY_N]
   int16_t* tab_c0 = reinterpret_cast<int16_t*>(Ty + TY_N);
   int16_t* tab_p = tab_c0 + RT;
+  int16_t* tab_d1b = tab_p + RT;
   const int tid = threadIdx.x;
   {
     const int pp = g_perm[tid];
     const int q = pp >= 0 ? pp : 0;
     tab_c0[tid] = pp >= 0 ? int16_t((q % 7 + 3) + 13 * ((q / 7) % 7 + 3) + 169 * (q / 49 + 3)) : -1;
     tab_p[tid] = int16_t(q);
+    tab_d1b[tid] = g_d1b[tid];
   }
   const int64_t no = m.n_owned;
   const int64_t fstride = m.dof_stride;
@@ -1348,35 +1351,7 @@ __global__ void __launch_bounds__(RT, 2)
       }
       const double* s = sw;
       // cooperative D1 pass (as in k_rhs)
-      if (tid < N_TXL) {
-        int y, z;
-        if (tid < 91) {
-          z = 3 + tid / 13;
-          y = tid % 13;
-        } else {
-          const int r2 = tid - 91, zz = r2 / 7;
-          z = zz < 3 ? zz : zz + 7;
-          y = 3 + r2 % 7;
-        }
-        const int b = 13 * y + 169 * z;
-        double v[13];
-#pragma unroll
-        for (int k = 0; k < 13; ++k) v[k] = s[b + k];
-#pragma unroll
-        for (int x = 3; x <= 9; ++x)
-          Tx[b + x - TX_OFF] = (v[x + 1] - v[x - 1]) * 45.0 - (v[x + 2] - v[x - 2]) * 9.0 +
-                               (v[x + 3] - v[x - 3]);
-      } else if (tid < N_TXL + N_TYL) {
-        const int qq = tid - N_TXL;
-        const int b = (3 + qq % 7) + 169 * (qq / 7);
-        double v[13];
-#pragma unroll
-        for (int k = 0; k < 13; ++k) v[k] = s[b + 13 * k];
-#pragma unroll
-        for (int y = 3; y <= 9; ++y)
-          Ty[b + 13 * y - TY_OFF] = (v[y + 1] - v[y - 1]) * 45.0 - (v[y + 2] - v[y - 2]) * 9.0 +
-                                    (v[y + 3] - v[y - 3]);
-      }
+      d1_pass(s, Tx, Ty, tid, tab_d1b);
       __syncthreads();
       if (c0 >= 0) {
         const Derivs d = derivs2(s, Tx, Ty, c0, ih, ko_scale);
@@ -1421,6 +1396,42 @@ void upload_rhs_tables(const double* wext) {
       if (next[r] < bucket[r].size()) perm[w * 32 + lane] = int16_t(bucket[r][next[r]++]);
     }
   cudaMemcpyToSymbol(g_perm, perm, sizeof(perm));
+  // D1-pass lines: per kind, fill each half-warp with lines of distinct b mod 16
+  // (greedy, the most frequent residues first)
+  int16_t d1b[RT];
+  for (int t = 0; t < RT; ++t) d1b[t] = -1;
+  std::vector<int> lx, ly;
+  for (int z = 3; z <= 9; ++z)
+    for (int y = 0; y < 13; ++y) lx.push_back(13 * y + 169 * z);
+  for (int z = 0; z < 13; ++z)
+    if (z < 3 || z > 9)
+      for (int y = 3; y <= 9; ++y) lx.push_back(13 * y + 169 * z);
+  for (int z = 0; z < 13; ++z)
+    for (int x = 3; x <= 9; ++x) ly.push_back(x + 169 * z);
+  auto assign = [&](std::vector<int>& lines, int t0, int t1) {
+    std::vector<std::vector<int>> byres(16);
+    for (int b : lines) byres[b % 16].push_back(b);
+    for (int h = t0; h < t1;) {
+      const int he = std::min(t1, (h / 16 + 1) * 16);   // the part of this half-warp in [t0, t1)
+      bool used[16] = {false};
+      for (int t = h; t < he; ++t) {
+        int best = -1;
+        for (int r = 0; r < 16; ++r)
+          if (!used[r] && !byres[r].empty() && (best < 0 || byres[r].size() > byres[best].size()))
+            best = r;
+        if (best < 0)   // every residue left is taken in this half-warp: any line
+          for (int r = 0; r < 16; ++r)
+            if (!byres[r].empty() && (best < 0 || byres[r].size() > byres[best].size())) best = r;
+        used[best] = true;
+        d1b[t] = int16_t(byres[best].back());
+        byres[best].pop_back();
+      }
+      h = he;
+    }
+  };
+  assign(lx, 0, N_TXL);
+  assign(ly, N_TXL, N_TXL + N_TYL);
+  cudaMemcpyToSymbol(g_d1b, d1b, sizeof(d1b));
 }
 
 template <bool U>

@@ -33,28 +33,19 @@ namespace {
 constexpr int RT = 352;   // threads (11 warps); 343 interior points
 constexpr int NPP = RT;   // slot stride in doubles: slots are indexed by thread
 
-// shared-memory slot map ([slot][NPP] doubles).  Slot reuse: during the gt
-// stages the A_AT slots hold gt^lm d_lm gt_ij (A_AT is first written by the
-// Christoffel block) and from the Christoffel block to the beta stages the A_B
-// slots hold CalGt^k (A_B is first written by the B stage).
-// DGR_TMEM_VALS (default): the point's read-only values gt_ij, At_ij and gt^ij
-// live in tensor memory (tm_* below) instead of 18 shared-memory slots.
-#ifndef DGR_TMEM_VALS
-#define DGR_TMEM_VALS 1
-#endif
-#if DGR_TMEM_VALS
+// shared-memory slot map ([slot][NPP] doubles, indexed by thread).  Slot
+// reuse: during the gt stages the A_AT slots hold gt^lm d_lm gt_ij (A_AT is
+// first written by the Christoffel block) and from the Christoffel block to the
+// beta stages the A_B slots hold CalGt^k (A_B is first written by the B stage).
 constexpr int A_GT = 0, A_BETA = 3, A_B = 6, A_GAM = 9, A_AT = 15;             // accumulators (21)
 constexpr int S0 = 21;                                                         // scratch (18)
 constexpr int NSLOT = 39;
-#else
-constexpr int V_GAM = 0, V_AT = 6;                                             // values (12)
-constexpr int A_GT = 12, A_BETA = 15, A_B = 18, A_GAM = 21, A_AT = 27;         // accumulators (21)
-constexpr int G_INV = 33;                                                      // gt^ij (6)
-constexpr int S0 = 39;                                                         // scratch (18)
-constexpr int NSLOT = 57;
-#endif
-// the point values' store: TV_GT gt_ij, TV_AT At_ij, TV_GI gt^ij (6 doubles each)
-enum { TV_GT = 0, TV_AT = 1, TV_GI = 2 };
+// The point's read-only values live in tensor memory (tm_* below; DESIGN.md
+// §7: a thread's TMEM lane is a private store outside the shared-memory data
+// pipe), 6 doubles per block: TV_GT gt_ij, TV_AT At_ij, TV_GI gt^ij, TV_EX the
+// epilogue's B^i (3) and the DOF this point is the zip owner of (bits of a
+// double), loaded with the other values in the prologue.
+enum { TV_GT = 0, TV_AT = 1, TV_GI = 2, TV_EX = 3 };
 // first x-/y-derivatives of the staged field for the mixed second derivatives
 // (D_xy = D1_y D1_x, D_xz = D1_z D1_x, D_yz = D1_z D1_y), stored at the patch
 // index c = x + 13y + 169z minus an offset so thread reads stay conflict-free
@@ -68,10 +59,10 @@ constexpr size_t SMEM_BYTES = size_t(NSLOT) * NPP * 8 + size_t(2) * STAGE_DBL * 
 // Tensor memory as per-thread storage (tcgen05.ld / tcgen05.st, 32x32b shape:
 // each thread moves 32-bit columns of its own TMEM lane).  Warp w reaches lanes
 // 32 (w % 4) .. + 31 only, so the 11 warps share the 4 lane quarters and take
-// column blocks of TM_WCOLS by w / 4 (3 x 36 = 108 of TM_COLS allocated).
+// column blocks of TM_WCOLS by w / 4 (3 x 48 = 144 of TM_COLS allocated).
 // A double is two columns (low word first).  Loads complete at tcgen05.wait::ld
 // (its register operands tie the loaded values to the wait).
-constexpr int TM_COLS = 128, TM_WCOLS = 36;
+constexpr int TM_COLS = 256, TM_WCOLS = 48;
 __device__ __forceinline__ void tm_ld6(uint32_t ta, double* v) {
   uint32_t r[12];
   asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
@@ -103,17 +94,6 @@ __device__ __forceinline__ void tm_st6(uint32_t ta, const double* v) {
                "r"(r[8]), "r"(r[9]), "r"(r[10]), "r"(r[11])
                : "memory");
 }
-#if !DGR_TMEM_VALS
-__device__ __forceinline__ int vslot(int w) { return w == TV_GT ? V_GAM : (w == TV_AT ? V_AT : G_INV); }
-__device__ __forceinline__ void slots_ld6(const double* p, double* v) {
-#pragma unroll
-  for (int r = 0; r < 6; ++r) v[r] = p[r * NPP];
-}
-__device__ __forceinline__ void slots_st6(double* p, const double* v) {
-#pragma unroll
-  for (int r = 0; r < 6; ++r) p[r * NPP] = v[r];
-}
-#endif
 __device__ __forceinline__ void tm_st_wait() {
   asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
 }
@@ -529,7 +509,6 @@ __global__ void __launch_bounds__(RT, 1)
     mbar_init(&bars[0], 1);
     mbar_init(&bars[1], 1);
   }
-#if DGR_TMEM_VALS
   if (tid < 32) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tm_base)),
                  "n"(TM_COLS)
@@ -543,11 +522,7 @@ __global__ void __launch_bounds__(RT, 1)
   const uint32_t tma = *tm_base + (uint32_t(32 * ((tid >> 5) & 3)) << 16) + TM_WCOLS * (tid >> 7);
 #define VALS_LD(w, v) tm_ld6(tma + 12 * (w), v)
 #define VALS_ST(w, v) tm_st6(tma + 12 * (w), v)
-#else
-  __syncthreads();
-#define VALS_LD(w, v) slots_ld6(slots + vslot(w) * NPP + tid, v)
-#define VALS_ST(w, v) slots_st6(slots + vslot(w) * NPP + tid, v)
-#endif
+
   if (FUSED) {
     load_gidx(e);
     gather_stage(0, 0);
@@ -633,6 +608,12 @@ __global__ void __launch_bounds__(RT, 1)
     }
     VALS_ST(TV_GT, g);
     VALS_ST(TV_AT, at);
+    {
+      // the epilogue's B^i and zip-owner DOF, in flight with the values above
+      const int dz = rhs_dof && active ? __ldg(m.own + int64_t(e) * NPT + max(int(tab_p[tid]), 0)) : -1;
+      const double ex[6] = {own(9), own(10), own(11), __hiloint2double(0, dz), 0.0, 0.0};
+      VALS_ST(TV_EX, ex);
+    }
     // inverse metric by adjugate / determinant
     const double a00 = g[3] * g[5] - g[4] * g[4];
     const double a01 = g[2] * g[4] - g[1] * g[5];
@@ -647,9 +628,7 @@ __global__ void __launch_bounds__(RT, 1)
     gi[4] = (g[1] * g[2] - g[0] * g[4]) * idet;
     gi[5] = (g[0] * g[3] - g[1] * g[1]) * idet;
     VALS_ST(TV_GI, gi);
-#if DGR_TMEM_VALS
     tm_st_wait();
-#endif
 #pragma unroll
     for (int q = 0; q < 6; ++q) SL(A_GT + q) = 0.0;     // A_GT, A_BETA
     if (!PRE) {
@@ -1117,14 +1096,13 @@ __global__ void __launch_bounds__(RT, 1)
     VALS_LD(TV_GI, gi);
     VALS_LD(TV_AT, At);
     if (TF_ONCE) VALS_LD(TV_GT, gtv);
-    const int cb = FUSED ? __ldg(m.o2s + int64_t(e) * NPT + p) : (active ? int(tab_c0[tid]) : C_CENTRE);
+    double ex[6];
+    VALS_LD(TV_EX, ex);
     // (zip by the store: the DOF this point is the zip owner of, or -1)
-    const int dz = rhs_dof && active ? __ldg(m.own + int64_t(e) * NPT + p) : -1;
+    const int dz = __double2loint(ex[3]);
 #pragma unroll
     for (int i = 0; i < 3; ++i)
-      B[i] = !FUSED ? __ldg(pbase + (9 + i) * fstride + cb)
-                    : (cb < ds ? __ldg(patches + (9 + i) * fstride + cb)
-                               : __ldg(m.aux + (9 + i) * m.aux_stride + (cb - ds)));
+      B[i] = ex[i];
     // At^k_j and At_ik At^k_j, At_ij At^ij
     double Am[3][3];
 #pragma unroll
@@ -1174,13 +1152,11 @@ __global__ void __launch_bounds__(RT, 1)
     }
   }
   }  // octant loop
-#if DGR_TMEM_VALS
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
   __syncthreads();
   if (tid < 32)
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tm_base), "n"(TM_COLS)
                  : "memory");
-#endif
 #undef SL
 #undef VALS_LD
 #undef VALS_ST

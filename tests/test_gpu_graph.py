@@ -43,3 +43,26 @@ def test_graph_step_bit_identical(cfgf):
     torch.cuda.synchronize()
     assert torch.equal(c, d)
     assert np.isfinite(c.cpu().numpy()).all()
+
+
+@pytest.mark.parametrize("cfgf", [configs.c1_uniform, lambda: configs.small_bbh(lmax=6, rho=0.5)])
+def test_rhs_repeatable(cfgf):
+    """Race check in lieu of compute-sanitizer (closed on this GPU pool in
+    round 3): the RHS (k_interp, k_gt_pre, k_rhs with its tensor-memory value
+    store and threads without a point, zip by store) and the RK4 step are
+    bitwise repeatable over calls, for the default and the upwind kernels."""
+    need_gpu()
+    cfg = cfgf()
+    m = dgr.Mesh(cfg)
+    xyz = m.dof_xyz_host()
+    u = to_dev(initial.for_config(cfg, xyz, kind="random", seed=9), m.dof_stride)
+    dt = 0.25 * m.info["h_min"]
+    for prm in (None, dgr.Params(upwind=1)):
+        r0 = m.rhs(u, prm=prm).clone()
+        s0 = u.clone()
+        m.rk4_step(s0, dt, prm=prm)
+        for _ in range(4):
+            assert torch.equal(m.rhs(u, prm=prm), r0)
+            s1 = u.clone()
+            m.rk4_step(s1, dt, prm=prm)
+            assert torch.equal(s1, s0)

@@ -376,8 +376,17 @@ dgr_status dgr_group_destroy(dgr_group g);
  *     graph on `stream` (one launch instead of 16+).  Changing any option or
  *     the arguments re-captures.  Not used while profiling (dgr_profile_enable)
  *     or on NCCL meshes.  Bit-identical to the eager sequence. */
+/*   DGR_OPT_FUSE_RK4 (default 1): dgr_rk4_step and dgr_rk4_step_host apply the
+ *     RK4 stage update (Alg. 1 l.9-10, classic tableau) in the RHS kernel's
+ *     zip-by-store epilogue — each zip owner updates its DOF's stage state and
+ *     accumulator (or the new state) instead of storing the RHS, the u_n /
+ *     accumulator rows prefetched into L2 two field stages ahead — with stage
+ *     states alternating between two library buffers; 0 = the RHS in DOF order,
+ *     then a streaming update kernel.  Fused path with zip by store only;
+ *     dgr_rk4_stage and the rank group always use the separate update.
+ *     Bit-identical. */
 enum { DGR_OPT_FUSED_UNZIP = 1, DGR_OPT_PHASES = 2, DGR_OPT_PREPASS = 3, DGR_OPT_ZIP_STORE = 4,
-       DGR_OPT_GRAPH = 5 };
+       DGR_OPT_GRAPH = 5, DGR_OPT_FUSE_RK4 = 7 };
 dgr_status dgr_set_option(dgr_mesh m, int option, int64_t value);
 
 /* Device-side timing helper for benchmarks: number of kernel launches the last

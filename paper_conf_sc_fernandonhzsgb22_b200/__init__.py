@@ -28,6 +28,7 @@ MAP_OCTANTS, MAP_O2N, MAP_HANGING, MAP_PAD_SRC, MAP_PAD_KIND, MAP_ZIP = 0, 1, 2,
 MAP_DOF_GID, MAP_DOF_XYZ, MAP_SEND, MAP_SEND_COUNTS, MAP_RECV_COUNTS = 6, 7, 8, 9, 10
 MAP_LOCAL_OCTS, MAP_O2N_LOCAL, MAP_RHS_ORDER, MAP_SENDBUF = 11, 12, 13, 14
 OPT_FUSED_UNZIP, OPT_PHASES, OPT_PREPASS, OPT_ZIP_STORE, OPT_GRAPH = 1, 2, 3, 4, 5
+OPT_FUSE_RK4 = 7
 
 
 class DgrError(RuntimeError):
@@ -474,6 +475,11 @@ class Mesh:
         """DGR_OPT_GRAPH: rk4_step replays a CUDA graph of its four stages (captured
         at the second call with the same arguments); bit-identical to eager."""
         _check(lib().dgr_set_option(self._h, OPT_GRAPH, int(bool(on))))
+
+    def set_fuse_rk4(self, on=True):
+        """DGR_OPT_FUSE_RK4: rk4_step / rk4_step_host apply the RK4 stage update in the
+        RHS kernel's epilogue (1) or in a separate streaming kernel (0); bit-identical."""
+        _check(lib().dgr_set_option(self._h, OPT_FUSE_RK4, int(bool(on))))
 
     def set_phases(self, mode=0):
         """DGR_OPT_PHASES: 0 = overlap interior octants with the ghost exchange when

@@ -152,6 +152,11 @@ struct dgr_mesh_s {
   // DGR_OPT_GRAPH: dgr_rk4_step replays a CUDA graph of its 4 stages (captured
   // on a library stream at the second call with the same arguments)
   bool use_graph = true;
+  // DGR_OPT_FUSE_RK4: dgr_rk4_step / dgr_rk4_step_host apply the RK4 stage
+  // update in k_rhs's zip-by-store epilogue (no k_rk4), the stage states
+  // alternating between d_us and d_us2 (a stage never writes what it gathers)
+  bool fuse_rk4 = true;
+  double* d_us2 = nullptr;
   cudaStream_t gstream = nullptr;
   cudaGraphExec_t gexec = nullptr;
   int64_t glaunches = 0;
@@ -941,11 +946,22 @@ static dgr_status ensure_xstream(dgr_mesh m) {
 // group driver (dgr_group_*) and completes at m->ev_xdone; otherwise it is done
 // here (NCCL) — on the caller's stream, or on m->xstream overlapped with the
 // interior octants.
+// rk (fused path with rhs_dof only): the RK4 stage update fields of RhsParams,
+// applied by k_rhs's epilogue instead of storing the RHS
 static dgr_status rhs_oct(dgr_mesh m, double* u, const dgr_params* prm, cudaStream_t st,
-                          double* rhs_dof = nullptr, bool preissued = false) {
+                          double* rhs_dof = nullptr, bool preissued = false,
+                          const RhsParams* rk = nullptr) {
   dgr_status s;
   const int64_t no = m->dm.n_owned, ni = m->n_interior;
-  const RhsParams rp = to_rp(prm);
+  RhsParams rp = to_rp(prm);
+  if (rk && rhs_dof) {
+    rp.rk_stage = rk->rk_stage;
+    rp.rk_dt = rk->rk_dt;
+    rp.rk_un = rk->rk_un;
+    rp.rk_acc = rk->rk_acc;
+    rp.rk_us = rk->rk_us;
+    rp.rk_out = rk->rk_out;
+  }
   double* pre = nullptr;
   if (m->fused && m->prepass && !(rp.sommerfeld && !m->host.periodic)) {
     if (!m->d_pre) CUDA_TRY(m->alloc(&m->d_pre, size_t(30) * no * 352));
@@ -1058,11 +1074,26 @@ dgr_status dgr_rhs(dgr_mesh m, double* u, double* rhs, const dgr_params* prm, vo
   return DGR_OK;
 }
 
+// u_s: the previous stage's state (gathered by stages 1-3); u_s_next (fused
+// RK4 update only, != u_s): where this stage writes its state
 static dgr_status stage(dgr_mesh m, int s_, double dt, double* u_n, double* u_s, double* acc,
                         double* u_out, const dgr_params* prm, cudaStream_t st,
-                        bool preissued = false) {
+                        bool preissued = false, double* u_s_next = nullptr) {
   dgr_status s;
   double* cur = s_ == 0 ? u_n : u_s;
+  if (u_s_next && zip_by_store(m, prm)) {
+    if (!m->d_rhs_dof) CUDA_TRY(m->alloc(&m->d_rhs_dof, size_t(NF) * m->dm.dof_stride));
+    RhsParams rk = to_rp(prm);
+    rk.rk_stage = s_;
+    rk.rk_dt = dt;
+    rk.rk_un = u_n;
+    rk.rk_acc = acc;
+    rk.rk_us = u_s_next;
+    rk.rk_out = u_out;
+    if ((s = rhs_oct(m, cur, prm, st, m->d_rhs_dof, preissued, &rk))) return s;
+    CUDA_TRY(cudaGetLastError());
+    return DGR_OK;
+  }
   // (applying the zip + RK4 update inside k_rhs measured 10.6 ms vs 7.5 + 0.8 ms
   // for RHS + k_zip_rk4 on C3 — the scattered state loads stall the single
   // persistent CTA per SM — so the update is a separate kernel; the zip itself
@@ -1077,6 +1108,24 @@ static dgr_status stage(dgr_mesh m, int s_, double dt, double* u_n, double* u_s,
   if ((s = rhs_oct(m, cur, prm, st, nullptr, preissued))) return s;
   PROF(m, 4, st, launch_zip_rk4(m->dm, m->d_rhs_oct, s_, dt, u_n, u_s, acc, u_out, st));
   CUDA_TRY(cudaGetLastError());
+  return DGR_OK;
+}
+
+// the four stages of one RK4 step of u (in place), with the fused update
+// (DGR_OPT_FUSE_RK4) when the path allows it: stage k gathers u, d_us, d_us2,
+// d_us and writes d_us, d_us2, d_us, u
+static dgr_status four_stages(dgr_mesh m, double dt, double* u, const dgr_params* prm,
+                              cudaStream_t q) {
+  const bool fz = m->fuse_rk4 && zip_by_store(m, prm);
+  if (fz && !m->d_us2) {
+    CUDA_TRY(m->alloc(&m->d_us2, size_t(NF) * m->dm.dof_stride));
+    CUDA_TRY(cudaMemset(m->d_us2, 0, size_t(NF) * m->dm.dof_stride * 8));
+  }
+  for (int k = 0; k < 4; ++k) {
+    double* in = k == 2 && fz ? m->d_us2 : m->d_us;
+    double* out = fz ? (k == 1 ? m->d_us2 : m->d_us) : nullptr;
+    if (dgr_status e = stage(m, k, dt, u, in, m->d_acc, u, prm, q, false, out)) return e;
+  }
   return DGR_OK;
 }
 
@@ -1104,9 +1153,7 @@ dgr_status dgr_rk4_step(dgr_mesh m, double dt, double* u, const dgr_params* prm,
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   auto eager = [&](cudaStream_t q) -> dgr_status {
     m->launches = 0;
-    for (int k = 0; k < 4; ++k)
-      if (dgr_status e = stage(m, k, dt, u, m->d_us, m->d_acc, u, prm, q)) return e;
-    return DGR_OK;
+    return four_stages(m, dt, u, prm, q);
   };
   // CUDA graph of the step (the 16+ launches of the 4 stages, and with N > 1
   // the exchange stream's pack / NCCL / unpack, captured once): the first call
@@ -1189,8 +1236,7 @@ dgr_status dgr_rk4_step_host(dgr_mesh m, double dt, int64_t n, const double* con
                                m->h2d));
     CUDA_TRY(cudaEventRecord(m->ev_in[b], m->h2d));
     CUDA_TRY(cudaStreamWaitEvent(st, m->ev_in[b], 0));
-    for (int k = 0; k < 4; ++k)   // (launch counts accumulate over the n steps)
-      if ((s = stage(m, k, dt, ub, m->d_us, m->d_acc, ub, prm, st))) return s;
+    if ((s = four_stages(m, dt, ub, prm, st))) return s;   // (launch counts accumulate)
     CUDA_TRY(cudaEventRecord(m->ev_done[b], st));
     CUDA_TRY(cudaStreamWaitEvent(m->d2h, m->ev_done[b], 0));
     CUDA_TRY(cudaMemcpy2DAsync(u_out[j], pitch, ub, pitch, width, NF, cudaMemcpyDeviceToHost,
@@ -1555,6 +1601,7 @@ dgr_status dgr_set_option(dgr_mesh m, int option, int64_t value) {
   if (!m) return fail(DGR_ERR_ARG, "null mesh");
   switch (option) {
     case DGR_OPT_GRAPH: m->use_graph = value != 0; m->drop_graph(); return DGR_OK;
+    case DGR_OPT_FUSE_RK4: m->fuse_rk4 = value != 0; m->drop_graph(); return DGR_OK;
     case DGR_OPT_FUSED_UNZIP: m->fused = value != 0; m->drop_graph(); return DGR_OK;
     case DGR_OPT_PREPASS: m->prepass = value != 0; m->drop_graph(); return DGR_OK;
     case DGR_OPT_ZIP_STORE: m->zip_store = value != 0; m->drop_graph(); return DGR_OK;

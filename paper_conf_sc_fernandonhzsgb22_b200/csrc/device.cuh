@@ -105,11 +105,42 @@ void launch_scatter_unpack(double* u, int64_t stride, int64_t n_owned, const dou
 
 void launch_dfma(int blocks, int iters, double* out, cudaStream_t s);
 
+// The RK4 stage update of element i from its RHS k (reading R11, classic
+// tableau), with explicit fma so k_rk4, k_zip_rk4 and the fused k_rhs epilogue
+// round alike:  s=0: acc = u_n + dt/6 k, u_s = u_n + dt/2 k;  s=1: acc += dt/3 k,
+// u_s = u_n + dt/2 k;  s=2: acc += dt/3 k, u_s = u_n + dt k;  s=3: u_out = acc + dt/6 k
+template <int S>
+__device__ __forceinline__ void rk4_update(int64_t i, double k, double dt, const double* u_n,
+                                           double* u_s, double* acc, double* u_out) {
+  if (S == 0) {
+    const double un = u_n[i];
+    acc[i] = __fma_rn(dt / 6.0, k, un);
+    u_s[i] = __fma_rn(dt / 2.0, k, un);
+  } else if (S == 1) {
+    acc[i] = __fma_rn(dt / 3.0, k, acc[i]);
+    u_s[i] = __fma_rn(dt / 2.0, k, u_n[i]);
+  } else if (S == 2) {
+    acc[i] = __fma_rn(dt / 3.0, k, acc[i]);
+    u_s[i] = __fma_rn(dt, k, u_n[i]);
+  } else {
+    u_out[i] = __fma_rn(dt / 6.0, k, acc[i]);
+  }
+}
+
 // rhs_kernel.cu
 struct RhsParams {
   double ko_sigma, eta, lambda_f0, lambda_f1, chi_floor;
   int sommerfeld;   // radiative outer boundary (reading R29)
   int upwind;       // lopsided advective derivatives (reading R9u)
+  // RK4 stage update fused into the zip-by-store epilogue (rk_stage >= 0,
+  // reading R11, the arithmetic of k_rk4): each zip owner updates its DOF's
+  // acc / u_s (stage 0..2) or u_out (stage 3) instead of storing the RHS
+  int rk_stage = -1;
+  double rk_dt = 0.0;
+  const double* rk_un = nullptr;
+  double* rk_acc = nullptr;
+  double* rk_us = nullptr;
+  double* rk_out = nullptr;
 };
 // fused = false: read 13^3 patches ([24][n_owned][PATCH_PITCH], TMA bulk copies);
 // fused = true: `src` is the state u; every patch is gathered from u and the

@@ -53,19 +53,7 @@ __global__ void k_zip_rk4(const int32_t* __restrict__ zip, int32_t n, int64_t no
   for (int d = blockIdx.x * blockDim.x + threadIdx.x; d < n; d += gridDim.x * blockDim.x) {
     const int64_t i = f * stride + d;
     const double k = __ldg(rhs_oct + f * no343 + __ldg(zip + d));
-    if (S == 0) {
-      const double un = u_n[i];
-      acc[i] = un + (dt / 6.0) * k;
-      u_s[i] = un + (dt / 2.0) * k;
-    } else if (S == 1) {
-      acc[i] += (dt / 3.0) * k;
-      u_s[i] = u_n[i] + (dt / 2.0) * k;
-    } else if (S == 2) {
-      acc[i] += (dt / 3.0) * k;
-      u_s[i] = u_n[i] + dt * k;
-    } else {
-      u_out[i] = acc[i] + (dt / 6.0) * k;
-    }
+    rk4_update<S>(i, k, dt, u_n, u_s, acc, u_out);
   }
 }
 
@@ -79,19 +67,7 @@ __global__ void k_rk4(int32_t n, int64_t stride, double dt, const double* __rest
   for (int d = blockIdx.x * blockDim.x + threadIdx.x; d < n; d += gridDim.x * blockDim.x) {
     const int64_t i = f * stride + d;
     const double k = __ldcs(rhs + i);
-    if (S == 0) {
-      const double un = u_n[i];
-      acc[i] = un + (dt / 6.0) * k;
-      u_s[i] = un + (dt / 2.0) * k;
-    } else if (S == 1) {
-      acc[i] += (dt / 3.0) * k;
-      u_s[i] = u_n[i] + (dt / 2.0) * k;
-    } else if (S == 2) {
-      acc[i] += (dt / 3.0) * k;
-      u_s[i] = u_n[i] + dt * k;
-    } else {
-      u_out[i] = acc[i] + (dt / 6.0) * k;
-    }
+    rk4_update<S>(i, k, dt, u_n, u_s, acc, u_out);
   }
 }
 

@@ -231,6 +231,11 @@ __device__ __forceinline__ void cp_async_wait1() {
 __constant__ double c_rWEXT[3 * 7];
 constexpr int GJ = (NPATCH + RT - 1) / RT;   // gather points per thread (7)
 constexpr int C_CENTRE = 6 + 13 * 6 + 169 * 6;   // patch centre (threads without a point)
+#ifndef DGR_RKB
+#define DGR_RKB 8   // (A/B, profiles/r3_experiments: 4 / 6 / 8 / 12 -> 27.60 / 27.32 / 27.25 / 27.33 ms per C3 step)
+#endif
+constexpr int RKB = DGR_RKB;   // fields per batch of the fused RK4 update's loads
+static_assert(NF % RKB == 0, "RKB divides 24");
 
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   uint32_t ok = 0;
@@ -756,6 +761,21 @@ __global__ void __launch_bounds__(RT, 1)
   }
   for (int st = 0; st < NST; ++st, ++g) {
     const int buf = g & 1;
+    if (FUSED && !SOMM && rhs_dof && prm.rk_stage >= 0 && st == NST - 3) {
+      // fused RK4 update: this point's u_n / acc rows into L2 for the epilogue
+      double ex[6];
+      VALS_LD(TV_EX, ex);
+      const int dz = __double2loint(ex[3]);
+      if (dz >= 0) {
+        const int64_t ds64 = m.dof_stride;
+        for (int f = 0; f < NF; ++f) {
+          if (prm.rk_stage <= 2)
+            asm volatile("prefetch.global.L2 [%0];" ::"l"(prm.rk_un + f * ds64 + dz));
+          if (prm.rk_stage >= 1)
+            asm volatile("prefetch.global.L2 [%0];" ::"l"(prm.rk_acc + f * ds64 + dz));
+        }
+      }
+    }
 #ifdef DGR_RHS_TIMING
     if (tid == 0) {   // per-stage cycle profile (experiment builds only)
       const long long t = clock64();
@@ -1141,7 +1161,42 @@ __global__ void __launch_bounds__(RT, 1)
       }
     double* out = rhs_oct + int64_t(e) * NPT + p;
     const int64_t ostr = no * NPT;
-    if (!SOMM && rhs_dof) {
+    if (!SOMM && rhs_dof && prm.rk_stage >= 0) {
+      // the RK4 stage update of the owned DOF dz (its u_n / acc rows were
+      // prefetched into L2 two stages ago), in batches of RKB fields
+      if (dz >= 0) {
+        const int S = prm.rk_stage;
+        const double dt = prm.rk_dt;
+        const int64_t ds64 = m.dof_stride;
+#pragma unroll
+        for (int f0 = 0; f0 < NF; f0 += RKB) {
+          double un[RKB], ac[RKB];
+#pragma unroll
+          for (int j = 0; j < RKB; ++j) {
+            const int64_t i = (f0 + j) * ds64 + dz;
+            un[j] = S <= 2 ? __ldcs(prm.rk_un + i) : 0.0;
+            ac[j] = S >= 1 ? __ldcs(prm.rk_acc + i) : 0.0;
+          }
+#pragma unroll
+          for (int j = 0; j < RKB; ++j) {
+            const int64_t i = (f0 + j) * ds64 + dz;
+            const double k = r[f0 + j];
+            if (S == 0) {
+              prm.rk_acc[i] = __fma_rn(dt / 6.0, k, un[j]);
+              prm.rk_us[i] = __fma_rn(dt / 2.0, k, un[j]);
+            } else if (S == 1) {
+              prm.rk_acc[i] = __fma_rn(dt / 3.0, k, ac[j]);
+              prm.rk_us[i] = __fma_rn(dt / 2.0, k, un[j]);
+            } else if (S == 2) {
+              prm.rk_acc[i] = __fma_rn(dt / 3.0, k, ac[j]);
+              prm.rk_us[i] = __fma_rn(dt, k, un[j]);
+            } else {
+              prm.rk_out[i] = __fma_rn(dt / 6.0, k, ac[j]);
+            }
+          }
+        }
+      }
+    } else if (!SOMM && rhs_dof) {
       if (dz >= 0) {
 #pragma unroll
         for (int f = 0; f < NF; ++f) st_out(&rhs_dof[f * int64_t(m.dof_stride) + dz], r[f]);

@@ -41,13 +41,15 @@ INTERP_BYTES_PER_ELEM = 24 * 343 * 8 + 343 * 4    # read the element's nodal val
 RHS_BYTES_PER_OCT = 24 * (2197 + 343) * 8         # patch read + rhs write (eq 21a denominator)
 PAPER_FLOPS_PER_POINT = 5502 + 3998               # eq (21a) numerator per point, O_A from Q_L = 6.68
 # executed fp64 FLOPs per interior point (2 DFMA + DADD + DMUL thread instructions from
-# ncu sm__sass_thread_inst_executed_op_d{fma,add,mul}_pred_on, C3, 8,329,412 points):
-# fused = k_gt_pre 976.5 + k_rhs 3,434.9 per point (profiles/r2l_flops.csv, round 2:
-# light-field pair stages, zip owner = coarsest leaf), two-pass = the single k_rhs
-# 36.283e9 (profiles/r1o_flops_twopass.csv).  (Round-1 history: 5,358 /
-# 5,265 before the Ricci / At^ij contraction-order and trace-free-once changes removed
-# ~950 FLOP/point.)
-RHS_EXEC_FLOPS_PER_POINT = {"fused": 4411.4, "two-pass": 4356.0}
+# ncu sm__sass_thread_inst_executed_op_d{fma,add,mul}_pred_on, C3, 8,329,412 points;
+# profiles/r3y_flops*.csv, round 2 final code): fused = k_gt_pre 976.5 + k_rhs
+# 3,603.4 x 343/352 (k_rhs runs its 9 threads without a point through the same
+# warp-wide code since the tensor-memory value store; their share is discounted;
+# k_rhs now also applies the RK4 stage update, ~58 FLOP per point), two-pass =
+# the single k_rhs 4,451.2 x 343/352.  (History: 4,411.4 / 4,356.0 before the
+# round-2 session's TMEM / fused-update changes; round 1 5,358 / 5,265 before the
+# Ricci / At^ij contraction-order and trace-free-once changes.)
+RHS_EXEC_FLOPS_PER_POINT = {"fused": 976.5 + 3603.4 * 343 / 352, "two-pass": 4451.2 * 343 / 352}
 # DRAM bytes per launch (dram__bytes_read.sum + dram__bytes_write.sum) from one
 # ncu --set full capture of the C3 workload on 1 GPU, per path
 # (profiles/ncu_traffic_c3.json, written by tools/ncu_traffic.py)

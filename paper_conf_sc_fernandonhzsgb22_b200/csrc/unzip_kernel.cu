@@ -97,20 +97,24 @@ __global__ void __launch_bounds__(IP_THREADS)
   __syncthreads();
   for (int gi = 0; gi < el.z; ++gi) {
   const int4 gr = m.igrp[el.y + gi];
-  int lo[3], n[3];
-#pragma unroll
-  for (int k = 0; k < 3; ++k) {
-    lo[k] = (gr.z >> (4 * k)) & 15;
-    n[k] = ((gr.z >> (12 + 4 * k)) & 15) - lo[k] + 1;
-  }
   const int a1 = (gr.z >> 24) & 3;   // the group's face normal (host-chosen, partition-invariant)
   const int a2 = a1 == 0 ? 1 : 0, a3 = a1 == 2 ? 1 : 2;
-  const int n1 = n[a1], n2 = n[a2];
+  // bounding box along a1 and a2 (4-bit fields: lo at 4a, hi at 12 + 4a)
+  const int lo1 = (gr.z >> (4 * a1)) & 15, lo2 = (gr.z >> (4 * a2)) & 15;
+  const int n1 = ((gr.z >> (12 + 4 * a1)) & 15) - lo1 + 1, n2 = ((gr.z >> (12 + 4 * a2)) & 15) - lo2 + 1;
   const int es1 = a1 == 0 ? 1 : (a1 == 1 ? 7 : 49);
   const int es2 = a2 == 0 ? 1 : (a2 == 1 ? 7 : 49);
   const int es3 = a3 == 0 ? 1 : (a3 == 1 ? 7 : 49);
-  const int lo1 = lo[a1], lo2 = lo[a2];
   const float rn1 = 1.0f / float(n1), rn2 = 1.0f / float(n2);
+  // this thread's slots of the group (k = tid + IP_THREADS i): their half-grid
+  // points are loaded now, so the last sweep does not wait on global loads
+  constexpr int IP_KMAX = (13 * 13 * IP_N1 + IP_THREADS - 1) / IP_THREADS;   // slots <= box volume
+  uint32_t tk[IP_KMAX];
+#pragma unroll
+  for (int i = 0; i < IP_KMAX; ++i) {
+    const int k = tid + IP_THREADS * i;
+    tk[i] = k < gr.y ? __ldg(m.ipt + gr.x + k) : 0u;
+  }
   // T1[g][r3][r2][i1] = sum_m W[lo1+i1][m] E_g[m, r2, r3]
   for (int idx = tid; idx < 49 * n1; idx += IP_THREADS) {
     const int r = fdiv(idx, rn1), i1 = idx - r * n1;   // r = r3 * 7 + r2
@@ -163,10 +167,14 @@ __global__ void __launch_bounds__(IP_THREADS)
   __syncthreads();
   // slot value = sum_m W[t2_a3][m] T2[g][m][i2][i1]
   double* out = m.aux + gr.x;
-  for (int k = tid; k < gr.y; k += IP_THREADS) {
-    const int t = __ldg(m.ipt + gr.x + k);
-    const int t2[3] = {t & 15, (t >> 4) & 15, (t >> 8) & 15};
-    const int i1 = t2[a1] - lo1, i2 = t2[a2] - lo2, tt = t2[a3];
+#pragma unroll
+  for (int ii = 0; ii < IP_KMAX; ++ii) {
+    const int k = tid + IP_THREADS * ii;
+    if (k < gr.y) {
+    // (axis fields by shifts: a runtime-indexed local array would live in local memory)
+    const int t = int(tk[ii]);
+    const int i1 = ((t >> (4 * a1)) & 15) - lo1, i2 = ((t >> (4 * a2)) & 15) - lo2,
+              tt = (t >> (4 * a3)) & 15;
     const int col = i2 * n1 + i1, st = n2 * n1;
     double v[IP_FG];
     if (tt & 1) {
@@ -186,6 +194,7 @@ __global__ void __launch_bounds__(IP_THREADS)
 #pragma unroll
     for (int g = 0; g < IP_FG; ++g)
       if (f0 + g < nf) out[(f0 + g) * as + k] = v[g];
+    }
   }
   __syncthreads();   // T1/T2 reused by the next group
   }  // face groups

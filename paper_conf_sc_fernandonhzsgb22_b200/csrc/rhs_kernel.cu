@@ -566,10 +566,14 @@ __global__ void __launch_bounds__(RT, 1)
             ((oi.y + sd == nside) << 4) | ((oi.z + sd == nside) << 5);
   }
   const bool bnd = omask != 0;
-  if (FUSED && en >= 0 && tid == 32)   // next octant's gather map into L2
-    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(m.gmap + int64_t(en) * GM_PITCH),
+  if (FUSED && en >= 0 && tid == 32) {   // next octant's gather rows (gmap_s, gdst) into L2
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(m.gmap_s + int64_t(en) * GM_PITCH),
                  "r"(uint32_t(GM_PITCH * 4))
                  : "memory");
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(m.gdst + int64_t(en) * GM_PITCH),
+                 "r"(uint32_t(GM_PITCH * 2))
+                 : "memory");
+  }
   const double ih = (6.0 * double(int64_t(1) << oi.w)) / m.width;   // 1/h
   const double ko_scale = prm.ko_sigma * ih * (1.0 / 64.0);
   // Sommerfeld (reading R29): this point is a node on a face of the domain
@@ -1302,6 +1306,14 @@ __global__ void __launch_bounds__(RT, 2)
       const int nside = 1 << m.D, sd = 1 << (m.D - oi.w);
       omask = (oi.x == 0) | ((oi.y == 0) << 1) | ((oi.z == 0) << 2) | ((oi.x + sd == nside) << 3) |
               ((oi.y + sd == nside) << 4) | ((oi.z + sd == nside) << 5);
+    }
+    if (en >= 0 && tid == 32) {   // next octant's gather rows (gmap_s, gdst) into L2
+      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(m.gmap_s + int64_t(en) * GM_PITCH),
+                   "r"(uint32_t(GM_PITCH * 4))
+                   : "memory");
+      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(m.gdst + int64_t(en) * GM_PITCH),
+                   "r"(uint32_t(GM_PITCH * 2))
+                   : "memory");
     }
     const double ih = (6.0 * double(int64_t(1) << oi.w)) / m.width;   // 1/h
     const double ko_scale = prm.ko_sigma * ih * (1.0 / 64.0);

@@ -1234,7 +1234,13 @@ __global__ void __launch_bounds__(RT, 1)
 // Same stencils, same gather/extrapolation and same arithmetic order as the
 // gt stages of k_rhs, so both paths give bit-identical results.
 constexpr int NPRE = 30;
-constexpr int PRE_NBUF = 3;   // stage ring depth of the pre-pass
+#ifndef DGR_PRE_NBUF
+#define DGR_PRE_NBUF 2   // (A/B r3ag: 27.01 -> 26.91 ms per C3 step with 2)
+#endif
+// stage ring depth of the pre-pass: 3 = one barrier per field (the gather of
+// field g+2 goes into the buffer of g-1 after the start barrier); 2 = a second
+// barrier per field, 17.6 KB less shared memory per CTA (more L1)
+constexpr int PRE_NBUF = DGR_PRE_NBUF;
 constexpr size_t PRE_SMEM_BYTES = size_t(PRE_NBUF) * STAGE_DBL * 8 + size_t(TX_N + TY_N) * 8 +
                                   size_t(3) * RT * 2;
 
@@ -1348,8 +1354,8 @@ __global__ void __launch_bounds__(RT, 2)
       const int buf = g % PRE_NBUF;
       cp_async_wait1();   // this thread's copies of stage g (g+1 may be in flight)
       __syncthreads();    // everyone's; and everyone is done with stage g-1
-      {
-        // stage g+2 into the buffer of stage g-1
+      auto issue_next = [&]() {
+        // stage g+2 into the buffer of stage g-1 (ring of 3) / of stage g (ring of 2)
         double* dst = stage + ((g + 2) % PRE_NBUF) * STAGE_DBL;
         if (q + 2 < 6) {
           gather(dst, 12 + q + 2);
@@ -1358,7 +1364,8 @@ __global__ void __launch_bounds__(RT, 2)
           if (en >= 0) gather(dst, 12 + q + 2 - 6);
           else cp_async_commit();
         }
-      }
+      };
+      if (PRE_NBUF == 3) issue_next();
       double* sw = stage + buf * STAGE_DBL;
       if (omask) {
         for (int a = 0; a < 3; ++a) {
@@ -1402,6 +1409,10 @@ __global__ void __launch_bounds__(RT, 2)
         for (int k = 0; k < 3; ++k) st_out(&out[(6 * k + q) * ostr], d.d1[k]);
         st_out(&out[(18 + q) * ostr], trace6(gi, d.dd));
         st_out(&out[(24 + q) * ostr], __dadd_rn(advect<UPW>(s, c0, beta, d.d1, ih), d.ko));
+      }
+      if (PRE_NBUF == 2) {
+        __syncthreads();   // everyone is done with this stage buffer
+        issue_next();
       }
     }
   }

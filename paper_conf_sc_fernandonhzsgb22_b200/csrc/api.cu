@@ -964,7 +964,7 @@ static dgr_status rhs_oct(dgr_mesh m, double* u, const dgr_params* prm, cudaStre
   }
   double* pre = nullptr;
   if (m->fused && m->prepass && !(rp.sommerfeld && !m->host.periodic)) {
-    if (!m->d_pre) CUDA_TRY(m->alloc(&m->d_pre, size_t(30) * no * 352));
+    if (!m->d_pre) CUDA_TRY(m->alloc(&m->d_pre, size_t(pre_rows()) * no * 352));
     pre = m->d_pre;
   }
   // ghosts current on `st` (no overlap)

@@ -156,6 +156,7 @@ void launch_rhs(const DevMesh& m, const double* src, double* rhs_oct, const RhsP
                 bool fused, int64_t first, int64_t count, int leave_sm, cudaStream_t s,
                 double* pre = nullptr, double* rhs_dof = nullptr);
 size_t rhs_smem_bytes();
+int pre_rows();   // metric pre-pass values per interior point
 void upload_rhs_tables(const double* wext);
 
 // gen/rhs_alg.cu (generated by codegen/gen.py): the algebraic part A of the RHS

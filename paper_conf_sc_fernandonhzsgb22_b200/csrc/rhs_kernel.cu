@@ -1233,7 +1233,8 @@ __global__ void __launch_bounds__(RT, 1)
 // which k_rhs<..., PRE = true> reads instead of staging the gt fields itself.
 // Same stencils, same gather/extrapolation and same arithmetic order as the
 // gt stages of k_rhs, so both paths give bit-identical results.
-constexpr int NPRE = 30;
+constexpr int NPRE = 30;   // rows per point (api.cu allocates pre_rows() of them)
+int pre_rows() { return NPRE; }
 #ifndef DGR_PRE_NBUF
 #define DGR_PRE_NBUF 2   // (A/B r3ag: 27.01 -> 26.91 ms per C3 step with 2)
 #endif

@@ -54,7 +54,7 @@ constexpr int TY_OFF = 42, TY_N = 2113;   // x, y in 3..9, z in 0..12
 constexpr int T_N = 2 * STAGE_DBL;        // Tx + Ty, or two light-field stage halves
 static_assert(TX_N + TY_N <= T_N, "Tx/Ty fit the two pair halves");
 constexpr size_t SMEM_BYTES = size_t(NSLOT) * NPP * 8 + size_t(2) * STAGE_DBL * 8 +
-                              size_t(T_N) * 8 + 16 + size_t(3) * RT * 2 + 16;
+                              size_t(T_N) * 8 + 16 + 16 + size_t(RT) * 4 + size_t(3) * RT * 2 + 16;
 
 // Tensor memory as per-thread storage (tcgen05.ld / tcgen05.st, 32x32b shape:
 // each thread moves 32-bit columns of its own TMEM lane).  Warp w reaches lanes
@@ -437,9 +437,13 @@ __global__ void __launch_bounds__(RT, 1)
   double* Tx = stage + 2 * STAGE_DBL;             // [TX_N] (T region: [T_N])
   double* Ty = Tx + TX_N;                         // [TY_N]
   uint64_t* bars = reinterpret_cast<uint64_t*>(Tx + T_N);
+  // FUSED: the octant-to-come's anchor (16 B) and each thread's o2s index of
+  // its point in it, copied asynchronously two stages before its prologue
+  int4* sm_oi = reinterpret_cast<int4*>(bars + 2);
+  int32_t* tab_cv = reinterpret_cast<int32_t*>(sm_oi + 1);
   // this thread's point: patch index c0 (-1: no point) and interior index p, kept
   // in shared memory and re-read where needed (cheaper than a register spill)
-  int16_t* tab_c0 = reinterpret_cast<int16_t*>(bars + 2);
+  int16_t* tab_c0 = reinterpret_cast<int16_t*>(tab_cv + RT);
   int16_t* tab_p = tab_c0 + RT;
   int16_t* tab_d1b = tab_p + RT;                                  // D1-pass line (g_d1b)
   uint32_t* tm_base = reinterpret_cast<uint32_t*>(tab_d1b + RT);  // TMEM allocation address
@@ -483,9 +487,20 @@ __global__ void __launch_bounds__(RT, 1)
   };
   // FUSED: stage k's field(s) into stage buffer b (and T-region half b), one
   // cp.async group per stage
-  auto gather_stage = [&](int b, int k) {
+  // (oct_next >= 0: also the next octant's anchor and o2s index, which land
+  // with this group, before that octant's prologue)
+  auto gather_stage = [&](int b, int k, int oct_next = -1) {
     gather(stage + b * STAGE_DBL, stA(k));
     if (stB(k) >= 0) gather(Tx + b * STAGE_DBL, stB(k));
+    if (oct_next >= 0) {
+      asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(tab_cv + tid)),
+                   "l"(m.o2s + int64_t(oct_next) * NPT + max(int(tab_p[tid]), 0))
+                   : "memory");
+      if (tid == 0)
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(smem_u32(sm_oi)),
+                     "l"(m.oct + oct_next)
+                     : "memory");
+    }
     cp_async_commit();
   };
   // FUSED: the value of field f at element node (e, p), through o2s
@@ -520,6 +535,10 @@ __global__ void __launch_bounds__(RT, 1)
                  : "memory");
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
   }
+  if (FUSED) {   // the first octant's anchor and o2s index (later ones arrive by cp.async)
+    tab_cv[tid] = __ldg(m.o2s + int64_t(e) * NPT + max(int(tab_p[tid]), 0));
+    if (tid == 0) *sm_oi = m.oct[e];
+  }
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
@@ -549,14 +568,14 @@ __global__ void __launch_bounds__(RT, 1)
   const bool active = tab_c0[tid] >= 0;
   // the point's own values: patch index c0 of the staged patches, or (FUSED)
   // element node p of u / a hanging-node slot through o2s
-  const int cv = FUSED ? __ldg(m.o2s + int64_t(e) * NPT + max(int(tab_p[tid]), 0))
+  const int cv = FUSED ? tab_cv[tid]
                        : (active ? int(tab_c0[tid]) : C_CENTRE);
   auto own = [&](int f) -> double {
     if (!FUSED) return __ldg(pbase + f * fstride + cv);
     return cv < ds ? __ldg(patches + f * fstride + cv) : __ldg(m.aux + f * m.aux_stride + (cv - ds));
   };
 
-  const int4 oi = m.oct[e];
+  const int4 oi = FUSED ? *sm_oi : m.oct[e];
   // FUSED: which faces of this octant lie on a non-periodic domain boundary
   // (bit a: low face along axis a outside the domain, bit 3 + a: high face)
   int omask = 0;
@@ -1081,7 +1100,7 @@ __global__ void __launch_bounds__(RT, 1)
     __syncthreads();  // everyone is done with this stage buffer
     if (FUSED) {
       if (st + 2 < NST) {
-        gather_stage(buf, st + 2);
+        gather_stage(buf, st + 2, st + 3 == NST ? en : -1);
       } else {
         if (st + 2 == NST && en >= 0) load_gidx(en);   // the current octant's gathers are issued
         if (en >= 0) gather_stage(buf, st + 2 - NST);

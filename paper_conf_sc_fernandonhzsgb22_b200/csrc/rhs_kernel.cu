@@ -1262,7 +1262,7 @@ int pre_rows() { return NPRE; }
 // barrier per field, 17.6 KB less shared memory per CTA (more L1)
 constexpr int PRE_NBUF = DGR_PRE_NBUF;
 constexpr size_t PRE_SMEM_BYTES = size_t(PRE_NBUF) * STAGE_DBL * 8 + size_t(TX_N + TY_N) * 8 +
-                                  size_t(3) * RT * 2;
+                                  16 + size_t(RT) * 4 + size_t(3) * RT * 2;
 
 // Fused path only (patches gathered from u and the slots).  Three-deep stage
 // ring: the CTA barrier that releases stage g's data also proves every thread
@@ -1276,7 +1276,10 @@ __global__ void __launch_bounds__(RT, 2)
   double* stage = smem;                           // [PRE_NBUF][STAGE_DBL]
   double* Tx = stage + PRE_NBUF * STAGE_DBL;      // [TX_N]
   double* Ty = Tx + TX_N;                         // [TY_N]
-  int16_t* tab_c0 = reinterpret_cast<int16_t*>(Ty + TY_N);
+  // the octant-to-come's anchor and each thread's o2s index (cp.async, as k_rhs)
+  int4* sm_oi = reinterpret_cast<int4*>(Ty + TY_N);
+  int32_t* tab_cv = reinterpret_cast<int32_t*>(sm_oi + 1);
+  int16_t* tab_c0 = reinterpret_cast<int16_t*>(tab_cv + RT);
   int16_t* tab_p = tab_c0 + RT;
   int16_t* tab_d1b = tab_p + RT;
   const int tid = threadIdx.x;
@@ -1306,7 +1309,7 @@ __global__ void __launch_bounds__(RT, 2)
       gdst[j] = pt < NPATCH ? int(__ldg(gd + pt)) : 0;
     }
   };
-  auto gather = [&](double* dst, int f) {
+  auto gather = [&](double* dst, int f, int oct_next = -1) {
     // (gt fields: the three slabs the stencils and the D1 pass read)
     const uint32_t d0 = smem_u32(dst);
     const double* uf = patches + f * fstride;
@@ -1314,8 +1317,19 @@ __global__ void __launch_bounds__(RT, 2)
 #pragma unroll
     for (int j = 0; j < GJ; ++j)
       if (tid + RT * j < G_SLABS) cp_async8(d0 + 8 * gdst[j], uf, af, gidx[j], ds);
+    if (oct_next >= 0) {   // (lands before that octant's prologue)
+      asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(tab_cv + tid)),
+                   "l"(m.o2s + int64_t(oct_next) * NPT + int(tab_p[tid]))
+                   : "memory");
+      if (tid == 0)
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(smem_u32(sm_oi)),
+                     "l"(m.oct + oct_next)
+                     : "memory");
+    }
     cp_async_commit();
   };
+  tab_cv[tid] = __ldg(m.o2s + int64_t(e) * NPT + int(tab_p[tid]));
+  if (tid == 0) *sm_oi = m.oct[e];
   __syncthreads();
   load_gidx(e);
   gather(stage, 12);
@@ -1326,7 +1340,7 @@ __global__ void __launch_bounds__(RT, 2)
     const int en = li + int(gridDim.x) < count ? ol[li + gridDim.x] : -1;
     const int c0 = tab_c0[tid];
     const int p = tab_p[tid];
-    const int4 oi = m.oct[e];
+    const int4 oi = *sm_oi;
     int omask = 0;
     if (!m.periodic) {
       const int nside = 1 << m.D, sd = 1 << (m.D - oi.w);
@@ -1346,7 +1360,7 @@ __global__ void __launch_bounds__(RT, 2)
     // values at the point: gt (for gt^ij) and beta (advection)
     double gi[6] = {0, 0, 0, 0, 0, 0}, beta[3] = {0, 0, 0};
     if (c0 >= 0) {
-      const int cv = __ldg(m.o2s + int64_t(e) * NPT + p);
+      const int cv = tab_cv[tid];
       auto own = [&](int f) -> double {
         return cv < ds ? __ldg(patches + f * fstride + cv) : __ldg(m.aux + f * m.aux_stride + (cv - ds));
       };
@@ -1378,7 +1392,7 @@ __global__ void __launch_bounds__(RT, 2)
         // stage g+2 into the buffer of stage g-1 (ring of 3) / of stage g (ring of 2)
         double* dst = stage + ((g + 2) % PRE_NBUF) * STAGE_DBL;
         if (q + 2 < 6) {
-          gather(dst, 12 + q + 2);
+          gather(dst, 12 + q + 2, q == 3 ? en : -1);
         } else {
           if (q == 4 && en >= 0) load_gidx(en);
           if (en >= 0) gather(dst, 12 + q + 2 - 6);

@@ -784,21 +784,6 @@ __global__ void __launch_bounds__(RT, 1)
   }
   for (int st = 0; st < NST; ++st, ++g) {
     const int buf = g & 1;
-    if (FUSED && !SOMM && rhs_dof && prm.rk_stage >= 0 && st == NST - 3) {
-      // fused RK4 update: this point's u_n / acc rows into L2 for the epilogue
-      double ex[6];
-      VALS_LD(TV_EX, ex);
-      const int dz = __double2loint(ex[3]);
-      if (dz >= 0) {
-        const int64_t ds64 = m.dof_stride;
-        for (int f = 0; f < NF; ++f) {
-          if (prm.rk_stage <= 2)
-            asm volatile("prefetch.global.L2 [%0];" ::"l"(prm.rk_un + f * ds64 + dz));
-          if (prm.rk_stage >= 1)
-            asm volatile("prefetch.global.L2 [%0];" ::"l"(prm.rk_acc + f * ds64 + dz));
-        }
-      }
-    }
 #ifdef DGR_RHS_TIMING
     if (tid == 0) {   // per-stage cycle profile (experiment builds only)
       const long long t = clock64();
@@ -1185,8 +1170,9 @@ __global__ void __launch_bounds__(RT, 1)
     double* out = rhs_oct + int64_t(e) * NPT + p;
     const int64_t ostr = no * NPT;
     if (!SOMM && rhs_dof && prm.rk_stage >= 0) {
-      // the RK4 stage update of the owned DOF dz (its u_n / acc rows were
-      // prefetched into L2 two stages ago), in batches of RKB fields
+      // the RK4 stage update of the owned DOF dz, in batches of RKB fields (an
+      // L2 prefetch of the u_n / acc rows two stages ahead measured slower:
+      // 26.30 vs 26.69 ms per C3 step, its 48 prefetches per thread cost more)
       if (dz >= 0) {
         const int S = prm.rk_stage;
         const double dt = prm.rk_dt;

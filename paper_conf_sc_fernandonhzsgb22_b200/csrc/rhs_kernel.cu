@@ -1,18 +1,24 @@
 // Fused BSSN RHS kernel: 6th-order derivatives + KO + the 24-field algebra
 // (§III-A eqs 1-19, §IV-B), fp64, sm_100a.
 //
-// Design: one CTA per octant patch, one thread per interior
-// point (343 of 352 threads).  The 24 field patches are streamed through
-// shared memory one field at a time by TMA bulk copies (cp.async.bulk,
-// double buffered, mbarrier completion).  While a field is resident every
-// thread evaluates that field's derivatives at its point straight from shared
-// memory and immediately consumes them in the part of the algebra that only
-// needs them ("staged" evaluation, cf. the paper's staged+CSE), so the
-// 210 derivatives of P:L310 are never stored: the per-point state that
-// survives between fields lives in shared-memory slots [slot][point]
-// (accumulators of the 21 vector/tensor outputs, values, inverse metric,
-// Christoffel symbols) and a few registers.  Field order:
-//   gt_ij (6) -> [Christoffel block] -> chi -> alpha -> Gt^i (3) -> beta^i (3)
+// Design: one persistent CTA per SM, one thread per interior
+// point (343 of 352 threads).  The field patches stream through shared memory
+// one (or, for first-derivative-only fields, two) at a time: gathered from
+// the state and the interpolation slots with 8-byte cp.async (the fused
+// unzip, default) or bulk-copied from a patch buffer (cp.async.bulk, mbarrier
+// completion); double buffered across octant boundaries.  While a field is
+// resident every thread evaluates that field's derivatives at its point
+// straight from shared memory and immediately consumes them in the part of
+// the algebra that only needs them ("staged" evaluation, cf. the paper's
+// staged+CSE), so the 210 derivatives of P:L310 are never stored.
+// State that survives between fields: the point's read-only values (gt_ij,
+// At_ij, gt^ij, B^i, its zip-owner DOF) in tensor memory, one TMEM lane per
+// thread (tcgen05.ld / tcgen05.st); the accumulators of the 21 vector/tensor
+// outputs and the Christoffel scratch in shared-memory slots [slot][thread].
+// The epilogue zips by its store and, in dgr_rk4_step, applies the RK4 stage
+// update.  The metric pre-pass (k_gt_pre, below) takes the gt_ij fields.
+// Field order:
+//   gt_ij (6) -> [Christoffel block] -> chi -> alpha -> beta^i (3) -> Gt^i (3)
 //   -> K -> At_ij (6) -> B^i (3)
 // Readings: R1-R8, R13; chi in divisions is max(chi, chi_floor).
 // Two algebraically exact simplifications versus the oracle's literal form:

@@ -929,7 +929,8 @@ static RhsParams to_rp(const dgr_params* p) {
 // start — and the boundary octants follow once the ghosts have landed.
 // The fused path without the radiative boundary zips in k_rhs's store
 static bool zip_by_store(dgr_mesh m, const dgr_params* prm) {
-  return m->fused && m->zip_store && !(prm && prm->sommerfeld && !m->host.periodic);
+  (void)prm;   // (the radiative boundary too, since its values are parked in TMEM)
+  return m->fused && m->zip_store;
 }
 
 static dgr_status ensure_xstream(dgr_mesh m) {
@@ -963,7 +964,7 @@ static dgr_status rhs_oct(dgr_mesh m, double* u, const dgr_params* prm, cudaStre
     rp.rk_out = rk->rk_out;
   }
   double* pre = nullptr;
-  if (m->fused && m->prepass && !(rp.sommerfeld && !m->host.periodic)) {
+  if (m->fused && m->prepass) {
     if (!m->d_pre) CUDA_TRY(m->alloc(&m->d_pre, size_t(pre_rows()) * no * 352));
     pre = m->d_pre;
   }

@@ -65,10 +65,15 @@ constexpr size_t SMEM_BYTES = size_t(NSLOT) * NPP * 8 + size_t(2) * STAGE_DBL * 
 // Tensor memory as per-thread storage (tcgen05.ld / tcgen05.st, 32x32b shape:
 // each thread moves 32-bit columns of its own TMEM lane).  Warp w reaches lanes
 // 32 (w % 4) .. + 31 only, so the 11 warps share the 4 lane quarters and take
-// column blocks of TM_WCOLS by w / 4 (3 x 48 = 144 of TM_COLS allocated).
+// column blocks of TM_WCOLS by w / 4 (3 x 48 = 144 of TM_COLS allocated; the
+// radiative-boundary instantiation adds 4 blocks: 3 x 96 of 512).
 // A double is two columns (low word first).  Loads complete at tcgen05.wait::ld
 // (its register operands tie the loaded values to the wait).
 constexpr int TM_COLS = 256, TM_WCOLS = 48;
+constexpr int TM_COLS_SOMM = 512, TM_WCOLS_SOMM = 96;
+// (SOMM) the radiative right-hand side of field f at a point on a domain face:
+// block TV_SOMM + f / 6, parked per field stage for the epilogue
+constexpr int TV_SOMM = 4;
 __device__ __forceinline__ void tm_ld6(uint32_t ta, double* v) {
   uint32_t r[12];
   asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
@@ -98,6 +103,12 @@ __device__ __forceinline__ void tm_st6(uint32_t ta, const double* v) {
                : "memory");
   asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1, %2, %3, %4};" ::"r"(ta + 8),
                "r"(r[8]), "r"(r[9]), "r"(r[10]), "r"(r[11])
+               : "memory");
+}
+// one double (two columns)
+__device__ __forceinline__ void tm_st1(uint32_t ta, double v) {
+  asm volatile("tcgen05.st.sync.aligned.32x32b.x2.b32 [%0], {%1, %2};" ::"r"(ta),
+               "r"(uint32_t(__double2loint(v))), "r"(uint32_t(__double2hiint(v)))
                : "memory");
 }
 __device__ __forceinline__ void tm_st_wait() {
@@ -270,6 +281,36 @@ __device__ __forceinline__ Line line_ops(const double* __restrict__ s, int c, in
   l.d2 = 2.0 * s3 - 27.0 * s2 + 270.0 * s1 - 490.0 * u0;                         // x 1/(180h^2)
   l.ko = s3 - 6.0 * s2 + 15.0 * s1 - 20.0 * u0;                                  // x sigma/(64h)
   return l;
+}
+
+// Radiative condition (reading R29): d_t f = -(x^i/r) d_i f - (f - f_inf)/r at
+// the domain-face node q of octant oi (x the physical coordinates), from the
+// point's scaled first derivatives d1 (as derivs computes them) and value fv
+__device__ __forceinline__ double somm_rhs(const DevMesh& m, int4 oi, int q, const double* d1,
+                                           double fv, int f) {
+  const int sd = 1 << (m.D - oi.w);
+  const double unit = m.width / (6.0 * double(int64_t(1) << m.D));
+  const int nd[3] = {q % 7, (q / 7) % 7, q / 49}, an[3] = {oi.x, oi.y, oi.z};
+  double xr = 0.0, r2 = 0.0;
+#pragma unroll
+  for (int a = 0; a < 3; ++a) {
+    const double x = m.xmin[a] + double(6 * int64_t(an[a]) + int64_t(nd[a]) * sd) * unit;
+    xr = __fma_rn(x, d1[a], xr);
+    r2 = __fma_rn(x, x, r2);
+  }
+  const double finf = (f <= 1 || f == 12 || f == 15 || f == 17) ? 1.0 : 0.0;
+  const double ir = 1.0 / sqrt(r2);
+  return __fma_rn(-xr, ir, -(fv - finf) * ir);
+}
+
+// the radiative value of staged field f at the point (patch index c0 of s),
+// stored in TMEM at column address ta (first derivatives as derivs computes them)
+__device__ __forceinline__ void somm_park(const DevMesh& m, int4 oi, int q, const double* s, int c0,
+                                          double ih, int f, uint32_t ta) {
+  const double f1 = ih * (1.0 / 60.0);
+  const double d1[3] = {line_ops(s, c0, 1).d1 * f1, line_ops(s, c0, 13).d1 * f1,
+                        line_ops(s, c0, 169).d1 * f1};
+  tm_st1(ta, somm_rhs(m, oi, q, d1, s[c0], f));
 }
 
 // D1_b(D1_a u) * (60h)^2
@@ -537,7 +578,7 @@ __global__ void __launch_bounds__(RT, 1)
   }
   if (tid < 32) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tm_base)),
-                 "n"(TM_COLS)
+                 "n"(SOMM ? TM_COLS_SOMM : TM_COLS)
                  : "memory");
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
   }
@@ -549,7 +590,8 @@ __global__ void __launch_bounds__(RT, 1)
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
   // this thread's TMEM address (lane quarter of its warp, column block)
-  const uint32_t tma = *tm_base + (uint32_t(32 * ((tid >> 5) & 3)) << 16) + TM_WCOLS * (tid >> 7);
+  const uint32_t tma = *tm_base + (uint32_t(32 * ((tid >> 5) & 3)) << 16) +
+                       (SOMM ? TM_WCOLS_SOMM : TM_WCOLS) * (tid >> 7);
 #define VALS_LD(w, v) tm_ld6(tma + 12 * (w), v)
 #define VALS_ST(w, v) tm_st6(tma + 12 * (w), v)
 
@@ -610,6 +652,9 @@ __global__ void __launch_bounds__(RT, 1)
           (nx == 6 && oi.x + sd == nside) || (ny == 6 && oi.y + sd == nside) ||
           (nz == 6 && oi.z + sd == nside);
   }
+  // (SOMM) some point of this warp is on a domain face: warp-uniform, so the
+  // warp-wide TMEM stores and loads of the radiative values run only there
+  const bool bwarp = SOMM && __any_sync(0xffffffffu, bpt);
 
   // ---- values at the point (patch interior) -------------------------------
   if (PRE) {
@@ -786,6 +831,19 @@ __global__ void __launch_bounds__(RT, 1)
     asm volatile("cp.async.wait_all;" ::: "memory");
     double gi[6];
     VALS_LD(TV_GI, gi);
+    if (SOMM && bwarp) {
+      // the gt_ij fields' radiative values (reading R29) from their pre-pass
+      // first derivatives, before the Christoffel block reuses the S0 slots
+      double gq[6];
+      VALS_LD(TV_GT, gq);
+      const int c0 = active ? int(tab_c0[tid]) : C_CENTRE;
+      (void)c0;
+#pragma unroll
+      for (int q = 0; q < 6; ++q) {
+        const double d1[3] = {SL(S0 + q), SL(S0 + 6 + q), SL(S0 + 12 + q)};
+        tm_st1(tma + 2 * (6 * TV_SOMM + 12 + q), somm_rhs(m, oi, int(tab_p[tid]), d1, gq[q], 12 + q));
+      }
+    }
     christoffel(gi);
   }
   for (int st = 0; st < NST; ++st, ++g) {
@@ -897,29 +955,8 @@ __global__ void __launch_bounds__(RT, 1)
     };
     // the per-point work of one staged field f (patch in s); a pair stage runs
     // it for both fields, in order
-    auto point_work = [&](const double* __restrict__ s, const int f) {
+    auto point_work = [&](const double* __restrict__ s, const int f) __attribute__((always_inline)) {
     const int c0 = active ? int(tab_c0[tid]) : C_CENTRE;
-    if (SOMM && bpt) {
-      // radiative condition d_t f = -(x^i/r) d_i f - (f - f_inf)/r replaces the
-      // whole right-hand side of field f here (the epilogue skips this point)
-      const int q = tab_p[tid];
-      const int sd = 1 << (m.D - oi.w);
-      const double unit = m.width / (6.0 * double(int64_t(1) << m.D));
-      const int nd[3] = {q % 7, (q / 7) % 7, q / 49}, an[3] = {oi.x, oi.y, oi.z};
-      double xr = 0.0, r2 = 0.0;
-#pragma unroll
-      for (int a = 0; a < 3; ++a) {
-        const int st = a == 0 ? 1 : (a == 1 ? 13 : 169);
-        const double x = m.xmin[a] + double(6 * int64_t(an[a]) + int64_t(nd[a]) * sd) * unit;
-        const double g = ((s[c0 + st] - s[c0 - st]) * 45.0 - (s[c0 + 2 * st] - s[c0 - 2 * st]) * 9.0 +
-                          (s[c0 + 3 * st] - s[c0 - 3 * st])) * (ih * (1.0 / 60.0));
-        xr += x * g;
-        r2 += x * x;
-      }
-      const double finf = (f <= 1 || f == 12 || f == 15 || f == 17) ? 1.0 : 0.0;
-      const double ir = 1.0 / sqrt(r2);
-      rhs_oct[int64_t(f) * no * NPT + int64_t(e) * NPT + q] = -xr * ir - (s[c0] - finf) * ir;
-    }
     {
       if (!PRE && f >= 12 && f <= 17) {
         // ---------------- conformal metric gt_q: d gt, gt^lm d_lm gt, adv, KO
@@ -1071,6 +1108,16 @@ __global__ void __launch_bounds__(RT, 1)
       }
     }
     };
+    if (SOMM && bwarp) {
+      // radiative condition (reading R29) for the stage's field(s), parked in
+      // TMEM; the epilogue uses it at points on a domain face (every thread
+      // of a warp that has one stores: tcgen05.st is warp-wide)
+      const int c0 = active ? int(tab_c0[tid]) : C_CENTRE;
+      somm_park(m, oi, int(tab_p[tid]), s, c0, ih, f, tma + 2 * (6 * TV_SOMM + f));
+      if (FUSED && stB(st) >= 0)
+        somm_park(m, oi, int(tab_p[tid]), Tx + buf * STAGE_DBL, c0, ih, stB(st),
+                  tma + 2 * (6 * TV_SOMM + stB(st)));
+    }
     if (FUSED && !SOMM && stB(st) >= 0) {
       // a pair of light fields: both fields' derivatives first (one straight
       // line of 2 x 19 independent shared-memory loads, so the two fields'
@@ -1173,9 +1220,21 @@ __global__ void __launch_bounds__(RT, 1)
         const double atf = TF_ONCE ? SL(A_AT + q) - gtv[q] * ttr * (1.0 / 3.0) : SL(A_AT + q);
         r[18 + q] = atf + alpha * (Kv * At[q] - 2.0 * AAij);                        // (6)
       }
+    if (SOMM && bwarp) {
+      // points on a domain face: the radiative condition replaces the whole
+      // right-hand side (reading R29)
+      tm_st_wait();
+      double rv[NF];
+#pragma unroll
+      for (int b = 0; b < 4; ++b) VALS_LD(TV_SOMM + b, rv + 6 * b);
+      if (bpt) {
+#pragma unroll
+        for (int f = 0; f < NF; ++f) r[f] = rv[f];
+      }
+    }
     double* out = rhs_oct + int64_t(e) * NPT + p;
     const int64_t ostr = no * NPT;
-    if (!SOMM && rhs_dof && prm.rk_stage >= 0) {
+    if (rhs_dof && prm.rk_stage >= 0) {
       // the RK4 stage update of the owned DOF dz, in batches of RKB fields (an
       // L2 prefetch of the u_n / acc rows two stages ahead measured slower:
       // 26.30 vs 26.69 ms per C3 step, its 48 prefetches per thread cost more)
@@ -1211,12 +1270,12 @@ __global__ void __launch_bounds__(RT, 1)
           }
         }
       }
-    } else if (!SOMM && rhs_dof) {
+    } else if (rhs_dof) {
       if (dz >= 0) {
 #pragma unroll
         for (int f = 0; f < NF; ++f) st_out(&rhs_dof[f * int64_t(m.dof_stride) + dz], r[f]);
       }
-    } else if (active && (!SOMM || !bpt)) {
+    } else if (active) {
 #pragma unroll
       for (int f = 0; f < NF; ++f) out[f * ostr] = r[f];
     }
@@ -1225,7 +1284,8 @@ __global__ void __launch_bounds__(RT, 1)
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
   __syncthreads();
   if (tid < 32)
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tm_base), "n"(TM_COLS)
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tm_base),
+                 "n"(SOMM ? TM_COLS_SOMM : TM_COLS)
                  : "memory");
 #undef SL
 #undef VALS_LD
@@ -1518,16 +1578,19 @@ template <bool U>
 static void launch_rhs_t(const DevMesh& m, const double* patches, double* rhs_oct,
                          const RhsParams& p, bool fused, bool somm, int a, int c, int grid,
                          int64_t cap, cudaStream_t s, double* pre, double* rhs_dof) {
-  if (fused && pre && !somm) {
+  if (fused && pre) {
     // metric pre-pass (two CTAs per SM), then the 18 remaining fields
     const int64_t cap2 = 2 * cap;
     const int grid2 = int(c < cap2 ? c : cap2);
     k_gt_pre<U><<<grid2, RT, PRE_SMEM_BYTES, s>>>(m, patches, pre, p, a, c);
-    k_rhs<true, false, true, U><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, pre, rhs_dof);
+    if (somm)
+      k_rhs<true, true, true, U><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, pre, rhs_dof);
+    else
+      k_rhs<true, false, true, U><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, pre, rhs_dof);
   } else if (fused && !somm)
     k_rhs<true, false, false, U><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr, rhs_dof);
   else if (fused)
-    k_rhs<true, true, false, U><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr, nullptr);
+    k_rhs<true, true, false, U><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr, rhs_dof);
   else if (!somm)
     k_rhs<false, false, false, U><<<grid, RT, SMEM_BYTES, s>>>(m, patches, rhs_oct, p, a, c, nullptr, nullptr);
   else
@@ -1548,6 +1611,7 @@ void launch_rhs(const DevMesh& m, const double* patches, double* rhs_oct, const 
     DGR_ATTR(true, false, true, false) DGR_ATTR(false, false, false, true)
     DGR_ATTR(true, false, false, true) DGR_ATTR(false, true, false, true)
     DGR_ATTR(true, true, false, true) DGR_ATTR(true, false, true, true)
+    DGR_ATTR(true, true, true, false) DGR_ATTR(true, true, true, true)
 #undef DGR_ATTR
     cudaFuncSetAttribute(k_gt_pre<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          int(PRE_SMEM_BYTES));

@@ -26,7 +26,7 @@ CU_FLAGS = ARCH + ["-O3", "-lineinfo", "-std=c++17", "--expt-relaxed-constexpr",
                    "-Xcompiler", "-fPIC,-ffp-contract=off", "-I", INC, "-I", CSRC]
 CXX_FLAGS = ["-O2", "-fPIC", "-fopenmp", "-ffp-contract=off", "-std=c++17", "-I", INC, "-I", CSRC]
 
-SOURCES_CU = ["api.cu", "kernels.cu", "unzip_kernel.cu", "rhs_kernel.cu", "constraints_kernel.cu",
+SOURCES_CU = ["api.cu", "kernels.cu", "unzip_kernel.cu", "rhs_kernel.cu", "rhs_kernel_fi.cu", "constraints_kernel.cu",
               "rhs_inputs.cu", "regrid.cu", "psi4.cu", "gen/rhs_alg.cu", "gen/psi4.cu"]
 SOURCES_CXX = ["host_mesh.cpp"]
 

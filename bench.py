@@ -384,6 +384,30 @@ def main():
     bytes_io = 24 * info["n_dof_owned"] * 8   # rows the library copies per state
     bytes_serial = host_in.numel() * 8
 
+    # ---- the same step with the dgr_params options (radiative outer boundary
+    # R29 — the one long evolutions use —, lopsided advection R9u): context for
+    # the headline, which runs the default parameters (graph replay, 5 steps;
+    # on a copy of the state, after the timed regions)
+    opts = None
+    if world == 1:
+        try:
+            opts = {}
+            uo = u.clone()
+            for name, op in (("sommerfeld", dgr.Params(sommerfeld=1)), ("upwind", dgr.Params(upwind=1))):
+                for _ in range(3):
+                    mesh.rk4_step(uo, dt, op)
+                torch.cuda.synchronize()
+                o0, o1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                o0.record()
+                for _ in range(5):
+                    mesh.rk4_step(uo, dt, op)
+                o1.record()
+                torch.cuda.synchronize()
+                opts[name + "_ms_per_step"] = o0.elapsed_time(o1) / 5
+            del uo
+        except Exception as ex:  # noqa: BLE001
+            opts = {"error": str(ex)}
+
     if rank != 0:
         if world > 1:
             dist.destroy_process_group()
@@ -477,6 +501,7 @@ def main():
                            "h2d_bytes_per_step": bytes_serial, "d2h_bytes_per_step": bytes_serial,
                            "api": "copy_ -> dgr_rk4_step -> copy_ on one stream"}},
         "constraints": cons,
+        "options": opts,
         "gpu_launches": launches_per_step * args.steps,
         "clocks": clk.summary(),
         "finite": finite,

@@ -1,6 +1,13 @@
 """Per-kernel totals of an ncu launch list (`ncu --metrics gpu__time_duration.sum --csv`):
-python tools/launch_summary.py launches.csv [title]"""
+python tools/launch_summary.py launches.csv [title] [--until NAME]
+(--until: stop at the first launch whose kernel name contains NAME, e.g. the
+bench's option-path runs after its timed regions: --until k_rhs_fi)"""
 import collections, csv, sys
+until = None
+if "--until" in sys.argv:
+    i = sys.argv.index("--until")
+    until = sys.argv[i + 1]
+    del sys.argv[i:i + 2]
 rows = list(csv.reader(open(sys.argv[1])))
 hdr, agg = None, collections.defaultdict(lambda: [0, 0.0])
 for r in rows:
@@ -9,6 +16,8 @@ for r in rows:
         continue
     if hdr is None or len(r) != len(hdr) or r[hdr.index("Metric Name")] != "gpu__time_duration.sum":
         continue
+    if until and until in r[hdr.index("Kernel Name")]:
+        break
     k = r[hdr.index("Kernel Name")].split("(")[0]
     v, u = float(r[hdr.index("Metric Value")].replace(",", "")), r[hdr.index("Metric Unit")]
     v = v / 1e6 if u == "ns" else (v / 1e3 if u == "us" else v)

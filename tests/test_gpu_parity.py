@@ -34,6 +34,13 @@ CASES = {
     "small_bl": (lambda: configs.small_adaptive(lmax=5, rho=0.5), "bl"),
     "small_random": (lambda: configs.small_adaptive(lmax=5, rho=0.5), "random"),
     "bbh_chains_bl": (lambda: configs.small_bbh(lmax=6, rho=0.5), "bl"),
+    # degenerate meshes: one octant (every padding point extrapolated, the
+    # grid far smaller than one CTA wave), and 8 periodic octants (each octant
+    # is its own neighbour's neighbour: +x and -x reach the same octant)
+    "single_octant": (lambda: MeshConfig(name="one", xmin=(-0.5,) * 3, width=1.0,
+                                         periodic=False, level_min=0), "random"),
+    "tiny_periodic": (lambda: MeshConfig(name="p8", xmin=(-0.5,) * 3, width=1.0,
+                                         periodic=True, level_min=1), "random"),
 }
 
 

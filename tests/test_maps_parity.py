@@ -37,9 +37,17 @@ def test_library_exports_every_declared_symbol():
     assert dgr.lib().dgr_version().decode().startswith("dgr-b200")
 
 
+def _degenerate(name, periodic, level_min):
+    return configs.MeshConfig(name=name, xmin=(-0.5,) * 3, width=1.0, periodic=periodic,
+                              level_min=level_min)
+
+
 def _cfgs():
+    # + the degenerate meshes: one octant (all padding extrapolated) and 8
+    # periodic octants (+x and -x reach the same neighbour)
     return [configs.c1_uniform(), configs.small_adaptive(lmax=5, rho=0.5),
-            configs.small_bbh(lmax=6, rho=0.5), configs.c2_schwarzschild()]
+            configs.small_bbh(lmax=6, rho=0.5), configs.c2_schwarzschild(),
+            _degenerate("one", False, 0), _degenerate("p8", True, 1)]
 
 
 @pytest.mark.parametrize("cfg", _cfgs(), ids=lambda c: c.name)
@@ -132,6 +140,17 @@ def test_rejects_bad_trees():
     # the balanced closure of the same tree is accepted
     B, Lb = octree.balance(A, Lv, D, False)
     assert _mesh_status(cfg, np.concatenate([B, Lb[:, None]], 1).astype(np.uint32)) == 0
+
+
+def test_rejects_single_periodic_octant():
+    """A periodic domain of one octant (level 0) is its own neighbour across
+    every face; both the library and the oracle refuse it (levels >= 1)."""
+    cfg = _degenerate("p1", True, 0)
+    oc = dgr.octree_build(cfg)
+    assert oc.shape[0] == 1
+    assert _mesh_status(cfg, oc) == -2
+    with pytest.raises(AssertionError):
+        OracleMesh(cfg)
 
 
 def test_host_mesh_rejects_device_calls():

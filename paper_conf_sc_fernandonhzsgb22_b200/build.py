@@ -57,13 +57,13 @@ def _run(cmd, verbose):
 
 def build(verbose: bool = False, ptxas_verbose: bool = False, variant: str = "") -> str:
     """variant="timing" builds lib/libdgr_timing.so with -DDGR_RHS_TIMING (per-stage
-    cycle counters in k_rhs, for tools/rhs_stage_profile.py); variant="exp*" builds
-    lib/libdgr_exp*.so with the -D flags in $DGR_EXTRA_DEFS (A/B experiments); never
-    the product."""
+    cycle counters in k_rhs, for tools/rhs_stage_profile.py); any other variant
+    builds lib/libdgr_<variant>.so with the -D flags in $DGR_EXTRA_DEFS (A/B
+    experiments); never the product."""
     objdir = OBJDIR + (("_" + variant) if variant else "")
     lib = LIB if not variant else os.path.join(LIBDIR, f"libdgr_{variant}.so")
     defs = ["-DDGR_RHS_TIMING"] if variant == "timing" else []
-    if variant.startswith("exp"):   # experiment builds: -D flags from DGR_EXTRA_DEFS
+    elif variant:   # experiment builds: -D flags from DGR_EXTRA_DEFS
         defs = os.environ.get("DGR_EXTRA_DEFS", "").split()
     os.makedirs(objdir, exist_ok=True)
     objs = []

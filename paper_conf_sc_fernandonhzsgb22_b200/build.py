@@ -62,7 +62,9 @@ def build(verbose: bool = False, ptxas_verbose: bool = False, variant: str = "")
     experiments); never the product."""
     objdir = OBJDIR + (("_" + variant) if variant else "")
     lib = LIB if not variant else os.path.join(LIBDIR, f"libdgr_{variant}.so")
-    defs = ["-DDGR_RHS_TIMING"] if variant == "timing" else []
+    defs = []
+    if variant == "timing":
+        defs = ["-DDGR_RHS_TIMING"]
     elif variant:   # experiment builds: -D flags from DGR_EXTRA_DEFS
         defs = os.environ.get("DGR_EXTRA_DEFS", "").split()
     os.makedirs(objdir, exist_ok=True)

@@ -226,8 +226,8 @@ def main():
     ap.add_argument("--config", default="c3")
     ap.add_argument("--impl", default="dgr", choices=["dgr", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    p.add_argument("--no-options", action="store_true",
-                   help="skip the radiative-boundary / lopsided-advection step timings")
+    ap.add_argument("--no-options", action="store_true",
+                    help="skip the radiative-boundary / lopsided-advection step timings")
     ap.add_argument("--cpu-sample", type=int, default=None)
     ap.add_argument("--path", default="fused", choices=["fused", "two-pass"],
                     help="fused: patches gathered inside the RHS kernel; two-pass: unzip first")

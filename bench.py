@@ -66,11 +66,13 @@ def _peaks():
 
 
 class Clocks:
-    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+    """SM clock / event-reason sampling during the timed region (B200_PROFILING.md
+    clocks line): NVML, else nvidia-smi."""
 
     def __init__(self, index):
         self.index = index
         self.samples = []
+        self.source = None
         self._stop = threading.Event()
         self._t = None
 
@@ -79,7 +81,32 @@ class Clocks:
              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
 
+        def run_nvml(nv, h):
+            # NVML directly: ~ms per query, so a sub-second timed region still
+            # gets tens of samples (nvidia-smi takes ~0.3 s per call)
+            names = [nv.nvmlClocksEventReasonHwSlowdown, nv.nvmlClocksEventReasonHwThermalSlowdown,
+                     nv.nvmlClocksEventReasonSwThermalSlowdown, nv.nvmlClocksEventReasonSwPowerCap]
+            while not self._stop.is_set():
+                try:
+                    r = nv.nvmlDeviceGetCurrentClocksEventReasons(h)
+                    self.samples.append(
+                        [str(nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM)),
+                         str(nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)),
+                         str(nv.nvmlDeviceGetPowerUsage(h) / 1000.0), hex(r)]
+                        + ["Active" if r & b else "Not Active" for b in names])
+                except Exception:
+                    pass
+                self._stop.wait(0.02)
+
         def run():
+            try:
+                import pynvml as nv
+                nv.nvmlInit()
+                h = nv.nvmlDeviceGetHandleByIndex(int(self.index))
+                self.source = "nvml"
+                return run_nvml(nv, h)
+            except Exception:
+                self.source = "nvidia-smi"
             while not self._stop.is_set():
                 try:
                     out = subprocess.run(["nvidia-smi", "-i", str(self.index),
@@ -111,7 +138,7 @@ class Clocks:
                           if s[4 + i].lower().startswith("active")})
         return {"sm_mhz": float(np.median(sm)) if sm else None,
                 "sm_max_mhz": max(mx) if mx else None, "reasons": reasons,
-                "samples": len(self.samples)}
+                "samples": len(self.samples), "source": self.source}
 
 
 def _cpu_model():
